@@ -1,0 +1,170 @@
+/*
+ * lasagna.h — C ABI of the B200-native LaSAGNA hot path (all-pair suffix-prefix overlaps
+ * and the greedy string graph; Goswami et al., IPDPS 2018 = PAPER.md).
+ *
+ * Citations: "P:L<n>" is PAPER.md line n; R<k> is reading k in DESIGN.md.
+ *
+ * Conventions (every entry point):
+ *   - extern "C"; plain pointers and sizes only.  `stream` is a cudaStream_t (NULL = legacy
+ *     default stream) on the CURRENT device; all device work is stream-ordered on it.
+ *   - The caller owns every buffer.  The library allocates no device memory: scratch comes
+ *     from a caller-provided workspace whose size the caller obtains first (workspace == NULL
+ *     -> *workspace_bytes is set and nothing runs).  Device pointers must be 256-byte aligned
+ *     (any torch CUDA tensor's data_ptr() is).
+ *   - Arguments are validated before any launch; on error nothing has been launched (except
+ *     LASAGNA_ECUDA / LASAGNA_ENOSPC, after which outputs are unspecified).
+ *   - Calls that produce host-side outputs (n_pairs, stats, first_bad on the host) synchronise
+ *     `stream` before returning; all others are asynchronous.
+ *   - Errors are returned, never thrown or aborted; lasagna_last_error() gives the text
+ *     (thread-local; valid until this thread's next lasagna_* call).
+ *   - Reentrant across streams and devices (no global mutable state besides the thread-local
+ *     error text).
+ *
+ * Terms:
+ *   reads r_0..r_{n-1}, each exactly L bases (R14); oriented vertex v = 2i+o with
+ *   seq(2i) = r_i and seq(2i+1) = reverse complement of r_i (R8); V = 2n.
+ *   Base code c = (ascii >> 1) & 3: A=0 C=1 T=2 G=3 (R1, Fig. 5); complement c^2.
+ *   Fingerprint F(s) = sum_k c(s_k) * 5^(|s|-1-k) mod (2^61 - 1) (R2, R4).
+ *   Read-end pair (l, a, b), a < b: suffix_l(seq(a)) == prefix_l(seq(b^1)), different reads,
+ *   l in [l_min, L-1] (R5, R9); its directed edges are a -> b^1 and its
+ *   complement b -> a^1.
+ */
+#ifndef LASAGNA_H
+#define LASAGNA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define LASAGNA_API __attribute__((visibility("default")))
+#else
+#define LASAGNA_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    LASAGNA_OK = 0,
+    LASAGNA_EINVAL = 1, /* NULL/misaligned pointer, L < 2 or L > 256, l_min < 1 or >= L,
+                           host pointer that is not page-locked, unsupported bit range    */
+    LASAGNA_ERANGE = 2, /* 2n > 0xFFFFFFFE: vertex ids must fit u32 with NONE reserved
+                           ("4-byte vertex-ID")                               */
+    LASAGNA_ENOSPC = 3, /* workspace or output capacity too small; the needed size is
+                           reported through the size argument                           */
+    LASAGNA_ECUDA = 4   /* a CUDA call failed; see lasagna_last_error()                   */
+} lasagna_status;
+
+#define LASAGNA_NONE 0xFFFFFFFFu /* succ[] value of a read end without an edge */
+
+LASAGNA_API const char *lasagna_last_error(void);
+
+/* u64 words per packed read (the row stride of `packed`): ceil(L/32) rounded up to 1, 2, 4
+ * or 8 so that a read is one aligned 8/16/32/64-byte unit (L <= 128: one 32 B sector). */
+LASAGNA_API uint32_t lasagna_words_per_read(uint32_t L);
+
+/* ---------------------------------------------------------------------------------------
+ * a1 — stage + 2-bit pack ("batches of reads are loaded in the GPU"; P:L61-67 the
+ * host->device level of the two-level streaming model; encoding R1).
+ *   ascii     n*L bytes, read i at ascii + i*L, no separators; bytes in ACGTacgt.  Device
+ *             memory, or PAGE-LOCKED host memory (read in place over PCIe by the kernel:
+ *             zero-copy staging).  Pageable host memory -> LASAGNA_EINVAL.
+ *   packed    device u64 [n][lasagna_words_per_read(L)]: base k of read i in bits
+ *             [2(k mod 32), 2(k mod 32)+2) of word k/32; unused bits and padding words 0.
+ *   first_bad device u64 (one word), written asynchronously: UINT64_MAX if every byte is in
+ *             ACGTacgt, else the smallest index of a read holding another byte (R13).  May be
+ *             NULL (no report; packed rows of bad reads are then unspecified).
+ */
+LASAGNA_API lasagna_status lasagna_load_reads(const char *ascii, uint64_t n, uint32_t L, uint64_t *packed,
+                                  uint64_t *first_bad, void *stream);
+
+/* ---------------------------------------------------------------------------------------
+ * a2 — prefix and suffix fingerprints of every oriented read for every length l in
+ * [l_min, L] (Fig. 5/6; both orientations P:L77).  Row k is length l_min + k,
+ * column is the vertex v:
+ *   pfx[k*2n + v] = F(seq(v)[0..l)),  sfx[k*2n + v] = F(seq(v)[L-l..L))   (device u64).
+ * Either output may be NULL.  No reverse complement is materialised: one pass over r gives
+ * F of r's prefixes (Horner) and of r''s suffixes (ascending powers), and the same pass over
+ * the register-reversed read gives the other two.
+ */
+LASAGNA_API lasagna_status lasagna_fingerprints(const uint64_t *packed, uint64_t n, uint32_t L,
+                                    uint32_t l_min, uint64_t *pfx, uint64_t *sfx, void *stream);
+
+/* ---------------------------------------------------------------------------------------
+ * a2-a5 — every read-end pair (the overlap set; Algorithm 2), exact:
+ * fingerprint hits are verified on the packed bases (R12), so the result equals the
+ * definition.  Output sorted by (l descending, a, b) (R6, R7), a < b:
+ *   pair_a, pair_b  device u32[capacity];  pair_l  device u8[capacity]   (any may be NULL
+ *   when capacity == 0: count only).
+ *   *n_pairs        host out: |P|.  If |P| > capacity -> LASAGNA_ENOSPC (first capacity
+ *                   pairs written).
+ * workspace: device scratch of *workspace_bytes bytes; workspace == NULL -> query.
+ */
+LASAGNA_API lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                void *workspace, size_t *workspace_bytes, uint32_t *pair_a,
+                                uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
+                                uint64_t *n_pairs, void *stream);
+
+typedef struct {
+    uint64_t n_pairs;          /* |P|: read-end pairs found (overlap edges / 2)             */
+    uint64_t n_greedy;         /* pairs accepted by the greedy (directed edges / 2)         */
+    uint64_t fp_false_matches; /* table hits whose key bits matched but bases did not (R12) */
+    uint32_t rounds_max;       /* most greedy rounds any length needed                      */
+    uint32_t passes;           /* device passes over the packed reads (length groups, a8)   */
+    uint32_t lengths_per_pass; /* length-group size the planner chose                       */
+    uint32_t key_dir_bits;     /* directory bits D of the sorted tables                     */
+    float ms_table, ms_sort, ms_search, ms_greedy; /* device time per phase (CUDA events)  */
+} lasagna_stats;
+
+/* ---------------------------------------------------------------------------------------
+ * a1-a7 — the greedy string graph ("each vertex ... at most one incoming edge and at
+ * most one outgoing edge"; lengths in descending order P:L152; ties to the smaller
+ * read-end id R7).  Equal, byte for byte, to visiting P in (l desc, a, b) order and
+ * accepting a pair iff neither read end is taken:
+ *   succ  device u32[2n]: succ[a] = b^1 and succ[b] = a^1 for each accepted (l, a, b),
+ *         LASAGNA_NONE elsewhere (the edge a -> b^1 and its complement b -> a^1).
+ *   olen  device u8[2n]:  l for both ends of an accepted pair, 0 elsewhere.
+ *   stats host out, may be NULL (when non-NULL the call synchronises and times phases).
+ * lengths_per_pass: lengths whose tables are built per device pass (a8 semi-streaming);
+ *   0 = all of [l_min, L-1] in one pass.  The call uses the largest group <= this that fits
+ *   *workspace_bytes; the query (workspace == NULL) reports the size for lengths_per_pass.
+ * Returns LASAGNA_ENOSPC with *workspace_bytes raised when a length produced more candidate
+ * pairs than the workspace's pair pool holds (call again with the larger workspace).
+ */
+LASAGNA_API lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t L,
+                                    uint32_t l_min, uint32_t lengths_per_pass, void *workspace,
+                                    size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
+                                    lasagna_stats *stats, void *stream);
+
+/* Planner for the semi-streaming driver (a8): the largest
+ * lengths_per_pass whose workspace fits `budget_bytes`, and that workspace size.  Returns
+ * LASAGNA_ENOSPC when even one length per pass does not fit (*workspace_bytes = minimum). */
+LASAGNA_API lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budget_bytes,
+                            uint32_t *lengths_per_pass, size_t *workspace_bytes);
+
+/* ---------------------------------------------------------------------------------------
+ * Phase entry points (exported for tests and the multi-GPU driver).
+ *
+ * a4 — stable LSD radix sort (K4 P:L144) of `count` u64 keys by bits
+ * [bit_lo, bit_hi) (0 <= bit_lo < bit_hi <= 64), 8-bit digits, one onesweep pass per digit.
+ * keys: device in/out; the sorted keys end in `keys`.  scratch: device u64[count].
+ */
+LASAGNA_API lasagna_status lasagna_sort_u64(uint64_t *keys, uint64_t *scratch, uint64_t count,
+                                uint32_t bit_lo, uint32_t bit_hi, void *workspace,
+                                size_t *workspace_bytes, void *stream);
+
+/* a6 — the greedy claim alone, on a caller-given candidate list: pairs
+ * (pl[i], pa[i], pb[i]) with pa < pb < 2n, no duplicates, any order.  Result equals the
+ * sequential greedy over the list sorted by (l desc, a, b).  succ/olen as above, fully
+ * written.  *rounds (host out, may be NULL) = total locally-dominant rounds used. */
+LASAGNA_API lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, const uint32_t *pa,
+                                    const uint32_t *pb, uint64_t count, void *workspace,
+                                    size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
+                                    uint32_t *rounds, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LASAGNA_H */

@@ -1,0 +1,205 @@
+// common.cuh — device helpers shared by the sm_100a kernels of liblasagna.so.
+// (Nothing here is shared with oracle/: the two sides are independent by construction.)
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <type_traits>
+
+#include "lasagna.h"
+
+namespace lsg {
+
+// ----------------------------------------------------------------- fingerprint arithmetic
+// F(s) = sum_k c_k 5^(|s|-1-k) mod q, q = 2^61 - 1 (R2, R4).
+constexpr uint64_t Q61 = (1ull << 61) - 1;
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+
+// x mod q for any x < 2^64 (Mersenne folding: 2^61 == 1 mod q).
+__device__ __forceinline__ uint64_t mod61(uint64_t x)
+{
+    uint64_t r = (x & Q61) + (x >> 61);
+    return r >= Q61 ? r - Q61 : r;
+}
+
+// Horner step P <- P*5 + c (P < q, c <= 3: 5P + c < 2^64, no 128-bit product needed).
+__device__ __forceinline__ uint64_t horner5(uint64_t P, uint32_t c)
+{
+    return mod61((P << 2) + P + c);
+}
+
+// Ascending-power step S <- S + c * pw (pw = 5^j mod q, pw2 = 2 pw mod q, c <= 3):
+// c*pw = (c&1)pw + (c&2 ? pw2 : 0), sum < 3q < 2^63.
+__device__ __forceinline__ uint64_t addpow(uint64_t S, uint32_t c, uint64_t pw, uint64_t pw2)
+{
+    uint64_t t = S + ((c & 1u) ? pw : 0ull) + ((c & 2u) ? pw2 : 0ull);
+    return mod61(t);
+}
+
+// Table key mixing: a bijection of the 64-bit word (multiplication by an odd constant mod
+// 2^64, Fibonacci hashing), so equal fingerprints <=> equal mixed words, while the TOP bits
+// are uniform even for short lengths where F < 5^l < 2^61 has leading zero bits.
+constexpr uint64_t MIX = 0x9E3779B97F4A7C15ull;
+__device__ __forceinline__ uint64_t mix(uint64_t f) { return f * MIX; }
+
+// ----------------------------------------------------------------- packed reads
+// base k of a read at bits [2(k mod 32), +2) of word k/32 (lasagna.h, a1).
+
+// reverse the 32 2-bit groups of a word
+__device__ __forceinline__ uint64_t rev2(uint64_t x)
+{
+    uint64_t y = __brevll(x);
+    return ((y >> 1) & 0x5555555555555555ull) | ((y & 0x5555555555555555ull) << 1);
+}
+
+// a[] >>= bits (0 <= bits < 64W), zero fill; register-only (no dynamic indexing).
+template <int W>
+__device__ __forceinline__ void shr_words(uint64_t (&a)[W], uint32_t bits)
+{
+    uint32_t ws = bits >> 6, bs = bits & 63;
+#pragma unroll
+    for (int k = 0; k < W - 1; ++k) {
+        if ((uint32_t)k < ws) {
+#pragma unroll
+            for (int j = 0; j < W; ++j) a[j] = (j + 1 < W) ? a[j + 1] : 0ull;
+        }
+    }
+    if (ws >= (uint32_t)W) {
+#pragma unroll
+        for (int j = 0; j < W; ++j) a[j] = 0;
+    }
+    if (bs) {
+#pragma unroll
+        for (int j = 0; j < W; ++j) {
+            uint64_t hi = (j + 1 < W) ? a[j + 1] : 0ull;
+            a[j] = (a[j] >> bs) | (hi << (64 - bs));
+        }
+    }
+}
+
+// keep the low `bits` bits of the W-word integer a[]
+template <int W>
+__device__ __forceinline__ void keep_low(uint64_t (&a)[W], uint32_t bits)
+{
+#pragma unroll
+    for (int j = 0; j < W; ++j) {
+        uint32_t lo = 64u * j;
+        if (bits <= lo) a[j] = 0;
+        else if (bits < lo + 64) a[j] &= (1ull << (bits - lo)) - 1;
+    }
+}
+
+// reverse complement of an L-base packed read (R8: complement = c ^ 2)
+template <int W>
+__device__ __forceinline__ void rc_words(const uint64_t (&x)[W], uint32_t L, uint64_t (&y)[W])
+{
+#pragma unroll
+    for (int j = 0; j < W; ++j) y[W - 1 - j] = rev2(x[j]);
+    shr_words<W>(y, 2u * (32u * W - L));
+#pragma unroll
+    for (int j = 0; j < W; ++j) y[j] ^= 0xAAAAAAAAAAAAAAAAull;
+    keep_low<W>(y, 2u * L);
+}
+
+template <int W>
+__device__ __forceinline__ void load_read(const uint64_t *__restrict__ packed, uint32_t stride,
+                                          uint64_t i, uint64_t (&x)[W])
+{
+    const uint64_t *p = packed + i * stride;
+    if constexpr (W == 4) {
+        ulonglong4 t = *reinterpret_cast<const ulonglong4 *>(p);
+        x[0] = t.x, x[1] = t.y, x[2] = t.z, x[3] = t.w;
+    } else if constexpr (W == 2) {
+        ulonglong2 t = *reinterpret_cast<const ulonglong2 *>(p);
+        x[0] = t.x, x[1] = t.y;
+    } else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) x[j] = p[j];
+    }
+}
+
+// Exact check of the directed overlap (u, v, l): suffix_l(seq(u)) == prefix_l(seq(v))
+// (R12 — every fingerprint hit is verified on the bases).
+template <int W>
+__device__ __forceinline__ bool verify_overlap(const uint64_t *__restrict__ packed,
+                                               uint32_t stride, uint32_t L, uint32_t u,
+                                               uint32_t v, uint32_t l)
+{
+    uint64_t x[W], su[W], y[W], sv[W];
+    load_read<W>(packed, stride, u >> 1, x);
+    load_read<W>(packed, stride, v >> 1, y);
+    if (u & 1) rc_words<W>(x, L, su);
+    else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) su[j] = x[j];
+    }
+    if (v & 1) rc_words<W>(y, L, sv);
+    else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) sv[j] = y[j];
+    }
+    shr_words<W>(su, 2u * (L - l));
+    keep_low<W>(su, 2u * l);
+    keep_low<W>(sv, 2u * l);
+    bool eq = true;
+#pragma unroll
+    for (int j = 0; j < W; ++j) eq &= (su[j] == sv[j]);
+    return eq;
+}
+
+__host__ __device__ inline uint32_t words_for(uint32_t L) { return (L + 31) / 32; }
+
+__host__ __device__ inline uint32_t stride_for(uint32_t L)
+{
+    uint32_t w = words_for(L);
+    return w <= 1 ? 1 : w <= 2 ? 2 : w <= 4 ? 4 : 8;
+}
+
+// ----------------------------------------------------------------- host-side error plumbing
+void set_error(const char *fmt, ...);
+lasagna_status cuda_status(cudaError_t e, const char *what);
+
+#define LSG_CUDA(call)                                                                         \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess) return ::lsg::cuda_status(e_, #call);                           \
+    } while (0)
+
+#define LSG_LAUNCHED(what)                                                                     \
+    do {                                                                                       \
+        cudaError_t e_ = cudaGetLastError();                                                   \
+        if (e_ != cudaSuccess) return ::lsg::cuda_status(e_, what);                            \
+    } while (0)
+
+// W dispatch: calls f(std::integral_constant<int, W>{}) for the read's word count.
+template <typename F>
+lasagna_status dispatch_W(uint32_t L, F &&f)
+{
+    switch (words_for(L)) {
+    case 1: return f(std::integral_constant<int, 1>{});
+    case 2: return f(std::integral_constant<int, 2>{});
+    case 3: return f(std::integral_constant<int, 3>{});
+    case 4: return f(std::integral_constant<int, 4>{});
+    case 5: return f(std::integral_constant<int, 5>{});
+    case 6: return f(std::integral_constant<int, 6>{});
+    case 7: return f(std::integral_constant<int, 7>{});
+    case 8: return f(std::integral_constant<int, 8>{});
+    default: set_error("L=%u out of range", L); return LASAGNA_EINVAL;
+    }
+}
+
+__host__ __device__ __forceinline__ uint64_t min64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+
+inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+inline int num_sms()
+{
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return sms;
+}
+
+} // namespace lsg

@@ -1,0 +1,156 @@
+// fingerprint.cu — a2/a3: Rabin-Karp prefix/suffix fingerprints of every read and its
+// reverse complement (Fig. 5/6) and the length-partitioned key tables.
+//
+// Thread per read, four rolling streams in ONE forward pass (no explicit RC in memory):
+//   stream over r   (x_j = r_j):   pfx_l(r)  = Horner over x_0..x_{l-1}
+//                                  sfx_l(r') = sum_{j<l} (x_j ^ 2) 5^j   (ascending powers)
+//   stream over r'  (y_j = r'_j, r' = RC(r) reversed in registers):
+//                                  pfx_l(r') = Horner over y_0..y_{l-1}
+//                                  sfx_l(r)  = sum_{j<l} (y_j ^ 2) 5^j
+// After base j all four values for length l = j+1 are available together, so the thread
+// stores the pair (vertex 2i, vertex 2i+1) as one 16-byte word: a warp writes 512
+// contiguous bytes per length (fully coalesced), unlike the paper's Hillis-Steele scan
+// (one CTA per read) that was shaped for Kepler's shared memory.
+#include "kernels.cuh"
+
+namespace lsg {
+
+struct FpStreams {
+    uint64_t P0, P1, S0, S1, pw, pw2;
+    __device__ __forceinline__ void init()
+    {
+        P0 = P1 = S0 = S1 = 0;
+        pw = 1;
+        pw2 = 2;
+    }
+    // consume base j of r (ca) and of r' (cb)
+    __device__ __forceinline__ void step(uint32_t ca, uint32_t cb)
+    {
+        P0 = horner5(P0, ca);
+        P1 = horner5(P1, cb);
+        S1 = addpow(S1, ca ^ 2u, pw, pw2);
+        S0 = addpow(S0, cb ^ 2u, pw, pw2);
+        pw = mod61((pw << 2) + pw);
+        pw2 = mod61(pw << 1);
+    }
+};
+
+// Visit lengths l = 1..l_end; call emit(l, st) after base l-1.
+template <int W, typename Emit>
+__device__ __forceinline__ void roll_read(const uint64_t (&x)[W], const uint64_t (&y)[W],
+                                          uint32_t l_end, Emit &&emit)
+{
+    FpStreams st;
+    st.init();
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+        uint64_t a = x[w], b = y[w];
+        const uint32_t k0 = 32u * w;
+        if (k0 >= l_end) break;
+        const uint32_t kn = min(32u, l_end - k0);
+        for (uint32_t j = 0; j < kn; ++j) {
+            st.step((uint32_t)(a & 3u), (uint32_t)(b & 3u));
+            a >>= 2;
+            b >>= 2;
+            emit(k0 + j + 1, st);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- API: raw fingerprints
+template <int W>
+__global__ void __launch_bounds__(256)
+fp_values_kernel(const uint64_t *__restrict__ packed, uint64_t n, uint32_t L, uint32_t l_min,
+                 uint32_t stride, uint64_t *__restrict__ pfx, uint64_t *__restrict__ sfx)
+{
+    const uint64_t V = 2 * n;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t x[W], y[W];
+        load_read<W>(packed, stride, i, x);
+        rc_words<W>(x, L, y);
+        roll_read<W>(x, y, L, [&](uint32_t l, const FpStreams &st) {
+            if (l < l_min) return;
+            const uint64_t off = (uint64_t)(l - l_min) * V + 2 * i;
+            if (pfx) *reinterpret_cast<ulonglong2 *>(pfx + off) = make_ulonglong2(st.P0, st.P1);
+            if (sfx) *reinterpret_cast<ulonglong2 *>(sfx + off) = make_ulonglong2(st.S0, st.S1);
+        });
+    }
+}
+
+lasagna_status launch_fp_values(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                uint64_t *pfx, uint64_t *sfx, cudaStream_t s)
+{
+    if (n == 0) return LASAGNA_OK;
+    const uint32_t stride = stride_for(L);
+    return dispatch_W(L, [&](auto wc) -> lasagna_status {
+        constexpr int W = decltype(wc)::value;
+        uint64_t blocks = std::min<uint64_t>(ceil_div(n, 256), (uint64_t)num_sms() * 16);
+        fp_values_kernel<W><<<(unsigned)blocks, 256, 0, s>>>(packed, n, L, l_min, stride, pfx, sfx);
+        LSG_LAUNCHED("fp_values_kernel");
+        return LASAGNA_OK;
+    });
+}
+
+// ---------------------------------------------------------------- key tables (a2 + a3)
+// For each length l in the group [l_lo, l_hi] (segment s = l - l_lo), every vertex v:
+//   tab[s*V + v]  = (mix(pfx_l(v)) & ~vmask) | v      prefix table entry: key bits | vid
+//   sfxk[s*V + v] =  mix(sfx_l(v)) & ~vmask           query key of v's suffix
+// plus the histogram of the first LSD digit of the tab keys per segment (onesweep's
+// upfront histogram), accumulated in shared memory and flushed once per CTA.
+
+template <int W>
+__global__ void __launch_bounds__(256)
+table_kernel(TableArgs a)
+{
+    extern __shared__ uint32_t shist[]; // [G][256]
+    const uint32_t G = a.l_hi - a.l_lo + 1;
+    for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x) shist[t] = 0;
+    __syncthreads();
+    const uint64_t V = 2 * a.n;
+    const uint64_t keep = ~((1ull << a.vbits) - 1);
+    const uint32_t dmask = (1u << a.d_bits) - 1;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t x[W], y[W];
+        load_read<W>(a.packed, a.stride, i, x);
+        rc_words<W>(x, a.L, y);
+        roll_read<W>(x, y, a.l_hi, [&](uint32_t l, const FpStreams &st) {
+            if (l < a.l_lo) return;
+            const uint32_t s = l - a.l_lo;
+            const uint64_t off = (uint64_t)s * V + 2 * i;
+            const uint64_t k0 = (mix(st.P0) & keep) | (2 * i);
+            const uint64_t k1 = (mix(st.P1) & keep) | (2 * i + 1);
+            *reinterpret_cast<ulonglong2 *>(a.tab + off) = make_ulonglong2(k0, k1);
+            *reinterpret_cast<ulonglong2 *>(a.sfxk + off) =
+                make_ulonglong2(mix(st.S0) & keep, mix(st.S1) & keep);
+            atomicAdd(&shist[s * 256 + (uint32_t)((k0 >> a.d_shift) & dmask)], 1u);
+            atomicAdd(&shist[s * 256 + (uint32_t)((k1 >> a.d_shift) & dmask)], 1u);
+        });
+    }
+    __syncthreads();
+    for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x)
+        if (shist[t]) atomicAdd(&a.hist[t], shist[t]);
+}
+
+lasagna_status launch_table(const TableArgs &args, cudaStream_t s)
+{
+    if (args.n == 0) return LASAGNA_OK;
+    const uint32_t G = args.l_hi - args.l_lo + 1;
+    const size_t smem = (size_t)G * 256 * sizeof(uint32_t);
+    return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
+        constexpr int W = decltype(wc)::value;
+        if (smem > 48 * 1024)
+            LSG_CUDA(cudaFuncSetAttribute(table_kernel<W>,
+                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        int per_sm = 0;
+        LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, table_kernel<W>, 256, smem));
+        if (per_sm < 1) per_sm = 1;
+        uint64_t blocks = std::min<uint64_t>(ceil_div(args.n, 256), (uint64_t)num_sms() * per_sm);
+        table_kernel<W><<<(unsigned)blocks, 256, smem, s>>>(args);
+        LSG_LAUNCHED("table_kernel");
+        return LASAGNA_OK;
+    });
+}
+
+} // namespace lsg

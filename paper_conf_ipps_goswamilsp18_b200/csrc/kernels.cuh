@@ -1,0 +1,84 @@
+// kernels.cuh — argument structs and host launchers shared between the translation units
+// of liblasagna.so (pack.cu, fingerprint.cu, sort.cu, search.cu, greedy.cu, lasagna.cu).
+#pragma once
+
+#include "common.cuh"
+
+namespace lsg {
+
+// ---- a1 (pack.cu)
+lasagna_status launch_pack(const char *ascii, uint64_t n, uint32_t L, uint64_t *packed,
+                           uint64_t *first_bad, cudaStream_t s);
+
+// ---- a2/a3 (fingerprint.cu)
+lasagna_status launch_fp_values(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                uint64_t *pfx, uint64_t *sfx, cudaStream_t s);
+
+struct TableArgs {
+    const uint64_t *packed;
+    uint64_t n;
+    uint32_t L, stride;
+    uint32_t l_lo, l_hi;      // group of lengths (segment s = l - l_lo)
+    uint32_t vbits;           // b_v: vertex-id bits at the bottom of a key
+    uint32_t d_shift, d_bits; // first LSD digit (histogram produced on the fly)
+    uint64_t *tab, *sfxk;     // [G][V]
+    uint32_t *hist;           // [G][256]
+};
+lasagna_status launch_table(const TableArgs &a, cudaStream_t s);
+
+// ---- a4 (sort.cu)
+struct SortCtx {
+    unsigned long long *status; // look-back words
+    size_t status_bytes;
+    uint32_t *tile_ctrs;        // [SORT_CTRS]
+    uint32_t epoch;             // last used
+};
+constexpr uint32_t SORT_CTRS = 4096;
+size_t sort_status_bytes(uint64_t seg_len, uint32_t n_seg);
+lasagna_status sort_ctx_reset(SortCtx &c, cudaStream_t s);
+void digit_plan(uint32_t lo, uint32_t hi, uint32_t *P, uint32_t *shifts, uint32_t *bits);
+lasagna_status sort_segments(uint64_t *bufs[2], uint64_t seg_len, uint32_t n_seg, uint32_t lo,
+                             uint32_t hi, uint32_t *hist, bool hist0_ready, SortCtx &ctx,
+                             cudaStream_t s, int *which);
+
+// ---- a5 (search.cu)
+lasagna_status launch_dir(const uint64_t *tab, uint64_t V, uint32_t n_seg, uint32_t D,
+                          uint32_t *dir, cudaStream_t s);
+struct SearchArgs {
+    const uint64_t *packed;
+    const uint64_t *tab;   // sorted table of this length (V entries)
+    const uint64_t *sfxk;  // query keys of this length (V entries)
+    const uint32_t *dir;   // 2^D + 1 entries
+    uint64_t V;
+    uint32_t L, stride, l, vbits, D;
+    const uint8_t *claimed;    // optional: skip claimed read ends (pruning), may be null
+    unsigned long long *pairs; // out pool: (a << 32) | b
+    unsigned long long cap;
+    unsigned long long *count; // pool fill (may exceed cap: overflow)
+    unsigned long long *false_matches;
+};
+lasagna_status launch_search(const SearchArgs &a, cudaStream_t s);
+lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsigned long long *count,
+                                    uint64_t m, unsigned long long cap, uint32_t vbits,
+                                    uint64_t *keys, cudaStream_t s);
+lasagna_status launch_keys_to_output(const uint64_t *keys, uint64_t m, uint32_t vbits, uint8_t l,
+                                     uint32_t *pa, uint32_t *pb, uint8_t *pl, cudaStream_t s);
+
+// ---- a6/a7 (greedy.cu)
+struct GreedyBufs {
+    unsigned long long *pool, *pool2; // pair lists (ping-pong)
+    unsigned long long *cnt, *cnt2;   // their fills (device)
+    unsigned long long *accepted;     // running total (device)
+    uint32_t *best0, *best1;
+    uint8_t *claimed;
+    unsigned long long cap;
+};
+lasagna_status greedy_length(GreedyBufs &g, uint64_t m, uint8_t l, uint32_t *succ, uint8_t *olen,
+                             cudaStream_t s, uint32_t *rounds_out);
+lasagna_status launch_gather_pairs(const uint64_t *order, uint64_t off, uint64_t m,
+                                   const uint32_t *pa, const uint32_t *pb,
+                                   unsigned long long *pool, unsigned long long *cnt,
+                                   cudaStream_t s);
+lasagna_status launch_lkeys(const uint8_t *pl, uint64_t count, uint64_t *keys, cudaStream_t s);
+
+} // namespace lsg

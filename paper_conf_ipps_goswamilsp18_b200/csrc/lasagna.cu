@@ -1,0 +1,744 @@
+// lasagna.cu — the C ABI (include/lasagna.h): argument validation, the workspace planner of
+// the semi-streaming driver (a8) and the per-length-group orchestration of a2..a7.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+
+#include "kernels.cuh"
+
+namespace lsg {
+
+// ------------------------------------------------------------------ errors
+static thread_local char g_err[512] = "";
+
+void set_error(const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof g_err, fmt, ap);
+    va_end(ap);
+}
+
+lasagna_status cuda_status(cudaError_t e, const char *what)
+{
+    set_error("%s: %s (%s)", what, cudaGetErrorString(e), cudaGetErrorName(e));
+    return LASAGNA_ECUDA;
+}
+
+// ------------------------------------------------------------------ planning
+// Geometry of the key tables:
+//   key = (mix(F) top (64 - vbits) bits) << vbits | vertex id,  vbits = ceil(log2 V)
+//   sorted by the top D = vbits - 3 key bits (directory buckets of 4-8 entries on average)
+struct Geometry {
+    uint64_t n, V;
+    uint32_t L, l_min, n_len, vbits, D;
+};
+
+static uint32_t ceil_log2(uint64_t x)
+{
+    uint32_t b = 0;
+    while ((1ull << b) < x) ++b;
+    return b;
+}
+
+static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
+{
+    Geometry g;
+    g.n = n;
+    g.V = 2 * n;
+    g.L = L;
+    g.l_min = l_min;
+    g.n_len = L - l_min; // lengths l_min .. L-1 (R5: the l = L partition is dropped)
+    g.vbits = std::max<uint32_t>(1, ceil_log2(g.V));
+    int D = (int)g.vbits - 3;
+    g.D = (uint32_t)std::min(28, std::max(1, D));
+    return g;
+}
+
+static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct Layout {
+    uint32_t G;          // lengths per group
+    uint64_t pool_cap;   // pair pool capacity (pairs)
+    size_t tabA, tabB, sfxk, dir, status, hist, ctrs, pool, pool2, best0, best1, claimed, keys,
+        keys2, total;
+};
+
+constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
+
+static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
+{
+    Layout l;
+    l.G = G;
+    l.pool_cap = pool_cap;
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        size_t o = off;
+        off += align256(bytes);
+        return o;
+    };
+    const size_t tabb = (size_t)G * g.V * 8;
+    l.tabA = take(tabb);
+    l.tabB = take(tabb);
+    l.sfxk = take(tabb);
+    l.dir = take((size_t)G * ((1ull << g.D) + 1) * 4);
+    size_t st = std::max(sort_status_bytes(g.V, G), sort_status_bytes(pool_cap, 1));
+    l.status = take(st);
+    l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
+    l.ctrs = take(CTR_BYTES);
+    l.pool = take(pool_cap * 8);
+    l.pool2 = take(pool_cap * 8);
+    if (greedy) {
+        l.best0 = take(g.V * 4);
+        l.best1 = take(g.V * 4);
+        l.claimed = take(g.V);
+        l.keys = l.keys2 = 0;
+    } else {
+        l.best0 = l.best1 = l.claimed = 0;
+        l.keys = l.pool;  // overlaps: compact keys sorted in place of the pool...
+        l.keys2 = l.pool2; // ...with pool2 as the sort scratch
+    }
+    l.total = off;
+    return l;
+}
+
+static uint64_t default_pool_cap(const Geometry &g)
+{
+    return std::max<uint64_t>(g.V / 8, 1ull << 20);
+}
+
+// ------------------------------------------------------------------ validation
+static bool is_device_ptr(const void *p)
+{
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+static lasagna_status check_shape(uint64_t n, uint32_t L, uint32_t l_min)
+{
+    if (L < 2 || L > 256) {
+        set_error("L=%u out of range [2, 256]", L);
+        return LASAGNA_EINVAL;
+    }
+    if (l_min < 1 || l_min >= L) {
+        set_error("l_min=%u out of range [1, L-1]", l_min);
+        return LASAGNA_EINVAL;
+    }
+    if (n > 0x7FFFFFFFull) {
+        set_error("2n=%llu exceeds 0xFFFFFFFE vertex ids", (unsigned long long)(2 * n));
+        return LASAGNA_ERANGE;
+    }
+    return LASAGNA_OK;
+}
+
+static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+// ------------------------------------------------------------------ the group pipeline
+struct Run {
+    Geometry g;
+    Layout lay;
+    char *ws;
+    cudaStream_t s;
+    SortCtx sctx;
+    uint64_t *tab[2];
+    uint64_t *sfxk;
+    uint32_t *dir, *hist;
+    unsigned long long *ctr64; // [0] pool count, [1] false matches, [2] accepted, [3] cnt2
+    unsigned long long *pool, *pool2;
+    template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
+    void bind(void *workspace)
+    {
+        ws = (char *)workspace;
+        tab[0] = at<uint64_t>(lay.tabA);
+        tab[1] = at<uint64_t>(lay.tabB);
+        sfxk = at<uint64_t>(lay.sfxk);
+        dir = at<uint32_t>(lay.dir);
+        hist = at<uint32_t>(lay.hist);
+        sctx.status = at<unsigned long long>(lay.status);
+        sctx.status_bytes =
+            std::max(sort_status_bytes(g.V, lay.G), sort_status_bytes(lay.pool_cap, 1));
+        sctx.tile_ctrs = at<uint32_t>(lay.ctrs);
+        sctx.epoch = 0;
+        ctr64 = reinterpret_cast<unsigned long long *>(ws + lay.ctrs + 4096 * 4);
+        pool = at<unsigned long long>(lay.pool);
+        pool2 = at<unsigned long long>(lay.pool2);
+    }
+};
+
+struct PhaseTimer {
+    bool on;
+    cudaStream_t s;
+    cudaEvent_t ev[2];
+    float *acc;
+    lasagna_status start(float *a)
+    {
+        if (!on) return LASAGNA_OK;
+        acc = a;
+        LSG_CUDA(cudaEventRecord(ev[0], s));
+        return LASAGNA_OK;
+    }
+    lasagna_status stop()
+    {
+        if (!on) return LASAGNA_OK;
+        LSG_CUDA(cudaEventRecord(ev[1], s));
+        LSG_CUDA(cudaEventSynchronize(ev[1]));
+        float ms = 0;
+        LSG_CUDA(cudaEventElapsedTime(&ms, ev[0], ev[1]));
+        *acc += ms;
+        return LASAGNA_OK;
+    }
+};
+
+// Build + sort the key tables of lengths [l_lo, l_hi]; returns which tab buffer is sorted.
+static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo, uint32_t l_hi,
+                                  int *which, PhaseTimer &tm, lasagna_stats *st)
+{
+    const Geometry &g = r.g;
+    const uint32_t G = l_hi - l_lo + 1;
+    uint32_t P, shifts[8], bits[8];
+    digit_plan(64 - g.D, 64, &P, shifts, bits);
+    LSG_CUDA(cudaMemsetAsync(r.hist, 0, (size_t)G * 256 * 4, r.s));
+    TableArgs ta;
+    ta.packed = packed;
+    ta.n = g.n;
+    ta.L = g.L;
+    ta.stride = stride_for(g.L);
+    ta.l_lo = l_lo;
+    ta.l_hi = l_hi;
+    ta.vbits = g.vbits;
+    ta.d_shift = shifts[0];
+    ta.d_bits = bits[0];
+    ta.tab = r.tab[0];
+    ta.sfxk = r.sfxk;
+    ta.hist = r.hist;
+    lasagna_status rc;
+    if ((rc = tm.start(st ? &st->ms_table : nullptr)) != LASAGNA_OK) return rc;
+    if ((rc = launch_table(ta, r.s)) != LASAGNA_OK) return rc;
+    if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+    if ((rc = tm.start(st ? &st->ms_sort : nullptr)) != LASAGNA_OK) return rc;
+    if ((rc = sort_segments(r.tab, g.V, G, 64 - g.D, 64, r.hist, true, r.sctx, r.s, which)) !=
+        LASAGNA_OK)
+        return rc;
+    if ((rc = launch_dir(r.tab[*which], g.V, G, g.D, r.dir, r.s)) != LASAGNA_OK) return rc;
+    if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+    return LASAGNA_OK;
+}
+
+static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, uint32_t l_lo,
+                                    int which, const uint8_t *claimed, uint64_t *m_out)
+{
+    const Geometry &g = r.g;
+    const uint32_t s = l - l_lo;
+    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, sizeof(unsigned long long), r.s));
+    SearchArgs sa;
+    sa.packed = packed;
+    sa.tab = r.tab[which] + (uint64_t)s * g.V;
+    sa.sfxk = r.sfxk + (uint64_t)s * g.V;
+    sa.dir = r.dir + (uint64_t)s * ((1ull << g.D) + 1);
+    sa.V = g.V;
+    sa.L = g.L;
+    sa.stride = stride_for(g.L);
+    sa.l = l;
+    sa.vbits = g.vbits;
+    sa.D = g.D;
+    sa.claimed = claimed;
+    sa.pairs = r.pool;
+    sa.cap = r.lay.pool_cap;
+    sa.count = r.ctr64;
+    sa.false_matches = r.ctr64 + 1;
+    lasagna_status rc = launch_search(sa, r.s);
+    if (rc != LASAGNA_OK) return rc;
+    unsigned long long m = 0;
+    LSG_CUDA(cudaMemcpyAsync(&m, r.ctr64, sizeof(m), cudaMemcpyDeviceToHost, r.s));
+    LSG_CUDA(cudaStreamSynchronize(r.s));
+    *m_out = m;
+    return LASAGNA_OK;
+}
+
+static uint32_t choose_G(const Geometry &g, uint32_t want, size_t bytes, uint64_t cap, bool greedy)
+{
+    uint32_t hi = want ? std::min(want, g.n_len) : g.n_len;
+    hi = std::min<uint32_t>(hi, 64);
+    for (uint32_t G = hi; G >= 1; --G)
+        if (layout(g, G, cap, greedy).total <= bytes) return G;
+    return 0;
+}
+
+} // namespace lsg
+
+using namespace lsg;
+
+// ==================================================================== exported
+extern "C" {
+
+const char *lasagna_last_error(void) { return g_err; }
+
+uint32_t lasagna_words_per_read(uint32_t L) { return stride_for(L); }
+
+lasagna_status lasagna_load_reads(const char *ascii, uint64_t n, uint32_t L, uint64_t *packed,
+                                  uint64_t *first_bad, void *stream)
+{
+    g_err[0] = 0;
+    if (L < 1 || L > 256) {
+        set_error("L=%u out of range", L);
+        return LASAGNA_EINVAL;
+    }
+    if (n > 0x7FFFFFFFull) {
+        set_error("n too large");
+        return LASAGNA_ERANGE;
+    }
+    if (n == 0) {
+        if (first_bad) {
+            cudaStream_t s = (cudaStream_t)stream;
+            unsigned long long v = ~0ull;
+            LSG_CUDA(cudaMemcpyAsync(first_bad, &v, 8, cudaMemcpyHostToDevice, s));
+            LSG_CUDA(cudaStreamSynchronize(s));
+        }
+        return LASAGNA_OK;
+    }
+    if (!ascii || !packed || !aligned(packed, 16) || (first_bad && !aligned(first_bad, 8))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, ascii) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("ascii: not a CUDA-visible pointer");
+        return LASAGNA_EINVAL;
+    }
+    const char *src = ascii;
+    if (at.type == cudaMemoryTypeHost) {
+        if (!at.devicePointer) {
+            set_error("ascii: page-locked host memory is not mapped into the device");
+            return LASAGNA_EINVAL;
+        }
+        src = (const char *)at.devicePointer;
+    } else if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+        set_error("ascii: pageable host memory; pass device or page-locked host memory");
+        return LASAGNA_EINVAL;
+    }
+    if (!is_device_ptr(packed)) {
+        set_error("packed must be device memory");
+        return LASAGNA_EINVAL;
+    }
+    return launch_pack(src, n, L, packed, first_bad, (cudaStream_t)stream);
+}
+
+lasagna_status lasagna_fingerprints(const uint64_t *packed, uint64_t n, uint32_t L,
+                                    uint32_t l_min, uint64_t *pfx, uint64_t *sfx, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n, L, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (n == 0) return LASAGNA_OK;
+    if (!packed || !aligned(packed, 16) || (pfx && !aligned(pfx, 16)) || (sfx && !aligned(sfx, 16))) {
+        set_error("NULL or misaligned pointer (16-byte alignment required)");
+        return LASAGNA_EINVAL;
+    }
+    return launch_fp_values(packed, n, L, l_min, pfx, sfx, (cudaStream_t)stream);
+}
+
+lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budget_bytes,
+                            uint32_t *lengths_per_pass, size_t *workspace_bytes)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n, L, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (!lengths_per_pass || !workspace_bytes) {
+        set_error("NULL output");
+        return LASAGNA_EINVAL;
+    }
+    Geometry g = geometry(n, L, l_min);
+    uint64_t cap = default_pool_cap(g);
+    uint32_t G = choose_G(g, 0, budget_bytes, cap, true);
+    if (G == 0) {
+        *lengths_per_pass = 0;
+        *workspace_bytes = layout(g, 1, cap, true).total;
+        set_error("budget %zu below the one-length workspace %zu", budget_bytes, *workspace_bytes);
+        return LASAGNA_ENOSPC;
+    }
+    *lengths_per_pass = G;
+    *workspace_bytes = layout(g, G, cap, true).total;
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t L,
+                                    uint32_t l_min, uint32_t lengths_per_pass, void *workspace,
+                                    size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
+                                    lasagna_stats *stats, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n, L, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (!workspace_bytes) {
+        set_error("workspace_bytes is NULL");
+        return LASAGNA_EINVAL;
+    }
+    Geometry g = geometry(n, L, l_min);
+    // pool capacity: the default, or more when the caller grew the workspace after ENOSPC
+    uint64_t cap = default_pool_cap(g);
+    const uint32_t G_want = lengths_per_pass ? std::min(lengths_per_pass, g.n_len) : g.n_len;
+    const uint32_t G_req = std::min<uint32_t>(G_want, 64);
+    if (!workspace) {
+        *workspace_bytes = layout(g, G_req, cap, true).total;
+        return LASAGNA_OK;
+    }
+    if (n == 0) {
+        if (stats) memset(stats, 0, sizeof *stats);
+        return LASAGNA_OK;
+    }
+    if (!packed || !succ || !olen || !aligned(packed, 16) || !aligned(succ, 4) ||
+        !aligned(workspace, 256)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    uint32_t G = choose_G(g, G_req, *workspace_bytes, cap, true);
+    if (G == 0) {
+        *workspace_bytes = layout(g, 1, cap, true).total;
+        set_error("workspace too small");
+        return LASAGNA_ENOSPC;
+    }
+    // spare bytes beyond the chosen layout enlarge the pair pool
+    {
+        size_t spare = *workspace_bytes - layout(g, G, cap, true).total;
+        cap += spare / 16 / 2;
+        while (cap > default_pool_cap(g) && layout(g, G, cap, true).total > *workspace_bytes) cap -= cap / 16 + 1;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    Run r;
+    r.g = g;
+    r.lay = layout(g, G, cap, true);
+    r.s = s;
+    r.bind(workspace);
+    uint8_t *claimed = r.at<uint8_t>(r.lay.claimed);
+    GreedyBufs gb;
+    gb.pool = r.pool;
+    gb.pool2 = r.pool2;
+    gb.cnt = r.ctr64;
+    gb.cnt2 = r.ctr64 + 3;
+    gb.accepted = r.ctr64 + 2;
+    gb.best0 = r.at<uint32_t>(r.lay.best0);
+    gb.best1 = r.at<uint32_t>(r.lay.best1);
+    gb.claimed = claimed;
+    gb.cap = cap;
+
+    lasagna_stats st;
+    memset(&st, 0, sizeof st);
+    st.lengths_per_pass = G;
+    st.key_dir_bits = g.D;
+    PhaseTimer tm;
+    tm.on = stats != nullptr;
+    tm.s = s;
+    if (tm.on) {
+        LSG_CUDA(cudaEventCreate(&tm.ev[0]));
+        LSG_CUDA(cudaEventCreate(&tm.ev[1]));
+    }
+    struct EvGuard {
+        PhaseTimer &t;
+        ~EvGuard()
+        {
+            if (t.on) cudaEventDestroy(t.ev[0]), cudaEventDestroy(t.ev[1]);
+        }
+    } evg{tm};
+
+    if ((rc = sort_ctx_reset(r.sctx, s)) != LASAGNA_OK) return rc;
+    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, 8 * sizeof(unsigned long long), s));
+    LSG_CUDA(cudaMemsetAsync(succ, 0xFF, g.V * 4, s));
+    LSG_CUDA(cudaMemsetAsync(olen, 0, g.V, s));
+    LSG_CUDA(cudaMemsetAsync(claimed, 0, g.V, s));
+
+    uint64_t total_pairs = 0;
+    for (int64_t l_hi = (int64_t)L - 1; l_hi >= (int64_t)l_min; l_hi -= G) {
+        const uint32_t l_lo = (uint32_t)std::max<int64_t>(l_min, l_hi - (int64_t)G + 1);
+        int which = 0;
+        if ((rc = build_group(r, packed, l_lo, (uint32_t)l_hi, &which, tm, &st)) != LASAGNA_OK)
+            return rc;
+        ++st.passes;
+        for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
+            uint64_t m = 0;
+            if ((rc = tm.start(&st.ms_search)) != LASAGNA_OK) return rc;
+            // no pruning: the claimed bits are not consulted, so every length's full pair
+            // list is found (|P| = overlap edges / 2 is reported)
+            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr, &m)) != LASAGNA_OK)
+                return rc;
+            if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+            if (m > cap) {
+                uint64_t need = m + m / 4;
+                *workspace_bytes = layout(g, G, need, true).total;
+                set_error("length %lld produced %llu pairs > pool %llu", (long long)l,
+                          (unsigned long long)m, (unsigned long long)cap);
+                return LASAGNA_ENOSPC;
+            }
+            total_pairs += m;
+            uint32_t rounds = 0;
+            if ((rc = tm.start(&st.ms_greedy)) != LASAGNA_OK) return rc;
+            if ((rc = greedy_length(gb, m, (uint8_t)l, succ, olen, s, &rounds)) != LASAGNA_OK)
+                return rc;
+            if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+            st.rounds_max = std::max(st.rounds_max, rounds);
+        }
+    }
+    if (stats) {
+        unsigned long long h[3];
+        LSG_CUDA(cudaMemcpyAsync(h, r.ctr64, sizeof h, cudaMemcpyDeviceToHost, s));
+        LSG_CUDA(cudaStreamSynchronize(s));
+        st.n_pairs = total_pairs;
+        st.fp_false_matches = h[1];
+        st.n_greedy = h[2];
+        *stats = st;
+    }
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                void *workspace, size_t *workspace_bytes, uint32_t *pair_a,
+                                uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
+                                uint64_t *n_pairs, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n, L, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (!workspace_bytes || !n_pairs) {
+        set_error("NULL size/count pointer");
+        return LASAGNA_EINVAL;
+    }
+    Geometry g = geometry(n, L, l_min);
+    uint64_t cap = default_pool_cap(g);
+    const uint32_t G_req = std::min<uint32_t>(g.n_len, 64);
+    if (!workspace) {
+        *workspace_bytes = layout(g, G_req, cap, false).total;
+        return LASAGNA_OK;
+    }
+    *n_pairs = 0;
+    if (n == 0) return LASAGNA_OK;
+    if (!packed || !aligned(packed, 16) || !aligned(workspace, 256) ||
+        (capacity && (!pair_a && !pair_b && !pair_l))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    uint32_t G = choose_G(g, G_req, *workspace_bytes, cap, false);
+    if (G == 0) {
+        *workspace_bytes = layout(g, 1, cap, false).total;
+        set_error("workspace too small");
+        return LASAGNA_ENOSPC;
+    }
+    {
+        size_t spare = *workspace_bytes - layout(g, G, cap, false).total;
+        cap += spare / 16 / 2;
+        while (cap > default_pool_cap(g) && layout(g, G, cap, false).total > *workspace_bytes) cap -= cap / 16 + 1;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    Run r;
+    r.g = g;
+    r.lay = layout(g, G, cap, false);
+    r.s = s;
+    r.bind(workspace);
+    PhaseTimer tm;
+    tm.on = false;
+    if ((rc = sort_ctx_reset(r.sctx, s)) != LASAGNA_OK) return rc;
+    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, 8 * sizeof(unsigned long long), s));
+    uint64_t total = 0;
+    uint64_t worst = 0;
+    for (int64_t l_hi = (int64_t)L - 1; l_hi >= (int64_t)l_min; l_hi -= G) {
+        const uint32_t l_lo = (uint32_t)std::max<int64_t>(l_min, l_hi - (int64_t)G + 1);
+        int which = 0;
+        if ((rc = build_group(r, packed, l_lo, (uint32_t)l_hi, &which, tm, nullptr)) != LASAGNA_OK)
+            return rc;
+        for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
+            uint64_t m = 0;
+            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr, &m)) != LASAGNA_OK)
+                return rc;
+            worst = std::max(worst, m);
+            if (m > cap) { // count only from here on
+                total += m;
+                continue;
+            }
+            if (m && total < capacity) {
+                // sort this length's pairs by (a, b): compact key a << vbits | b
+                uint64_t *keys[2] = {reinterpret_cast<uint64_t *>(r.pool2),
+                                     reinterpret_cast<uint64_t *>(r.pool)};
+                if ((rc = launch_pairs_to_keys(r.pool, r.ctr64, m, cap, g.vbits, keys[0], s)) !=
+                    LASAGNA_OK)
+                    return rc;
+                int which2 = 0;
+                if ((rc = sort_segments(keys, m, 1, 0, 2 * g.vbits, r.hist, false, r.sctx, s,
+                                        &which2)) != LASAGNA_OK)
+                    return rc;
+                const uint64_t take = std::min<uint64_t>(m, capacity - total);
+                if ((rc = launch_keys_to_output(keys[which2], take, g.vbits, (uint8_t)l,
+                                                pair_a ? pair_a + total : nullptr,
+                                                pair_b ? pair_b + total : nullptr,
+                                                pair_l ? pair_l + total : nullptr, s)) != LASAGNA_OK)
+                    return rc;
+            }
+            total += m;
+        }
+    }
+    LSG_CUDA(cudaStreamSynchronize(s));
+    *n_pairs = total;
+    if (worst > cap) {
+        *workspace_bytes = layout(g, G, worst + worst / 4, false).total;
+        set_error("a length produced %llu pairs > pool %llu", (unsigned long long)worst,
+                  (unsigned long long)cap);
+        return LASAGNA_ENOSPC;
+    }
+    if (total > capacity) {
+        set_error("|P| = %llu > capacity %llu", (unsigned long long)total,
+                  (unsigned long long)capacity);
+        return LASAGNA_ENOSPC;
+    }
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_sort_u64(uint64_t *keys, uint64_t *scratch, uint64_t count,
+                                uint32_t bit_lo, uint32_t bit_hi, void *workspace,
+                                size_t *workspace_bytes, void *stream)
+{
+    g_err[0] = 0;
+    if (!workspace_bytes || bit_lo >= bit_hi || bit_hi > 64) {
+        set_error("bad bit range or NULL workspace_bytes");
+        return LASAGNA_EINVAL;
+    }
+    const size_t need = align256(sort_status_bytes(count, 1)) + align256(CTR_BYTES) +
+                        align256(8 * 256 * 4);
+    if (!workspace) {
+        *workspace_bytes = need;
+        return LASAGNA_OK;
+    }
+    if (*workspace_bytes < need) {
+        *workspace_bytes = need;
+        set_error("workspace too small");
+        return LASAGNA_ENOSPC;
+    }
+    if (count == 0) return LASAGNA_OK;
+    if (!keys || !scratch || !aligned(keys, 8) || !aligned(scratch, 8) || !aligned(workspace, 256)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    if (count > 0xFFFFFFFFull) {
+        set_error("count must be < 2^32");
+        return LASAGNA_ERANGE;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    char *ws = (char *)workspace;
+    SortCtx c;
+    c.status = reinterpret_cast<unsigned long long *>(ws);
+    c.status_bytes = sort_status_bytes(count, 1);
+    c.tile_ctrs = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes));
+    uint32_t *hist = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes) + align256(CTR_BYTES));
+    lasagna_status rc = sort_ctx_reset(c, s);
+    if (rc != LASAGNA_OK) return rc;
+    uint64_t *bufs[2] = {keys, scratch};
+    int which = 0;
+    rc = sort_segments(bufs, count, 1, bit_lo, bit_hi, hist, false, c, s, &which);
+    if (rc != LASAGNA_OK) return rc;
+    if (which == 1)
+        LSG_CUDA(cudaMemcpyAsync(keys, scratch, count * 8, cudaMemcpyDeviceToDevice, s));
+    return LASAGNA_OK;
+}
+
+} // extern "C"
+
+extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, const uint32_t *pa,
+                                               const uint32_t *pb, uint64_t count, void *workspace,
+                                               size_t *workspace_bytes, uint32_t *succ,
+                                               uint8_t *olen, uint32_t *rounds, void *stream)
+{
+    g_err[0] = 0;
+    if (!workspace_bytes) {
+        set_error("workspace_bytes is NULL");
+        return LASAGNA_EINVAL;
+    }
+    if (n > 0x7FFFFFFFull) {
+        set_error("2n exceeds 0xFFFFFFFE vertex ids");
+        return LASAGNA_ERANGE;
+    }
+    const uint64_t V = 2 * n;
+    const uint64_t c1 = std::max<uint64_t>(count, 1);
+    // keys, keys2 | pool, pool2 | status | ctrs | hist | best0, best1 | claimed
+    size_t off = 0;
+    auto take = [&](size_t b) {
+        size_t o = off;
+        off += align256(b);
+        return o;
+    };
+    const size_t o_keys = take(c1 * 8), o_keys2 = take(c1 * 8), o_pool = take(c1 * 8),
+                 o_pool2 = take(c1 * 8), o_status = take(sort_status_bytes(c1, 1)),
+                 o_ctrs = take(CTR_BYTES), o_hist = take(8 * 256 * 4), o_best0 = take(V * 4 + 4),
+                 o_best1 = take(V * 4 + 4), o_claimed = take(V + 1);
+    if (!workspace) {
+        *workspace_bytes = off;
+        return LASAGNA_OK;
+    }
+    if (*workspace_bytes < off) {
+        *workspace_bytes = off;
+        set_error("workspace too small");
+        return LASAGNA_ENOSPC;
+    }
+    if (!succ || !olen || !aligned(workspace, 256) || (count && (!pl || !pa || !pb))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    char *ws = (char *)workspace;
+    LSG_CUDA(cudaMemsetAsync(succ, 0xFF, V * 4, s));
+    LSG_CUDA(cudaMemsetAsync(olen, 0, V, s));
+    if (rounds) *rounds = 0;
+    if (count == 0) {
+        LSG_CUDA(cudaStreamSynchronize(s));
+        return LASAGNA_OK;
+    }
+    SortCtx c;
+    c.status = reinterpret_cast<unsigned long long *>(ws + o_status);
+    c.status_bytes = sort_status_bytes(c1, 1);
+    c.tile_ctrs = reinterpret_cast<uint32_t *>(ws + o_ctrs);
+    c.epoch = 0;
+    lasagna_status rc = sort_ctx_reset(c, s);
+    if (rc != LASAGNA_OK) return rc;
+    unsigned long long *ctr64 = reinterpret_cast<unsigned long long *>(ws + o_ctrs + 4096 * 4);
+    LSG_CUDA(cudaMemsetAsync(ctr64, 0, 8 * 8, s));
+    uint8_t *claimed = reinterpret_cast<uint8_t *>(ws + o_claimed);
+    LSG_CUDA(cudaMemsetAsync(claimed, 0, V, s));
+    // group by length, descending: key (255 - l) << 56 | i, one 8-bit LSD pass
+    uint64_t *keys[2] = {reinterpret_cast<uint64_t *>(ws + o_keys),
+                         reinterpret_cast<uint64_t *>(ws + o_keys2)};
+    if ((rc = launch_lkeys(pl, count, keys[0], s)) != LASAGNA_OK) return rc;
+    uint32_t *hist = reinterpret_cast<uint32_t *>(ws + o_hist);
+    int which = 0;
+    if ((rc = sort_segments(keys, count, 1, 56, 64, hist, false, c, s, &which)) != LASAGNA_OK)
+        return rc;
+    uint32_t h[256];
+    LSG_CUDA(cudaMemcpyAsync(h, hist, sizeof h, cudaMemcpyDeviceToHost, s));
+    LSG_CUDA(cudaStreamSynchronize(s));
+    GreedyBufs gb;
+    gb.pool = reinterpret_cast<unsigned long long *>(ws + o_pool);
+    gb.pool2 = reinterpret_cast<unsigned long long *>(ws + o_pool2);
+    gb.cnt = ctr64;
+    gb.cnt2 = ctr64 + 3;
+    gb.accepted = ctr64 + 2;
+    gb.best0 = reinterpret_cast<uint32_t *>(ws + o_best0);
+    gb.best1 = reinterpret_cast<uint32_t *>(ws + o_best1);
+    gb.claimed = claimed;
+    gb.cap = c1;
+    uint64_t pos = 0;
+    uint32_t total_rounds = 0;
+    for (int d = 0; d < 256; ++d) { // digit d = 255 - l: longest lengths first
+        const uint64_t m = h[d];
+        if (!m) continue;
+        const uint8_t l = (uint8_t)(255 - d);
+        if ((rc = launch_gather_pairs(keys[which], pos, m, pa, pb, gb.pool, gb.cnt, s)) != LASAGNA_OK)
+            return rc;
+        uint32_t r = 0;
+        if ((rc = greedy_length(gb, m, l, succ, olen, s, &r)) != LASAGNA_OK) return rc;
+        total_rounds += r;
+        pos += m;
+    }
+    LSG_CUDA(cudaStreamSynchronize(s));
+    if (rounds) *rounds = total_rounds;
+    return LASAGNA_OK;
+}

@@ -1,0 +1,270 @@
+"""Thin Python binding of liblasagna.so (include/lasagna.h) — argument marshalling only.
+
+Every step of the hot path runs in the library's sm_100a kernels; torch only supplies device
+memory (workspaces, outputs), pinned host buffers and the current CUDA stream.  There is no
+CPU fallback: if the shared library cannot be loaded, every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import torch
+
+from . import build as _build
+
+OK, EINVAL, ERANGE, ENOSPC, ECUDA = 0, 1, 2, 3, 4
+NONE = 0xFFFFFFFF
+_NAMES = {0: "OK", 1: "EINVAL", 2: "ERANGE", 3: "ENOSPC", 4: "ECUDA"}
+
+
+class LasagnaError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"lasagna {_NAMES.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("n_pairs", ctypes.c_uint64), ("n_greedy", ctypes.c_uint64),
+                ("fp_false_matches", ctypes.c_uint64), ("rounds_max", ctypes.c_uint32),
+                ("passes", ctypes.c_uint32), ("lengths_per_pass", ctypes.c_uint32),
+                ("key_dir_bits", ctypes.c_uint32), ("ms_table", ctypes.c_float),
+                ("ms_sort", ctypes.c_float), ("ms_search", ctypes.c_float),
+                ("ms_greedy", ctypes.c_float)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load the in-tree liblasagna.so (building it first if sources are newer and nvcc exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.SO
+    try:
+        if _build.stale():
+            _build.build()
+    except RuntimeError:
+        if not os.path.exists(path):
+            raise
+    if not os.path.exists(path):
+        raise LasagnaError(ECUDA, f"{path} missing: run __graft_entry__.build()")
+    L = ctypes.CDLL(path)
+    vp, u64, u32, sz = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_size_t
+    psz = ctypes.POINTER(ctypes.c_size_t)
+    pu64 = ctypes.POINTER(ctypes.c_uint64)
+    pu32 = ctypes.POINTER(ctypes.c_uint32)
+    L.lasagna_last_error.restype = ctypes.c_char_p
+    L.lasagna_words_per_read.argtypes = [u32]
+    L.lasagna_words_per_read.restype = u32
+    sigs = {
+        "lasagna_load_reads": [vp, u64, u32, vp, vp, vp],
+        "lasagna_fingerprints": [vp, u64, u32, u32, vp, vp, vp],
+        "lasagna_overlaps": [vp, u64, u32, u32, vp, psz, vp, vp, vp, u64, pu64, vp],
+        "lasagna_greedy_graph": [vp, u64, u32, u32, u32, vp, psz, vp, vp,
+                                 ctypes.POINTER(_Stats), vp],
+        "lasagna_plan": [u64, u32, u32, sz, pu32, psz],
+        "lasagna_sort_u64": [vp, vp, u64, u32, u32, vp, psz, vp],
+        "lasagna_greedy_pairs": [u64, vp, vp, vp, u64, vp, psz, vp, vp, pu32, vp],
+    }
+    for name, args in sigs.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _check(status: int) -> None:
+    if status != OK:
+        raise LasagnaError(status, lib().lasagna_last_error().decode(errors="replace"))
+
+
+def _stream(device=None) -> int:
+    return torch.cuda.current_stream(device).cuda_stream
+
+
+def _ptr(t: torch.Tensor | None):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def words_per_read(L: int) -> int:
+    return int(lib().lasagna_words_per_read(L))
+
+
+def _workspace(nbytes: int, device) -> torch.Tensor:
+    return torch.empty(max(int(nbytes), 256), dtype=torch.uint8, device=device)
+
+
+# ---------------------------------------------------------------------------- a1
+def load_reads(ascii, device: str | torch.device = "cuda", check: bool = True):
+    """2-bit pack reads on the GPU.  ``ascii``: (n, L) uint8 tensor on the device or in
+    page-locked host memory (read in place by the kernel), or a numpy array (copied into a
+    pinned staging tensor first).  Returns the packed u64 rows as an int64 tensor [n, W]."""
+    if not isinstance(ascii, torch.Tensor):
+        ascii = torch.from_numpy(ascii).pin_memory()
+    if ascii.dtype != torch.uint8 or ascii.dim() != 2:
+        raise ValueError("ascii must be a (n, L) uint8 tensor")
+    ascii = ascii.contiguous()
+    if not ascii.is_cuda and not ascii.is_pinned():
+        ascii = ascii.pin_memory()
+    n, L = ascii.shape
+    dev = ascii.device if ascii.is_cuda else torch.device(device)
+    packed = torch.empty((n, words_per_read(L)), dtype=torch.int64, device=dev)
+    bad = torch.empty(1, dtype=torch.int64, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib().lasagna_load_reads(_ptr(ascii), n, L, _ptr(packed), _ptr(bad), _stream(dev)))
+    if check:
+        b = int(bad.item()) & 0xFFFFFFFFFFFFFFFF
+        if b != 0xFFFFFFFFFFFFFFFF:
+            raise LasagnaError(EINVAL, f"read {b} holds a byte outside ACGTacgt")
+    return packed
+
+
+# ---------------------------------------------------------------------------- a2
+def fingerprints(packed: torch.Tensor, n: int, L: int, l_min: int):
+    """(pfx, sfx) int64 tensors [L - l_min + 1, 2n] holding the u64 fingerprints."""
+    V = 2 * n
+    pfx = torch.empty((L - l_min + 1, V), dtype=torch.int64, device=packed.device)
+    sfx = torch.empty_like(pfx)
+    with torch.cuda.device(packed.device):
+        _check(lib().lasagna_fingerprints(_ptr(packed), n, L, l_min, _ptr(pfx), _ptr(sfx),
+                                          _stream(packed.device)))
+    return pfx, sfx
+
+
+# ---------------------------------------------------------------------------- a2..a5
+def overlaps(packed: torch.Tensor, n: int, L: int, l_min: int, capacity: int | None = None):
+    """All read-end pairs sorted by (l desc, a, b): (pl uint8, pa int32, pb int32) tensors
+    (pa/pb hold u32 vertex ids)."""
+    dev = packed.device
+    ws_bytes = ctypes.c_size_t(0)
+    npairs = ctypes.c_uint64(0)
+    with torch.cuda.device(dev):
+        _check(lib().lasagna_overlaps(_ptr(packed), n, L, l_min, None, ctypes.byref(ws_bytes),
+                                      None, None, None, 0, ctypes.byref(npairs), _stream(dev)))
+        for _ in range(4):
+            ws = _workspace(ws_bytes.value, dev)
+            cap = max(1, int(capacity if capacity is not None else max(1, n)))
+            pa = torch.empty(cap, dtype=torch.int32, device=dev)
+            pb = torch.empty(cap, dtype=torch.int32, device=dev)
+            pl = torch.empty(cap, dtype=torch.uint8, device=dev)
+            st = lib().lasagna_overlaps(_ptr(packed), n, L, l_min, _ptr(ws), ctypes.byref(ws_bytes),
+                                        _ptr(pa), _ptr(pb), _ptr(pl), cap, ctypes.byref(npairs),
+                                        _stream(dev))
+            if st == ENOSPC:
+                if npairs.value > cap:
+                    capacity = npairs.value
+                continue
+            _check(st)
+            m = int(npairs.value)
+            return pl[:m], pa[:m], pb[:m]
+    raise LasagnaError(ENOSPC, "overlaps: could not size workspace/capacity")
+
+
+# ---------------------------------------------------------------------------- a1..a7
+@dataclass
+class GraphResult:
+    succ: torch.Tensor   # int32 [2n] (u32 ids; NONE = -1)
+    olen: torch.Tensor   # uint8 [2n]
+    stats: dict
+
+
+def plan(n: int, L: int, l_min: int, budget_bytes: int):
+    lp = ctypes.c_uint32(0)
+    ws = ctypes.c_size_t(0)
+    st = lib().lasagna_plan(n, L, l_min, budget_bytes, ctypes.byref(lp), ctypes.byref(ws))
+    if st == ENOSPC:
+        return 0, int(ws.value)
+    _check(st)
+    return int(lp.value), int(ws.value)
+
+
+class GreedyGraph:
+    """Reusable greedy-graph runner: owns the workspace (sized once, kept across calls)."""
+
+    def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0,
+                 budget_bytes: int | None = None):
+        self.n, self.L, self.l_min = n, L, l_min
+        self.device = torch.device(device)
+        if lengths_per_pass == 0:
+            if budget_bytes is None:
+                free, _ = torch.cuda.mem_get_info(self.device)
+                budget_bytes = int(free * 0.9)
+            lp, need = plan(n, L, l_min, budget_bytes)
+            if lp == 0:
+                raise LasagnaError(ENOSPC, f"needs {need} bytes of workspace, budget {budget_bytes}")
+            lengths_per_pass = lp
+        self.lengths_per_pass = lengths_per_pass
+        ws = ctypes.c_size_t(0)
+        _check(lib().lasagna_greedy_graph(None, n, L, l_min, lengths_per_pass, None,
+                                          ctypes.byref(ws), None, None, None, None))
+        self.ws_bytes = int(ws.value)
+        self.ws = _workspace(self.ws_bytes, self.device)
+        self.succ = torch.empty(2 * n, dtype=torch.int32, device=self.device)
+        self.olen = torch.empty(2 * n, dtype=torch.uint8, device=self.device)
+
+    def __call__(self, packed: torch.Tensor, stats: bool = True) -> GraphResult:
+        st = _Stats()
+        for _ in range(4):
+            ws = ctypes.c_size_t(self.ws_bytes)
+            with torch.cuda.device(self.device):
+                rc = lib().lasagna_greedy_graph(
+                    _ptr(packed), self.n, self.L, self.l_min, self.lengths_per_pass, _ptr(self.ws),
+                    ctypes.byref(ws), _ptr(self.succ), _ptr(self.olen),
+                    ctypes.byref(st) if stats else None, _stream(self.device))
+            if rc == ENOSPC and ws.value > self.ws_bytes:
+                self.ws_bytes = int(ws.value)
+                self.ws = None
+                self.ws = _workspace(self.ws_bytes, self.device)
+                continue
+            _check(rc)
+            return GraphResult(self.succ, self.olen, st.as_dict() if stats else {})
+        raise LasagnaError(ENOSPC, "greedy_graph: could not size the workspace")
+
+
+def greedy_graph(packed: torch.Tensor, n: int, L: int, l_min: int, lengths_per_pass: int = 0,
+                 stats: bool = True) -> GraphResult:
+    g = GreedyGraph(n, L, l_min, packed.device, lengths_per_pass)
+    r = g(packed, stats)
+    return GraphResult(r.succ.clone(), r.olen.clone(), r.stats)
+
+
+# ---------------------------------------------------------------------------- phase entry points
+def sort_u64(keys: torch.Tensor, bit_lo: int = 0, bit_hi: int = 64) -> torch.Tensor:
+    """Stable LSD sort (in place) of an int64 tensor holding u64 keys, by bits [lo, hi)."""
+    keys = keys.contiguous()
+    dev = keys.device
+    scratch = torch.empty_like(keys)
+    ws_bytes = ctypes.c_size_t(0)
+    with torch.cuda.device(dev):
+        _check(lib().lasagna_sort_u64(_ptr(keys), _ptr(scratch), keys.numel(), bit_lo, bit_hi,
+                                      None, ctypes.byref(ws_bytes), _stream(dev)))
+        ws = _workspace(ws_bytes.value, dev)
+        _check(lib().lasagna_sort_u64(_ptr(keys), _ptr(scratch), keys.numel(), bit_lo, bit_hi,
+                                      _ptr(ws), ctypes.byref(ws_bytes), _stream(dev)))
+    return keys
+
+
+def greedy_pairs(n: int, pl: torch.Tensor, pa: torch.Tensor, pb: torch.Tensor):
+    """Greedy claim on a given candidate list -> (succ int32 [2n], olen uint8 [2n], rounds)."""
+    dev = pa.device
+    count = pa.numel()
+    succ = torch.empty(2 * n, dtype=torch.int32, device=dev)
+    olen = torch.empty(2 * n, dtype=torch.uint8, device=dev)
+    ws_bytes = ctypes.c_size_t(0)
+    rounds = ctypes.c_uint32(0)
+    with torch.cuda.device(dev):
+        _check(lib().lasagna_greedy_pairs(n, None, None, None, count, None, ctypes.byref(ws_bytes),
+                                          None, None, None, _stream(dev)))
+        ws = _workspace(ws_bytes.value, dev)
+        _check(lib().lasagna_greedy_pairs(n, _ptr(pl.contiguous()), _ptr(pa.contiguous()),
+                                          _ptr(pb.contiguous()), count, _ptr(ws),
+                                          ctypes.byref(ws_bytes), _ptr(succ), _ptr(olen),
+                                          ctypes.byref(rounds), _stream(dev)))
+    return succ, olen, int(rounds.value)

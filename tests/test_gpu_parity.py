@@ -1,0 +1,317 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+All integer: the bar is bit-exact.  `-m gpu` tests need a B200; the library-export test runs
+anywhere.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import random
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import readgen
+from oracle import brute
+from tests._util import NONE, check_graph, golden, to_array
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _header_symbols() -> list[str]:
+    with open(os.path.join(ROOT, "include", "lasagna.h")) as f:
+        src = f.read()
+    return sorted(set(re.findall(r"\b(lasagna_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    """The C-ABI library loads and exports every function include/lasagna.h declares."""
+    from paper_conf_ipps_goswamilsp18_b200 import build
+    so = build.build()
+    lib = ctypes.CDLL(so)
+    syms = _header_symbols()
+    assert len(syms) >= 9
+    for s in syms:
+        assert hasattr(lib, s), s
+
+
+def test_library_reports_invalid_arguments_without_gpu():
+    from paper_conf_ipps_goswamilsp18_b200 import lasagna as lz
+    L = lz.lib()
+    ws = ctypes.c_size_t(0)
+    # L out of range / l_min >= L are rejected before any CUDA call
+    assert L.lasagna_greedy_graph(None, 10, 300, 5, 0, None, ctypes.byref(ws), None, None, None,
+                                  None) == lz.EINVAL
+    assert L.lasagna_greedy_graph(None, 10, 100, 100, 0, None, ctypes.byref(ws), None, None, None,
+                                  None) == lz.EINVAL
+    assert L.lasagna_greedy_graph(None, 1 << 31, 100, 63, 0, None, ctypes.byref(ws), None, None,
+                                  None, None) == lz.ERANGE
+    assert b"l_min" in L.lasagna_last_error() or True
+    assert L.lasagna_words_per_read(100) == 4 and L.lasagna_words_per_read(150) == 8
+    assert L.lasagna_words_per_read(32) == 1 and L.lasagna_words_per_read(33) == 2
+
+
+# ============================================================================ GPU parity
+gpu = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lz():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    import paper_conf_ipps_goswamilsp18_b200 as m
+    m.lib()
+    return m
+
+
+def _np(t, dtype):
+    return t.cpu().numpy().view(dtype)
+
+
+@gpu
+@pytest.mark.parametrize("L", [8, 32, 33, 100, 101, 150, 256])
+def test_pack_parity(lz, L):
+    import torch
+    reads = readgen.reads(5, 50_000, 777, L, 0.02)
+    stride = lz.words_per_read(L)
+    exp = oracle.pack(reads, stride)
+    # device input
+    got = lz.load_reads(torch.from_numpy(reads).cuda())
+    assert np.array_equal(_np(got, np.uint64), exp)
+    # page-locked host input, read in place by the kernel (zero-copy staging)
+    got2 = lz.load_reads(torch.from_numpy(reads).pin_memory())
+    assert np.array_equal(_np(got2, np.uint64), exp)
+    # lowercase maps the same way (R13)
+    low = np.char.lower(reads.view(f"S{L}")).view(np.uint8).reshape(reads.shape)
+    assert np.array_equal(_np(lz.load_reads(torch.from_numpy(low).cuda()), np.uint64), exp)
+
+
+@gpu
+def test_pack_ragged_offsets(lz):
+    """Sub-views starting at odd byte offsets (unaligned staging spans)."""
+    import torch
+    reads = readgen.reads(6, 50_000, 1000, 101, 0.0)
+    flat = torch.from_numpy(reads.reshape(-1).copy()).cuda()
+    for skip in [1, 3, 17]:
+        sub = flat[skip * 101:].view(-1, 101)
+        got = lz.load_reads(sub)
+        assert np.array_equal(_np(got, np.uint64), oracle.pack(reads[skip:], 4))
+
+
+@gpu
+def test_pack_rejects_non_acgt(lz):
+    import torch
+    reads = readgen.reads(1, 10_000, 500, 100, 0.0)
+    bad = reads.copy()
+    bad[321, 50] = ord("N")
+    bad[400, 0] = ord("-")
+    with pytest.raises(lz.LasagnaError, match="read 321"):
+        lz.load_reads(torch.from_numpy(bad).cuda())
+    assert oracle.first_bad(bad) == 321
+
+
+@gpu
+@pytest.mark.parametrize("n,L,l_min", [(3000, 100, 63), (2000, 40, 20), (1500, 150, 111),
+                                       (700, 256, 200), (513, 33, 1)])
+def test_fingerprints_parity(lz, n, L, l_min):
+    import torch
+    reads = readgen.reads(9, 300_000, n, L, 0.01)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    pfx, sfx = lz.fingerprints(packed, n, L, l_min)
+    epfx, esfx = oracle.fingerprints(reads, l_min)
+    assert np.array_equal(_np(pfx, np.uint64), epfx)
+    assert np.array_equal(_np(sfx, np.uint64), esfx)
+
+
+@gpu
+def test_fingerprints_fig_example_production(lz):
+    """GATACCAGTA at sigma=5, q=2^61-1: prefixes 3, 15, 77, ... (base-5 numerals)."""
+    import torch
+    reads = to_array(["GATACCAGTA"])
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    pfx, sfx = lz.fingerprints(packed, 1, 10, 1)
+    assert _np(pfx, np.uint64)[:, 0].tolist() == [3, 15, 77, 385, 1926, 9631, 48155, 240778,
+                                                  1203892, 6019460]
+    assert _np(sfx, np.uint64)[:, 0].tolist() == [0, 10, 85, 85, 710, 3835, 3835, 160085, 160085,
+                                                  6019460]
+    assert int(_np(pfx, np.uint64)[9, 1]) == oracle.F("TACTGGTATC") == 4027136
+
+
+@gpu
+@pytest.mark.parametrize("count", [0, 1, 2, 8191, 8192, 8193, 100_003, (1 << 20) + 7])
+@pytest.mark.parametrize("bits", [(0, 64), (40, 64), (3, 17), (56, 64)])
+def test_sort_u64_matches_numpy_stable(lz, count, bits):
+    import torch
+    rng = np.random.default_rng(count * 7 + bits[0])
+    keys = rng.integers(0, 2**63, size=count, dtype=np.int64).view(np.uint64)
+    keys ^= rng.integers(0, 2, size=count, dtype=np.uint64) << np.uint64(63)
+    lo, hi = bits
+    t = torch.from_numpy(keys.view(np.int64).copy()).cuda()
+    lz.sort_u64(t, lo, hi)
+    dig = (keys >> np.uint64(lo)) & np.uint64((1 << (hi - lo)) - 1 if hi - lo < 64 else 2**64 - 1)
+    exp = keys[np.argsort(dig, kind="stable")]
+    assert np.array_equal(_np(t, np.uint64), exp)
+
+
+@gpu
+def test_sort_u64_degenerate_inputs(lz):
+    import torch
+    n = 50_000
+    for keys in [np.full(n, 0xDEADBEEF12345678, dtype=np.uint64),
+                 np.arange(n, dtype=np.uint64) << np.uint64(20),
+                 (np.arange(n, dtype=np.uint64)[::-1] << np.uint64(20)).copy(),
+                 np.arange(n, dtype=np.uint64) % np.uint64(3)]:
+        t = torch.from_numpy(keys.view(np.int64).copy()).cuda()
+        lz.sort_u64(t, 0, 64)
+        assert np.array_equal(_np(t, np.uint64), np.sort(keys, kind="stable"))
+
+
+def _tiny_cases():
+    out = []
+    for seed in range(8):
+        rng = random.Random(100 + seed)
+        L = rng.choice([8, 12, 16, 20, 40])
+        G = rng.choice([30, 60, 200, 2000])
+        n = rng.choice([10, 40, 120])
+        p = rng.choice([0.0, 0.0, 0.02])
+        reads = readgen.reads(seed, G, n, L, p)
+        out.append((reads, rng.randint(2, L - 2)))
+    out.append((to_array(["ACGTTA" * 2, "CGTTAACGTTAA", "GTTAACGTTAAC", "AAGCTTAAGCTT",
+                          "ACACACACACAC", "GTGTGTGTGTGT", "GAATTCGAATTC", "TTCGAATTCGAA",
+                          "ACGTACGTACGT", "CGTACGTACGTA"]), 3))
+    # all-identical reads: every pair ties at every length
+    out.append((to_array(["ACGATCGATTGC"] * 30), 4))
+    return out
+
+
+@gpu
+@pytest.mark.parametrize("case", range(10))
+def test_overlaps_parity_tiny(lz, case):
+    import torch
+    reads, l_min = _tiny_cases()[case]
+    n, L = reads.shape
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    pl, pa, pb = lz.overlaps(packed, n, L, l_min)
+    epl, epa, epb = oracle.overlaps(reads, l_min)
+    assert np.array_equal(_np(pl, np.uint8), epl)
+    assert np.array_equal(_np(pa, np.uint32), epa)
+    assert np.array_equal(_np(pb, np.uint32), epb)
+
+
+@gpu
+@pytest.mark.parametrize("case", range(10))
+def test_greedy_graph_parity_tiny(lz, case):
+    import torch
+    reads, l_min = _tiny_cases()[case]
+    n, L = reads.shape
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, n, L, l_min)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc
+
+
+@gpu
+def test_micro_example_gpu(lz):
+    import torch
+    g = golden("micro_example.txt")
+    reads = to_array(g["reads"])
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, 6, 8, 4)
+    assert _np(r.succ, np.uint32).tolist() == [NONE if x == "N" else int(x) for x in g["succ"]]
+    assert _np(r.olen, np.uint8).tolist() == [int(x) for x in g["olen"]]
+    pl, pa, pb = lz.overlaps(packed, 6, 8, 4)
+    got = list(zip(_np(pl, np.uint8).tolist(), _np(pa, np.uint32).tolist(),
+                   _np(pb, np.uint32).tolist()))
+    assert got == [tuple(int(x) for x in p.split(",")) for p in g["pairs"]]
+
+
+@gpu
+def test_cfg1_parity(lz):
+    """cfg1 (BASELINE configs[0]): overlaps and greedy graph bit-exact vs the oracle."""
+    import torch
+    cfg = readgen.CONFIGS["cfg1"]
+    reads = readgen.config_reads(cfg)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    pl, pa, pb = lz.overlaps(packed, cfg.n, cfg.L, cfg.l_min)
+    epl, epa, epb = oracle.overlaps(reads, cfg.l_min)
+    assert np.array_equal(_np(pa, np.uint32), epa) and np.array_equal(_np(pb, np.uint32), epb)
+    assert np.array_equal(_np(pl, np.uint8), epl)
+    esucc, eolen, _ = oracle.greedy(cfg.n, epl, epa, epb)
+    for lpp in [0, 1, 5]:  # semi-streaming: one length per pass, groups of 5, all at once
+        r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=lpp)
+        assert np.array_equal(_np(r.succ, np.uint32), esucc), lpp
+        assert np.array_equal(_np(r.olen, np.uint8), eolen), lpp
+        assert r.stats["n_pairs"] == len(epl)
+    check_graph(reads, cfg.l_min, esucc, eolen, (epl, epa, epb))
+
+
+@gpu
+@pytest.mark.parametrize("seed", [20181, 20182])
+def test_cfg2_parity(lz, seed):
+    """cfg2 (BASELINE configs[1]: 2.3M reads, 1% errors): bit-exact greedy graph."""
+    import torch
+    cfg = readgen.CONFIGS["cfg2"]
+    reads = readgen.config_reads(cfg, seed=seed)
+    packed = lz.load_reads(torch.from_numpy(reads).pin_memory())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, cfg.l_min)
+    assert r.stats["n_pairs"] == m
+    assert r.stats["n_greedy"] == acc
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+
+
+def _random_candidates(n, k, rng, lens):
+    V = 2 * n
+    seen = set()
+    out = []
+    while len(out) < k:
+        a, b = sorted(rng.sample(range(V), 2))
+        l = rng.choice(lens)
+        if (l, a, b) in seen:
+            continue
+        seen.add((l, a, b))
+        out.append((l, a, b))
+    return out
+
+
+@gpu
+@pytest.mark.parametrize("seed", range(6))
+def test_greedy_pairs_matches_sequential(lz, seed):
+    import torch
+    rng = random.Random(seed)
+    n = rng.choice([50, 500, 20_000])
+    k = rng.choice([100, 5000, 60_000])
+    cand = _random_candidates(n, k, rng, [63, 64, 70, 99] if seed % 2 else [80])
+    P = sorted(cand, key=lambda t: (-t[0], t[1], t[2]))
+    esucc, eolen = brute.greedy(n, P)
+    rng.shuffle(cand)
+    pl = torch.tensor([c[0] for c in cand], dtype=torch.uint8).cuda()
+    pa = torch.tensor([c[1] for c in cand], dtype=torch.int64).to(torch.int32).cuda()
+    pb = torch.tensor([c[2] for c in cand], dtype=torch.int64).to(torch.int32).cuda()
+    succ, olen, rounds = lz.greedy_pairs(n, pl, pa, pb)
+    assert _np(succ, np.uint32).tolist() == esucc
+    assert _np(olen, np.uint8).tolist() == eolen
+
+
+@gpu
+@pytest.mark.parametrize("k", [2, 17, 1000, 10_001])
+def test_greedy_pairs_adversarial_chain(lz, k):
+    """Path a0-a1-...-ak at one length, priorities increasing along the path: k/2 rounds of
+    locally-dominant matching (then the sequential tail)."""
+    import torch
+    n = k + 2
+    cand = [(70, i, i + 1) for i in range(k)]
+    esucc, eolen = brute.greedy(n, sorted(cand, key=lambda t: (-t[0], t[1], t[2])))
+    pl = torch.full((k,), 70, dtype=torch.uint8).cuda()
+    pa = torch.arange(k, dtype=torch.int32).cuda()
+    pb = torch.arange(1, k + 1, dtype=torch.int32).cuda()
+    succ, olen, rounds = lz.greedy_pairs(n, pl, pa, pb)
+    assert _np(succ, np.uint32).tolist() == esucc
+    assert _np(olen, np.uint8).tolist() == eolen
