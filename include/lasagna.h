@@ -60,6 +60,9 @@ typedef enum {
 
 LASAGNA_API const char *lasagna_last_error(void);
 
+/* Process-wide count of CUDA kernels launched by this library (monotonic). */
+LASAGNA_API uint64_t lasagna_kernel_launches(void);
+
 /* u64 words per packed read (the row stride of `packed`): ceil(L/32) rounded up to 1, 2, 4
  * or 8 so that a read is one aligned 8/16/32/64-byte unit (L <= 128: one 32 B sector). */
 LASAGNA_API uint32_t lasagna_words_per_read(uint32_t L);
@@ -110,11 +113,15 @@ typedef struct {
     uint64_t n_pairs;          /* |P|: read-end pairs found (overlap edges / 2)             */
     uint64_t n_greedy;         /* pairs accepted by the greedy (directed edges / 2)         */
     uint64_t fp_false_matches; /* table hits whose key bits matched but bases did not (R12) */
+    uint64_t kernel_launches;  /* CUDA kernels this call launched                           */
     uint32_t rounds_max;       /* most greedy rounds any length needed                      */
     uint32_t passes;           /* device passes over the packed reads (length groups, a8)   */
     uint32_t lengths_per_pass; /* length-group size the planner chose                       */
     uint32_t key_dir_bits;     /* directory bits D of the sorted tables                     */
-    float ms_table, ms_sort, ms_search, ms_greedy; /* device time per phase (CUDA events)  */
+    uint32_t sort_launches;    /* onesweep passes launched (each sorts a whole group)       */
+    uint32_t search_launches;  /* search launches (one per length)                          */
+    /* device time per phase, CUDA events on `stream` (ms) */
+    float ms_table, ms_sort, ms_dir, ms_search, ms_greedy;
 } lasagna_stats;
 
 /* ---------------------------------------------------------------------------------------

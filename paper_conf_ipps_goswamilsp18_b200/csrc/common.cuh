@@ -160,6 +160,8 @@ __host__ __device__ inline uint32_t stride_for(uint32_t L)
 // ----------------------------------------------------------------- host-side error plumbing
 void set_error(const char *fmt, ...);
 lasagna_status cuda_status(cudaError_t e, const char *what);
+void count_launch();
+uint64_t launch_count();
 
 #define LSG_CUDA(call)                                                                         \
     do {                                                                                       \
@@ -169,6 +171,7 @@ lasagna_status cuda_status(cudaError_t e, const char *what);
 
 #define LSG_LAUNCHED(what)                                                                     \
     do {                                                                                       \
+        ::lsg::count_launch();                                                                 \
         cudaError_t e_ = cudaGetLastError();                                                   \
         if (e_ != cudaSuccess) return ::lsg::cuda_status(e_, what);                            \
     } while (0)

@@ -1,6 +1,8 @@
 // lasagna.cu — the C ABI (include/lasagna.h): argument validation, the workspace planner of
 // the semi-streaming driver (a8) and the per-length-group orchestration of a2..a7.
 #include <algorithm>
+#include <atomic>
+#include <vector>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -9,8 +11,12 @@
 
 namespace lsg {
 
-// ------------------------------------------------------------------ errors
+// ------------------------------------------------------------------ errors, launch counter
 static thread_local char g_err[512] = "";
+static std::atomic<unsigned long long> g_launches{0};
+
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+uint64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
 
 void set_error(const char *fmt, ...)
 {
@@ -170,26 +176,50 @@ struct Run {
     }
 };
 
+// Phase timing without extra synchronisation: event pairs are recorded on the stream as the
+// call proceeds and read once at the end of the call (which synchronises anyway for stats).
+enum Phase { PH_TABLE, PH_SORT, PH_DIR, PH_SEARCH, PH_GREEDY, PH_N };
 struct PhaseTimer {
-    bool on;
-    cudaStream_t s;
-    cudaEvent_t ev[2];
-    float *acc;
-    lasagna_status start(float *a)
+    bool on = false;
+    cudaStream_t s = nullptr;
+    struct Rec {
+        int ph;
+        cudaEvent_t a, b;
+    };
+    std::vector<Rec> recs;
+    int open = -1;
+    ~PhaseTimer()
+    {
+        for (auto &r : recs) cudaEventDestroy(r.a), cudaEventDestroy(r.b);
+    }
+    lasagna_status start(int ph)
     {
         if (!on) return LASAGNA_OK;
-        acc = a;
-        LSG_CUDA(cudaEventRecord(ev[0], s));
+        Rec r;
+        r.ph = ph;
+        LSG_CUDA(cudaEventCreate(&r.a));
+        LSG_CUDA(cudaEventCreate(&r.b));
+        recs.push_back(r);
+        LSG_CUDA(cudaEventRecord(r.a, s));
         return LASAGNA_OK;
     }
     lasagna_status stop()
     {
         if (!on) return LASAGNA_OK;
-        LSG_CUDA(cudaEventRecord(ev[1], s));
-        LSG_CUDA(cudaEventSynchronize(ev[1]));
-        float ms = 0;
-        LSG_CUDA(cudaEventElapsedTime(&ms, ev[0], ev[1]));
-        *acc += ms;
+        LSG_CUDA(cudaEventRecord(recs.back().b, s));
+        return LASAGNA_OK;
+    }
+    lasagna_status finish(lasagna_stats *st)
+    {
+        if (!on) return LASAGNA_OK;
+        LSG_CUDA(cudaStreamSynchronize(s));
+        float *acc[PH_N] = {&st->ms_table, &st->ms_sort, &st->ms_dir, &st->ms_search,
+                            &st->ms_greedy};
+        for (auto &r : recs) {
+            float ms = 0;
+            LSG_CUDA(cudaEventElapsedTime(&ms, r.a, r.b));
+            *acc[r.ph] += ms;
+        }
         return LASAGNA_OK;
     }
 };
@@ -217,13 +247,16 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     ta.sfxk = r.sfxk;
     ta.hist = r.hist;
     lasagna_status rc;
-    if ((rc = tm.start(st ? &st->ms_table : nullptr)) != LASAGNA_OK) return rc;
+    if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
     if ((rc = launch_table(ta, r.s)) != LASAGNA_OK) return rc;
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
-    if ((rc = tm.start(st ? &st->ms_sort : nullptr)) != LASAGNA_OK) return rc;
+    if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
     if ((rc = sort_segments(r.tab, g.V, G, 64 - g.D, 64, r.hist, true, r.sctx, r.s, which)) !=
         LASAGNA_OK)
         return rc;
+    if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+    if (st) st->sort_launches += P;
+    if ((rc = tm.start(PH_DIR)) != LASAGNA_OK) return rc;
     if ((rc = launch_dir(r.tab[*which], g.V, G, g.D, r.dir, r.s)) != LASAGNA_OK) return rc;
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     return LASAGNA_OK;
@@ -277,6 +310,8 @@ using namespace lsg;
 extern "C" {
 
 const char *lasagna_last_error(void) { return g_err; }
+
+uint64_t lasagna_kernel_launches(void) { return launch_count(); }
 
 uint32_t lasagna_words_per_read(uint32_t L) { return stride_for(L); }
 
@@ -434,17 +469,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     PhaseTimer tm;
     tm.on = stats != nullptr;
     tm.s = s;
-    if (tm.on) {
-        LSG_CUDA(cudaEventCreate(&tm.ev[0]));
-        LSG_CUDA(cudaEventCreate(&tm.ev[1]));
-    }
-    struct EvGuard {
-        PhaseTimer &t;
-        ~EvGuard()
-        {
-            if (t.on) cudaEventDestroy(t.ev[0]), cudaEventDestroy(t.ev[1]);
-        }
-    } evg{tm};
+    const uint64_t launches0 = launch_count();
 
     if ((rc = sort_ctx_reset(r.sctx, s)) != LASAGNA_OK) return rc;
     LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, 8 * sizeof(unsigned long long), s));
@@ -461,7 +486,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
         ++st.passes;
         for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
             uint64_t m = 0;
-            if ((rc = tm.start(&st.ms_search)) != LASAGNA_OK) return rc;
+            if ((rc = tm.start(PH_SEARCH)) != LASAGNA_OK) return rc;
             // no pruning: the claimed bits are not consulted, so every length's full pair
             // list is found (|P| = overlap edges / 2 is reported)
             if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr, &m)) != LASAGNA_OK)
@@ -476,7 +501,8 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
             }
             total_pairs += m;
             uint32_t rounds = 0;
-            if ((rc = tm.start(&st.ms_greedy)) != LASAGNA_OK) return rc;
+            ++st.search_launches;
+            if ((rc = tm.start(PH_GREEDY)) != LASAGNA_OK) return rc;
             if ((rc = greedy_length(gb, m, (uint8_t)l, succ, olen, s, &rounds)) != LASAGNA_OK)
                 return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
@@ -490,6 +516,8 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
         st.n_pairs = total_pairs;
         st.fp_false_matches = h[1];
         st.n_greedy = h[2];
+        if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
+        st.kernel_launches = launch_count() - launches0;
         *stats = st;
     }
     return LASAGNA_OK;

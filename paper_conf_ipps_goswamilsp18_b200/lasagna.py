@@ -27,10 +27,12 @@ class LasagnaError(RuntimeError):
 
 class _Stats(ctypes.Structure):
     _fields_ = [("n_pairs", ctypes.c_uint64), ("n_greedy", ctypes.c_uint64),
-                ("fp_false_matches", ctypes.c_uint64), ("rounds_max", ctypes.c_uint32),
-                ("passes", ctypes.c_uint32), ("lengths_per_pass", ctypes.c_uint32),
-                ("key_dir_bits", ctypes.c_uint32), ("ms_table", ctypes.c_float),
-                ("ms_sort", ctypes.c_float), ("ms_search", ctypes.c_float),
+                ("fp_false_matches", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
+                ("rounds_max", ctypes.c_uint32), ("passes", ctypes.c_uint32),
+                ("lengths_per_pass", ctypes.c_uint32), ("key_dir_bits", ctypes.c_uint32),
+                ("sort_launches", ctypes.c_uint32), ("search_launches", ctypes.c_uint32),
+                ("ms_table", ctypes.c_float), ("ms_sort", ctypes.c_float),
+                ("ms_dir", ctypes.c_float), ("ms_search", ctypes.c_float),
                 ("ms_greedy", ctypes.c_float)]
 
     def as_dict(self) -> dict:
@@ -60,6 +62,7 @@ def lib() -> ctypes.CDLL:
     pu64 = ctypes.POINTER(ctypes.c_uint64)
     pu32 = ctypes.POINTER(ctypes.c_uint32)
     L.lasagna_last_error.restype = ctypes.c_char_p
+    L.lasagna_kernel_launches.restype = u64
     L.lasagna_words_per_read.argtypes = [u32]
     L.lasagna_words_per_read.restype = u32
     sigs = {
@@ -91,6 +94,11 @@ def _stream(device=None) -> int:
 
 def _ptr(t: torch.Tensor | None):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def kernel_launches() -> int:
+    """Process-wide number of kernels liblasagna.so has launched."""
+    return int(lib().lasagna_kernel_launches())
 
 
 def words_per_read(L: int) -> int:

@@ -269,6 +269,7 @@ def test_cfg2_parity(lz, seed):
 
 def _random_candidates(n, k, rng, lens):
     V = 2 * n
+    k = min(k, len(lens) * V * (V - 1) // 4)  # at most half of all distinct (l, a, b)
     seen = set()
     out = []
     while len(out) < k:
