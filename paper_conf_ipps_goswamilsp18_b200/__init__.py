@@ -6,8 +6,9 @@ There is no CPU fallback.
 """
 from .lasagna import (  # noqa: F401
     NONE, GraphResult, GreedyGraph, LasagnaError, fingerprints, greedy_graph, greedy_pairs,
+    kernel_launches,
     lib, load_reads, overlaps, plan, sort_u64, words_per_read,
 )
 
 __all__ = ["NONE", "GraphResult", "GreedyGraph", "LasagnaError", "fingerprints", "greedy_graph",
-           "greedy_pairs", "lib", "load_reads", "overlaps", "plan", "sort_u64", "words_per_read"]
+           "greedy_pairs", "kernel_launches", "lib", "load_reads", "overlaps", "plan", "sort_u64", "words_per_read"]
