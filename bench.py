@@ -131,21 +131,20 @@ def cpu_baseline(reads: np.ndarray, l_min: int, target_s: float = 12.0) -> dict:
 
 # ------------------------------------------------------------------ algorithmic bytes
 def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict) -> dict:
-    """Dominant phase and its achieved algorithmic GB/s (CUDA-event times per launch)."""
+    """Dominant phase and its achieved ALGORITHMIC GB/s (bytes per unit in DESIGN.md x units
+    per launch / CUDA-event time per launch)."""
     V = 2 * n
+    N = 2 * V                     # table entries per length (prefix + suffix list)
     n_len = L - l_min
-    D = stats["key_dir_bits"]
-    bucket = V / float(1 << D)
     G = stats["lengths_per_pass"]
+    verify = 64.0 * (stats["n_pairs"] + stats["fp_false_matches"]) / max(1, n_len)
     per = {
-        # one onesweep pass: every key of the group read once and written once
-        "onesweep_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * V),
-        # one search launch (one length): query key + 2 directory words + bucket scan (+ verify)
-        "search_kernel": (stats["ms_search"], stats["search_launches"],
-                          V * (8.0 + 8.0 + 8.0 * bucket) + 64.0 * stats["n_pairs"] / max(1, n_len)),
-        # table: tab key + query key written per entry, packed read loaded per read
-        "table_kernel": (stats["ms_table"], stats["passes"], 16.0 * G * V + 32.0 * n),
-        "dir_kernel": (stats["ms_dir"], stats["passes"], 8.0 * G * V + 4.0 * G * (1 << D)),
+        # one onesweep pass over a group: every key read once and written once
+        "onesweep_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
+        # one join launch (one length): the sorted table streamed once + verification loads
+        "join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
+        # table: 4 keys (32 B) written per read per length, the packed read loaded once
+        "table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
     }
     name = max(per, key=lambda k: per[k][0])
     ms, launches, bytes_per_launch = per[name]
@@ -265,7 +264,7 @@ def main() -> None:
 
     # ---- device-resident timed region
     sampler = ClockSampler(_bus_id(torch, 0))
-    agg = {k: 0.0 for k in ["ms_table", "ms_sort", "ms_dir", "ms_search", "ms_greedy"]}
+    agg = {k: 0.0 for k in ["ms_table", "ms_sort", "ms_search", "ms_greedy"]}
     cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes"]}
     sampler.start()
     torch.cuda.synchronize()
@@ -312,7 +311,7 @@ def main() -> None:
                    "G": cfg.G, "p_err": cfg.p_err, "seed": cfg.seed,
                    "lengths_per_pass": st["lengths_per_pass"], "passes": st["passes"] // args.steps,
                    "l2": "inputs larger than L2 (ASCII %.1f GB, key tables %.1f GB)"
-                         % (n * L / 1e9, 24.0 * 2 * n * st["lengths_per_pass"] / 1e9)},
+                         % (n * L / 1e9, 32.0 * 2 * n * st["lengths_per_pass"] / 1e9)},
         "overlap_edges_per_s": edges / (ms_step / 1e3),
         "read_end_pairs": st["n_pairs"], "greedy_pairs": st["n_greedy"],
         "fp_false_matches": st["fp_false_matches"], "greedy_rounds_max": st["rounds_max"],

@@ -117,11 +117,11 @@ typedef struct {
     uint32_t rounds_max;       /* most greedy rounds any length needed                      */
     uint32_t passes;           /* device passes over the packed reads (length groups, a8)   */
     uint32_t lengths_per_pass; /* length-group size the planner chose                       */
-    uint32_t key_dir_bits;     /* directory bits D of the sorted tables                     */
+    uint32_t key_sort_bits;    /* key bits T the tables are radix-sorted by (bucket bits)   */
     uint32_t sort_launches;    /* onesweep passes launched (each sorts a whole group)       */
-    uint32_t search_launches;  /* search launches (one per length)                          */
+    uint32_t search_launches;  /* search (join) launches, one per length                    */
     /* device time per phase, CUDA events on `stream` (ms) */
-    float ms_table, ms_sort, ms_dir, ms_search, ms_greedy;
+    float ms_table, ms_sort, ms_search, ms_greedy;
 } lasagna_stats;
 
 /* ---------------------------------------------------------------------------------------

@@ -93,12 +93,13 @@ lasagna_status launch_fp_values(const uint64_t *packed, uint64_t n, uint32_t L, 
 }
 
 // ---------------------------------------------------------------- key tables (a2 + a3)
-// For each length l in the group [l_lo, l_hi] (segment s = l - l_lo), every vertex v:
-//   tab[s*V + v]  = (mix(pfx_l(v)) & ~vmask) | v      prefix table entry: key bits | vid
-//   sfxk[s*V + v] =  mix(sfx_l(v)) & ~vmask           query key of v's suffix
-// plus the histogram of the first LSD digit of the tab keys per segment (onesweep's
-// upfront histogram), accumulated in shared memory and flushed once per CTA.
-
+// For each length l in the group [l_lo, l_hi] (segment s = l - l_lo) and every vertex v the
+// combined table of the paper's two lists P_l and S_l:
+//   tab[s*2V + 2v]     = (mix(pfx_l(v)) & keep) | 0 << vbits | v    prefix entry
+//   tab[s*2V + 2v + 1] = (mix(sfx_l(v)) & keep) | 1 << vbits | v    suffix entry
+// (keep = the bits above tag + vid), i.e. 32 contiguous bytes per read per length, plus the
+// histogram of the first LSD digit per segment (onesweep's upfront histogram), accumulated
+// in shared memory and flushed once per CTA.
 template <int W>
 __global__ void __launch_bounds__(256)
 table_kernel(TableArgs a)
@@ -107,8 +108,9 @@ table_kernel(TableArgs a)
     const uint32_t G = a.l_hi - a.l_lo + 1;
     for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x) shist[t] = 0;
     __syncthreads();
-    const uint64_t V = 2 * a.n;
-    const uint64_t keep = ~((1ull << a.vbits) - 1);
+    const uint64_t N = 4 * a.n; // 2V entries per length
+    const uint64_t keep = ~((2ull << a.vbits) - 1);
+    const uint64_t tagS = 1ull << a.vbits;
     const uint32_t dmask = (1u << a.d_bits) - 1;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
          i += (uint64_t)gridDim.x * blockDim.x) {
@@ -118,14 +120,17 @@ table_kernel(TableArgs a)
         roll_read<W>(x, y, a.l_hi, [&](uint32_t l, const FpStreams &st) {
             if (l < a.l_lo) return;
             const uint32_t s = l - a.l_lo;
-            const uint64_t off = (uint64_t)s * V + 2 * i;
-            const uint64_t k0 = (mix(st.P0) & keep) | (2 * i);
-            const uint64_t k1 = (mix(st.P1) & keep) | (2 * i + 1);
-            *reinterpret_cast<ulonglong2 *>(a.tab + off) = make_ulonglong2(k0, k1);
-            *reinterpret_cast<ulonglong2 *>(a.sfxk + off) =
-                make_ulonglong2(mix(st.S0) & keep, mix(st.S1) & keep);
-            atomicAdd(&shist[s * 256 + (uint32_t)((k0 >> a.d_shift) & dmask)], 1u);
-            atomicAdd(&shist[s * 256 + (uint32_t)((k1 >> a.d_shift) & dmask)], 1u);
+            const uint64_t v0 = 2 * i, v1 = 2 * i + 1;
+            const uint64_t p0 = (mix(st.P0) & keep) | v0, s0 = (mix(st.S0) & keep) | tagS | v0;
+            const uint64_t p1 = (mix(st.P1) & keep) | v1, s1 = (mix(st.S1) & keep) | tagS | v1;
+            ulonglong2 *dst = reinterpret_cast<ulonglong2 *>(a.tab + (uint64_t)s * N + 4 * i);
+            dst[0] = make_ulonglong2(p0, s0);
+            dst[1] = make_ulonglong2(p1, s1);
+            uint32_t *h = shist + s * 256;
+            atomicAdd(&h[(uint32_t)((p0 >> a.d_shift) & dmask)], 1u);
+            atomicAdd(&h[(uint32_t)((s0 >> a.d_shift) & dmask)], 1u);
+            atomicAdd(&h[(uint32_t)((p1 >> a.d_shift) & dmask)], 1u);
+            atomicAdd(&h[(uint32_t)((s1 >> a.d_shift) & dmask)], 1u);
         });
     }
     __syncthreads();

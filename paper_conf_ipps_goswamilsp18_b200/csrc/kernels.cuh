@@ -21,7 +21,7 @@ struct TableArgs {
     uint32_t l_lo, l_hi;      // group of lengths (segment s = l - l_lo)
     uint32_t vbits;           // b_v: vertex-id bits at the bottom of a key
     uint32_t d_shift, d_bits; // first LSD digit (histogram produced on the fly)
-    uint64_t *tab, *sfxk;     // [G][V]
+    uint64_t *tab;            // [G][2V]: entry 2v = prefix key of v, 2v+1 = suffix key of v
     uint32_t *hist;           // [G][256]
 };
 lasagna_status launch_table(const TableArgs &a, cudaStream_t s);
@@ -42,22 +42,17 @@ lasagna_status sort_segments(uint64_t *bufs[2], uint64_t seg_len, uint32_t n_seg
                              cudaStream_t s, int *which);
 
 // ---- a5 (search.cu)
-lasagna_status launch_dir(const uint64_t *tab, uint64_t V, uint32_t n_seg, uint32_t D,
-                          uint32_t *dir, cudaStream_t s);
-struct SearchArgs {
+struct JoinArgs {
     const uint64_t *packed;
-    const uint64_t *tab;   // sorted table of this length (V entries)
-    const uint64_t *sfxk;  // query keys of this length (V entries)
-    const uint32_t *dir;   // 2^D + 1 entries
-    uint64_t V;
-    uint32_t L, stride, l, vbits, D;
-    const uint8_t *claimed;    // optional: skip claimed read ends (pruning), may be null
+    const uint64_t *keys;      // sorted combined table of this length (N = 2V entries)
+    uint64_t N;
+    uint32_t L, stride, l, vbits, T; // T: sorted (bucket) bits
     unsigned long long *pairs; // out pool: (a << 32) | b
     unsigned long long cap;
     unsigned long long *count; // pool fill (may exceed cap: overflow)
     unsigned long long *false_matches;
 };
-lasagna_status launch_search(const SearchArgs &a, cudaStream_t s);
+lasagna_status launch_join(const JoinArgs &a, cudaStream_t s);
 lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsigned long long *count,
                                     uint64_t m, unsigned long long cap, uint32_t vbits,
                                     uint64_t *keys, cudaStream_t s);

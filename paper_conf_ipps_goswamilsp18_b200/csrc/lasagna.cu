@@ -2,6 +2,7 @@
 // the semi-streaming driver (a8) and the per-length-group orchestration of a2..a7.
 #include <algorithm>
 #include <atomic>
+#include <cmath>
 #include <vector>
 #include <cstdarg>
 #include <cstdio>
@@ -34,11 +35,13 @@ lasagna_status cuda_status(cudaError_t e, const char *what)
 
 // ------------------------------------------------------------------ planning
 // Geometry of the key tables:
-//   key = (mix(F) top (64 - vbits) bits) << vbits | vertex id,  vbits = ceil(log2 V)
-//   sorted by the top D = vbits - 3 key bits (directory buckets of 4-8 entries on average)
+//   N = 2V entries per length (prefix + suffix list), V = 2n vertices
+//   key = mix(F) top (63 - vbits) bits | tag << vbits | vertex id,  vbits = ceil(log2 V)
+//   radix-sorted by the top T = 8P key bits, P = ceil((log2 N - 11.5) / 8) passes, so a
+//   T-bit bucket holds ~N / 2^T <= ~2.9K entries (one shared-memory join tile)
 struct Geometry {
-    uint64_t n, V;
-    uint32_t L, l_min, n_len, vbits, D;
+    uint64_t n, V, N;
+    uint32_t L, l_min, n_len, vbits, T;
 };
 
 static uint32_t ceil_log2(uint64_t x)
@@ -53,12 +56,15 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     Geometry g;
     g.n = n;
     g.V = 2 * n;
+    g.N = 2 * g.V;
     g.L = L;
     g.l_min = l_min;
     g.n_len = L - l_min; // lengths l_min .. L-1 (R5: the l = L partition is dropped)
     g.vbits = std::max<uint32_t>(1, ceil_log2(g.V));
-    int D = (int)g.vbits - 3;
-    g.D = (uint32_t)std::min(28, std::max(1, D));
+    const double lg = g.N > 1 ? std::log2((double)g.N) : 0.0;
+    int P = (int)std::ceil((lg - 11.5) / 8.0);
+    P = std::max(1, std::min(P, 4));
+    g.T = std::min<uint32_t>(8u * (uint32_t)P, 63u - g.vbits);
     return g;
 }
 
@@ -67,8 +73,8 @@ static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Layout {
     uint32_t G;          // lengths per group
     uint64_t pool_cap;   // pair pool capacity (pairs)
-    size_t tabA, tabB, sfxk, dir, status, hist, ctrs, pool, pool2, best0, best1, claimed, keys,
-        keys2, total;
+    size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best0, best1, claimed,
+        total;
 };
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
@@ -84,13 +90,11 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
         off += align256(bytes);
         return o;
     };
-    const size_t tabb = (size_t)G * g.V * 8;
+    const size_t tabb = (size_t)G * g.N * 8;
     l.tabA = take(tabb);
     l.tabB = take(tabb);
-    l.sfxk = take(tabb);
-    l.dir = take((size_t)G * ((1ull << g.D) + 1) * 4);
-    size_t st = std::max(sort_status_bytes(g.V, G), sort_status_bytes(pool_cap, 1));
-    l.status = take(st);
+    l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
+    l.status = take(l.status_bytes);
     l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
     l.ctrs = take(CTR_BYTES);
     l.pool = take(pool_cap * 8);
@@ -99,11 +103,8 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
         l.best0 = take(g.V * 4);
         l.best1 = take(g.V * 4);
         l.claimed = take(g.V);
-        l.keys = l.keys2 = 0;
     } else {
-        l.best0 = l.best1 = l.claimed = 0;
-        l.keys = l.pool;  // overlaps: compact keys sorted in place of the pool...
-        l.keys2 = l.pool2; // ...with pool2 as the sort scratch
+        l.best0 = l.best1 = l.claimed = 0; // overlaps: pairs sorted in pool/pool2
     }
     l.total = off;
     return l;
@@ -152,8 +153,7 @@ struct Run {
     cudaStream_t s;
     SortCtx sctx;
     uint64_t *tab[2];
-    uint64_t *sfxk;
-    uint32_t *dir, *hist;
+    uint32_t *hist;
     unsigned long long *ctr64; // [0] pool count, [1] false matches, [2] accepted, [3] cnt2
     unsigned long long *pool, *pool2;
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
@@ -162,12 +162,9 @@ struct Run {
         ws = (char *)workspace;
         tab[0] = at<uint64_t>(lay.tabA);
         tab[1] = at<uint64_t>(lay.tabB);
-        sfxk = at<uint64_t>(lay.sfxk);
-        dir = at<uint32_t>(lay.dir);
         hist = at<uint32_t>(lay.hist);
         sctx.status = at<unsigned long long>(lay.status);
-        sctx.status_bytes =
-            std::max(sort_status_bytes(g.V, lay.G), sort_status_bytes(lay.pool_cap, 1));
+        sctx.status_bytes = lay.status_bytes;
         sctx.tile_ctrs = at<uint32_t>(lay.ctrs);
         sctx.epoch = 0;
         ctr64 = reinterpret_cast<unsigned long long *>(ws + lay.ctrs + 4096 * 4);
@@ -178,7 +175,7 @@ struct Run {
 
 // Phase timing without extra synchronisation: event pairs are recorded on the stream as the
 // call proceeds and read once at the end of the call (which synchronises anyway for stats).
-enum Phase { PH_TABLE, PH_SORT, PH_DIR, PH_SEARCH, PH_GREEDY, PH_N };
+enum Phase { PH_TABLE, PH_SORT, PH_SEARCH, PH_GREEDY, PH_N };
 struct PhaseTimer {
     bool on = false;
     cudaStream_t s = nullptr;
@@ -213,8 +210,7 @@ struct PhaseTimer {
     {
         if (!on) return LASAGNA_OK;
         LSG_CUDA(cudaStreamSynchronize(s));
-        float *acc[PH_N] = {&st->ms_table, &st->ms_sort, &st->ms_dir, &st->ms_search,
-                            &st->ms_greedy};
+        float *acc[PH_N] = {&st->ms_table, &st->ms_sort, &st->ms_search, &st->ms_greedy};
         for (auto &r : recs) {
             float ms = 0;
             LSG_CUDA(cudaEventElapsedTime(&ms, r.a, r.b));
@@ -231,7 +227,7 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     const Geometry &g = r.g;
     const uint32_t G = l_hi - l_lo + 1;
     uint32_t P, shifts[8], bits[8];
-    digit_plan(64 - g.D, 64, &P, shifts, bits);
+    digit_plan(64 - g.T, 64, &P, shifts, bits);
     LSG_CUDA(cudaMemsetAsync(r.hist, 0, (size_t)G * 256 * 4, r.s));
     TableArgs ta;
     ta.packed = packed;
@@ -244,47 +240,41 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     ta.d_shift = shifts[0];
     ta.d_bits = bits[0];
     ta.tab = r.tab[0];
-    ta.sfxk = r.sfxk;
     ta.hist = r.hist;
     lasagna_status rc;
     if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
     if ((rc = launch_table(ta, r.s)) != LASAGNA_OK) return rc;
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
-    if ((rc = sort_segments(r.tab, g.V, G, 64 - g.D, 64, r.hist, true, r.sctx, r.s, which)) !=
+    if ((rc = sort_segments(r.tab, g.N, G, 64 - g.T, 64, r.hist, true, r.sctx, r.s, which)) !=
         LASAGNA_OK)
         return rc;
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     if (st) st->sort_launches += P;
-    if ((rc = tm.start(PH_DIR)) != LASAGNA_OK) return rc;
-    if ((rc = launch_dir(r.tab[*which], g.V, G, g.D, r.dir, r.s)) != LASAGNA_OK) return rc;
-    if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     return LASAGNA_OK;
 }
 
+// Join (search + verify) of length l; *m_out = pairs found (host, synchronises).
 static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, uint32_t l_lo,
-                                    int which, const uint8_t *claimed, uint64_t *m_out)
+                                    int which, uint64_t *m_out)
 {
     const Geometry &g = r.g;
     const uint32_t s = l - l_lo;
     LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, sizeof(unsigned long long), r.s));
-    SearchArgs sa;
-    sa.packed = packed;
-    sa.tab = r.tab[which] + (uint64_t)s * g.V;
-    sa.sfxk = r.sfxk + (uint64_t)s * g.V;
-    sa.dir = r.dir + (uint64_t)s * ((1ull << g.D) + 1);
-    sa.V = g.V;
-    sa.L = g.L;
-    sa.stride = stride_for(g.L);
-    sa.l = l;
-    sa.vbits = g.vbits;
-    sa.D = g.D;
-    sa.claimed = claimed;
-    sa.pairs = r.pool;
-    sa.cap = r.lay.pool_cap;
-    sa.count = r.ctr64;
-    sa.false_matches = r.ctr64 + 1;
-    lasagna_status rc = launch_search(sa, r.s);
+    JoinArgs ja;
+    ja.packed = packed;
+    ja.keys = r.tab[which] + (uint64_t)s * g.N;
+    ja.N = g.N;
+    ja.L = g.L;
+    ja.stride = stride_for(g.L);
+    ja.l = l;
+    ja.vbits = g.vbits;
+    ja.T = g.T;
+    ja.pairs = r.pool;
+    ja.cap = r.lay.pool_cap;
+    ja.count = r.ctr64;
+    ja.false_matches = r.ctr64 + 1;
+    lasagna_status rc = launch_join(ja, r.s);
     if (rc != LASAGNA_OK) return rc;
     unsigned long long m = 0;
     LSG_CUDA(cudaMemcpyAsync(&m, r.ctr64, sizeof(m), cudaMemcpyDeviceToHost, r.s));
@@ -465,7 +455,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     lasagna_stats st;
     memset(&st, 0, sizeof st);
     st.lengths_per_pass = G;
-    st.key_dir_bits = g.D;
+    st.key_sort_bits = g.T;
     PhaseTimer tm;
     tm.on = stats != nullptr;
     tm.s = s;
@@ -489,7 +479,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
             if ((rc = tm.start(PH_SEARCH)) != LASAGNA_OK) return rc;
             // no pruning: the claimed bits are not consulted, so every length's full pair
             // list is found (|P| = overlap edges / 2 is reported)
-            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr, &m)) != LASAGNA_OK)
+            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, &m)) != LASAGNA_OK)
                 return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
             if (m > cap) {
@@ -579,7 +569,7 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
             return rc;
         for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
             uint64_t m = 0;
-            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr, &m)) != LASAGNA_OK)
+            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, &m)) != LASAGNA_OK)
                 return rc;
             worst = std::max(worst, m);
             if (m > cap) { // count only from here on

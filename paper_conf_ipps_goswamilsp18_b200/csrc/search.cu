@@ -1,129 +1,178 @@
-// search.cu — a5: batched sorted-table lookup of suffix fingerprints + exact verification
-// (Algorithm 2: lower bound L, upper bound U, count C = U - L of each suffix
-// key in the sorted prefix list; an edge per match; R12 exact check).
+// search.cu — a5: batched sorted-table lookup of suffix fingerprints against prefix
+// fingerprints + exact verification (Algorithm 2; R12).
 //
-// The table of one length is sorted by its top D key bits (a4), so the run of entries of
-// directory bucket d = key >> (64-D) is [dir[d], dir[d+1]).  For a query q = sfx key of u:
-//   L_u = dir[q >> (64-D)], U_u = dir[(q >> (64-D)) + 1]   (bucket bounds, ~4-8 entries)
-// and within the bucket the entries whose stored key bits equal q's are the fingerprint
-// matches (the lower/upper-bound interval of P:L164 restricted to equal keys).  Each match
-// v from a different read with u < v^1 is verified on the 2-bit bases and emitted as the
-// read-end pair (a = u, b = v^1): every pair exactly once (its twin has a > b).
+// Per length l the table holds BOTH lists of the paper — the prefix list P_l (tag 0) and
+// the suffix list S_l (tag 1) — as one array of 2V keys
+//     key = mix(F) top bits | tag << vbits | vertex id,
+// radix-sorted by the top T key bits (a4).  After the sort, equal fingerprints sit in the
+// same T-bit bucket, so Algorithm 2's windows W_S / W_P "such that a fingerprint present in
+// W_S cannot be present in any window except W_P" are exactly runs of whole
+// buckets.  Each CTA owns the buckets that START inside its chunk of the sorted array,
+// stages their entries in shared memory, builds a small hash table over the prefix entries
+// and looks every suffix entry up in it (the vectorised lower/upper bound of P:L164-166,
+// done as a shared-memory probe: all matches of a key are found, C = U - L of them).
+// Each fingerprint match v of a suffix u from a different read with u < v^1 is verified
+// on the 2-bit bases and emitted as the read-end pair (a = u, b = v^1), so every pair is
+// emitted exactly once (its twin has a > b).
+//
+// Traffic: the sorted array is streamed once (8 B per entry, 16 B per vertex); random
+// accesses are limited to the verification loads of fingerprint matches.
 #include "kernels.cuh"
 
 namespace lsg {
 
-// dir[d] = first index whose key has top-D bits >= d, d = 0..2^D (dir[2^D] = V)
-__global__ void dir_kernel(const uint64_t *__restrict__ tab, uint64_t V, uint32_t D,
-                           uint32_t *__restrict__ dir)
-{
-    const uint32_t s = blockIdx.y;
-    const uint64_t nd = 1ull << D;
-    const uint64_t *t = tab + (uint64_t)s * V;
-    uint32_t *dr = dir + (uint64_t)s * (nd + 1);
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const int64_t k = (int64_t)(t[i] >> (64 - D));
-        const int64_t kp = i ? (int64_t)(t[i - 1] >> (64 - D)) : -1;
-        for (int64_t d = kp + 1; d <= k; ++d) dr[d] = (uint32_t)i;
-        if (i == V - 1)
-            for (uint64_t d = (uint64_t)k + 1; d <= nd; ++d) dr[d] = (uint32_t)V;
+constexpr int JOIN_THREADS = 512;
+constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
+constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
+constexpr int JOIN_SLOTS = 8192;   // u16 hash slots (load <= 0.75 even when all staged are P)
+constexpr int JOIN_BUF = 1024;     // staged output pairs
+constexpr unsigned short SLOT_EMPTY = 0xFFFF;
+
+struct Emitter {
+    unsigned long long *buf;  // shared
+    uint32_t *bcount;         // shared
+    unsigned long long *pairs, cap, *count;
+    __device__ __forceinline__ void emit(unsigned long long rec)
+    {
+        uint32_t slot = atomicAdd(bcount, 1u);
+        if (slot < JOIN_BUF) buf[slot] = rec;
+        else {
+            unsigned long long gs = atomicAdd(count, 1ull);
+            if (gs < cap) pairs[gs] = rec;
+        }
     }
-    if (V == 0 && blockIdx.x == 0)
-        for (uint64_t d = threadIdx.x; d <= nd; d += blockDim.x) dr[d] = 0;
-}
-
-constexpr int SEARCH_THREADS = 256;
-constexpr int SEARCH_BUF = 4096; // staged pairs per CTA
-
+};
 
 template <int W>
-__global__ void __launch_bounds__(SEARCH_THREADS)
-search_kernel(SearchArgs a)
+__device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t s_ent, uint64_t p_ent,
+                                          uint64_t vmask, Emitter &em, unsigned long long &nfalse)
 {
-    __shared__ unsigned long long buf[SEARCH_BUF];
+    const uint32_t u = (uint32_t)(s_ent & vmask), v = (uint32_t)(p_ent & vmask);
+    const uint32_t b = v ^ 1u;
+    if ((u >> 1) == (v >> 1) || u >= b) return; // R9: no same-read edge; each pair once
+    if (!verify_overlap<W>(a.packed, a.stride, a.L, u, v, a.l)) {
+        ++nfalse;
+        return;
+    }
+    em.emit(((unsigned long long)u << 32) | b);
+}
+
+template <int W>
+__global__ void __launch_bounds__(JOIN_THREADS)
+join_kernel(JoinArgs a)
+{
+    extern __shared__ __align__(16) unsigned char jsm[];
+    uint64_t *ent = reinterpret_cast<uint64_t *>(jsm);                                   // [CAP]
+    unsigned long long *buf = reinterpret_cast<unsigned long long *>(jsm + JOIN_CAP * 8); // [BUF]
+    unsigned short *slot = reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);
     __shared__ uint32_t bcount;
     __shared__ unsigned long long gbase;
-    if (threadIdx.x == 0) bcount = 0;
-    __syncthreads();
+    __shared__ unsigned long long s_lo, s_hi;
+
+    const uint64_t N = a.N;
+    const uint64_t base = (uint64_t)blockIdx.x * JOIN_CHUNK;
+    if (base >= N) return;
+    const uint32_t bshift = 64 - a.T;
+    const uint32_t kshift = a.vbits + 1; // key bits above tag + vid
     const uint64_t vmask = (1ull << a.vbits) - 1;
-    const uint32_t dshift = 64 - a.D;
+    const uint64_t *A = a.keys;
+
+    if (threadIdx.x == 0) {
+        bcount = 0;
+        s_lo = ~0ull;
+        s_hi = ~0ull;
+    }
+    for (int t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = SLOT_EMPTY;
+    __syncthreads();
+
+    // bucket starts: i is a start if i == 0 or bucket(A[i]) != bucket(A[i-1]).
+    // lo = first start in [base, base+CHUNK); hi = first start >= base+CHUNK (or N).
+    const uint64_t cend = min64(N, base + JOIN_CHUNK);
+    for (uint64_t i = base + threadIdx.x; i < cend; i += JOIN_THREADS) {
+        bool st = (i == 0) || ((A[i] >> bshift) != (A[i - 1] >> bshift));
+        if (st) atomicMin(&s_lo, (unsigned long long)i);
+    }
+    __syncthreads();
+    const uint64_t lo = s_lo;
+    if (lo == ~0ull) return; // no bucket starts here: the chunk is inside an earlier bucket
+    for (uint64_t i0 = cend; i0 < N; i0 += JOIN_THREADS) {
+        uint64_t i = i0 + threadIdx.x;
+        if (i < N && (A[i] >> bshift) != (A[i - 1] >> bshift))
+            atomicMin(&s_hi, (unsigned long long)i);
+        __syncthreads();
+        if (s_hi != ~0ull) break;
+        __syncthreads();
+    }
+    __syncthreads();
+    const uint64_t hi = (s_hi == ~0ull) ? N : (uint64_t)s_hi;
+    const uint64_t cnt = hi - lo;
+
+    Emitter em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * SEARCH_THREADS; base < a.V;
-         base += (uint64_t)gridDim.x * SEARCH_THREADS) {
-        const uint64_t u = base + threadIdx.x;
-        if (u < a.V && !(a.claimed && a.claimed[u])) {
-            const uint64_t q = a.sfxk[u];
-            const uint64_t d = q >> dshift;
-            const uint32_t lo = a.dir[d], hi = a.dir[d + 1];
-            for (uint32_t j = lo; j < hi; ++j) {
-                const uint64_t e = a.tab[j];
-                if ((e ^ q) > vmask) continue; // key bits differ
-                const uint32_t v = (uint32_t)(e & vmask);
-                const uint32_t b = v ^ 1u;
-                if ((u >> 1) == (v >> 1) || u >= b) continue; // R9; emit each pair once
-                if (a.claimed && a.claimed[b]) continue;
-                if (!verify_overlap<W>(a.packed, a.stride, a.L, (uint32_t)u, v, a.l)) {
-                    ++nfalse;
-                    continue;
-                }
-                const unsigned long long rec = ((unsigned long long)u << 32) | b;
-                uint32_t slot = atomicAdd(&bcount, 1u);
-                if (slot < SEARCH_BUF) buf[slot] = rec;
-                else {
-                    unsigned long long gs = atomicAdd(a.count, 1ull);
-                    if (gs < a.cap) a.pairs[gs] = rec;
-                }
-            }
+
+    if (cnt <= JOIN_CAP) {
+        // ---- stage, build the hash of prefix entries, probe with suffix entries
+        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) ent[k] = A[lo + k];
+        __syncthreads();
+        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) {
+            uint64_t e = ent[k];
+            if ((e >> a.vbits) & 1) continue; // suffix entry
+            uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
+            while (atomicCAS(&slot[h], SLOT_EMPTY, (unsigned short)k) != SLOT_EMPTY)
+                h = (h + 1) & (JOIN_SLOTS - 1);
         }
         __syncthreads();
-        const uint32_t c = bcount;
-        if (c >= SEARCH_BUF / 2) {
-            const uint32_t m = min(c, (uint32_t)SEARCH_BUF);
-            if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)m);
-            __syncthreads();
-            for (uint32_t t = threadIdx.x; t < m; t += SEARCH_THREADS)
-                if (gbase + t < a.cap) a.pairs[gbase + t] = buf[t];
-            __syncthreads();
-            if (threadIdx.x == 0) bcount = 0;
-            __syncthreads();
+        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) {
+            uint64_t e = ent[k];
+            if (!((e >> a.vbits) & 1)) continue; // prefix entry
+            uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
+            while (true) {
+                unsigned short s = slot[h];
+                if (s == SLOT_EMPTY) break;
+                uint64_t p = ent[s];
+                if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+                h = (h + 1) & (JOIN_SLOTS - 1);
+            }
+        }
+    } else {
+        // ---- oversized run of buckets (only with massively repeated fingerprints): every
+        // suffix entry scans its own bucket in global memory.
+        for (uint64_t i = lo + threadIdx.x; i < hi; i += JOIN_THREADS) {
+            uint64_t e = A[i];
+            if (!((e >> a.vbits) & 1)) continue;
+            const uint64_t bk = e >> bshift;
+            uint64_t j0 = i;
+            while (j0 > lo && (A[j0 - 1] >> bshift) == bk) --j0;
+            for (uint64_t j = j0; j < hi && (A[j] >> bshift) == bk; ++j) {
+                uint64_t p = A[j];
+                if (((p >> a.vbits) & 1) == 0 && ((p ^ e) >> kshift) == 0)
+                    candidate<W>(a, e, p, vmask, em, nfalse);
+            }
         }
     }
     __syncthreads();
-    const uint32_t m = min(bcount, (uint32_t)SEARCH_BUF);
+    const uint32_t m = min(bcount, (uint32_t)JOIN_BUF);
     if (m) {
         if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)m);
         __syncthreads();
-        for (uint32_t t = threadIdx.x; t < m; t += SEARCH_THREADS)
+        for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS)
             if (gbase + t < a.cap) a.pairs[gbase + t] = buf[t];
     }
-    // false-match count: warp reduce then one atomic per warp
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
 
-lasagna_status launch_dir(const uint64_t *tab, uint64_t V, uint32_t n_seg, uint32_t D,
-                          uint32_t *dir, cudaStream_t s)
+lasagna_status launch_join(const JoinArgs &args, cudaStream_t s)
 {
-    dim3 grid((unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(V, 256), 65535)), n_seg);
-    dir_kernel<<<grid, 256, 0, s>>>(tab, V, D, dir);
-    LSG_LAUNCHED("dir_kernel");
-    return LASAGNA_OK;
-}
-
-lasagna_status launch_search(const SearchArgs &args, cudaStream_t s)
-{
-    if (args.V == 0) return LASAGNA_OK;
+    if (args.N == 0) return LASAGNA_OK;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        int per_sm = 0;
-        LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, search_kernel<W>,
-                                                               SEARCH_THREADS, 0));
-        if (per_sm < 1) per_sm = 1;
-        uint64_t blocks = std::min<uint64_t>(ceil_div(args.V, SEARCH_THREADS),
-                                             (uint64_t)num_sms() * per_sm * 4);
-        search_kernel<W><<<(unsigned)blocks, SEARCH_THREADS, 0, s>>>(args);
-        LSG_LAUNCHED("search_kernel");
+        const uint64_t blocks = ceil_div(args.N, JOIN_CHUNK);
+        const size_t smem = (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 2;
+        LSG_CUDA(cudaFuncSetAttribute(join_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)smem));
+        join_kernel<W><<<(unsigned)blocks, JOIN_THREADS, smem, s>>>(args);
+        LSG_LAUNCHED("join_kernel");
         return LASAGNA_OK;
     });
 }
@@ -132,7 +181,8 @@ lasagna_status launch_search(const SearchArgs &args, cudaStream_t s)
 __global__ void pairs_to_keys(const unsigned long long *pool, const unsigned long long *count,
                               unsigned long long cap, uint32_t vbits, uint64_t *keys)
 {
-    const unsigned long long m = min(*count, cap);
+    const unsigned long long c = *count;
+    const unsigned long long m = c < cap ? c : cap;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
          i += (uint64_t)gridDim.x * blockDim.x) {
         unsigned long long r = pool[i];

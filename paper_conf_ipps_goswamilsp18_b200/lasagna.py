@@ -29,10 +29,10 @@ class _Stats(ctypes.Structure):
     _fields_ = [("n_pairs", ctypes.c_uint64), ("n_greedy", ctypes.c_uint64),
                 ("fp_false_matches", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
                 ("rounds_max", ctypes.c_uint32), ("passes", ctypes.c_uint32),
-                ("lengths_per_pass", ctypes.c_uint32), ("key_dir_bits", ctypes.c_uint32),
+                ("lengths_per_pass", ctypes.c_uint32), ("key_sort_bits", ctypes.c_uint32),
                 ("sort_launches", ctypes.c_uint32), ("search_launches", ctypes.c_uint32),
                 ("ms_table", ctypes.c_float), ("ms_sort", ctypes.c_float),
-                ("ms_dir", ctypes.c_float), ("ms_search", ctypes.c_float),
+                ("ms_search", ctypes.c_float),
                 ("ms_greedy", ctypes.c_float)]
 
     def as_dict(self) -> dict:
