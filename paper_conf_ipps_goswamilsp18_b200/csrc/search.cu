@@ -24,9 +24,9 @@ namespace lsg {
 constexpr int JOIN_THREADS = 512;
 constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
 constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
-constexpr int JOIN_SLOTS = 8192;   // u16 hash slots (load <= 0.75 even when all staged are P)
+constexpr int JOIN_SLOTS = 8192;   // u32 hash slots (> JOIN_CAP: the probe always ends)
 constexpr int JOIN_BUF = 1024;     // staged output pairs
-constexpr unsigned short SLOT_EMPTY = 0xFFFF;
+constexpr uint32_t SLOT_EMPTY = 0xFFFFFFFFu;
 
 struct Emitter {
     unsigned long long *buf;  // shared
@@ -57,100 +57,141 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t s_ent, uin
     em.emit(((unsigned long long)u << 32) | b);
 }
 
+// first index i in [lo, hi) with (A[i] >> shift) >= b (lower bound of bucket b), by one
+// warp: each round the 32 lanes probe 32 evenly spaced positions (32-ary search).
+__device__ __forceinline__ uint64_t warp_lower_bound(const uint64_t *A, uint64_t lo, uint64_t hi,
+                                                     uint32_t shift, uint64_t b)
+{
+    const int lane = threadIdx.x & 31;
+    while (hi - lo > 32) {
+        const uint64_t step = (hi - lo) / 33;
+        const uint64_t p = lo + (uint64_t)(lane + 1) * step;
+        const bool below = (A[p] >> shift) < b;
+        const uint32_t m = __ballot_sync(0xffffffffu, below);
+        const int k = 32 - __clz((int)m); // number of probes below b (they are a prefix)
+        const uint64_t nlo = k ? lo + (uint64_t)k * step + 1 : lo;
+        const uint64_t nhi = k < 32 ? lo + (uint64_t)(k + 1) * step : hi;
+        lo = nlo;
+        hi = nhi;
+    }
+    const uint64_t p = lo + lane;
+    const bool below = p < hi && (A[p] >> shift) < b;
+    return lo + __popc(__ballot_sync(0xffffffffu, below));
+}
+
+// Persistent join: CTA c owns the buckets [c*B/grid, (c+1)*B/grid) of the 2^T buckets and
+// streams their (contiguous) entries through shared memory in windows of whole buckets.
 template <int W>
-__global__ void __launch_bounds__(JOIN_THREADS)
+__global__ void __launch_bounds__(JOIN_THREADS, 2)
 join_kernel(JoinArgs a)
 {
     extern __shared__ __align__(16) unsigned char jsm[];
     uint64_t *ent = reinterpret_cast<uint64_t *>(jsm);                                   // [CAP]
     unsigned long long *buf = reinterpret_cast<unsigned long long *>(jsm + JOIN_CAP * 8); // [BUF]
-    unsigned short *slot = reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);
+    uint32_t *slot = reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);     // [SLOTS]
     __shared__ uint32_t bcount;
-    __shared__ unsigned long long gbase;
-    __shared__ unsigned long long s_lo, s_hi;
+    __shared__ unsigned long long gbase, s_r[2], s_cut, s_end;
 
     const uint64_t N = a.N;
-    const uint64_t base = (uint64_t)blockIdx.x * JOIN_CHUNK;
-    if (base >= N) return;
     const uint32_t bshift = 64 - a.T;
     const uint32_t kshift = a.vbits + 1; // key bits above tag + vid
     const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint64_t *A = a.keys;
+    const uint64_t B = 1ull << a.T;
+    const int warp = threadIdx.x >> 5;
 
-    if (threadIdx.x == 0) {
-        bcount = 0;
-        s_lo = ~0ull;
-        s_hi = ~0ull;
-    }
-    for (int t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = SLOT_EMPTY;
-    __syncthreads();
-
-    // bucket starts: i is a start if i == 0 or bucket(A[i]) != bucket(A[i-1]).
-    // lo = first start in [base, base+CHUNK); hi = first start >= base+CHUNK (or N).
-    const uint64_t cend = min64(N, base + JOIN_CHUNK);
-    for (uint64_t i = base + threadIdx.x; i < cend; i += JOIN_THREADS) {
-        bool st = (i == 0) || ((A[i] >> bshift) != (A[i - 1] >> bshift));
-        if (st) atomicMin(&s_lo, (unsigned long long)i);
+    if (threadIdx.x == 0) bcount = 0;
+    if (warp < 2) {
+        const uint64_t b = (B * (blockIdx.x + warp)) / gridDim.x;
+        const uint64_t r = (b >= B) ? N : warp_lower_bound(A, 0, N, bshift, b);
+        if ((threadIdx.x & 31) == 0) s_r[warp] = r;
     }
     __syncthreads();
-    const uint64_t lo = s_lo;
-    if (lo == ~0ull) return; // no bucket starts here: the chunk is inside an earlier bucket
-    for (uint64_t i0 = cend; i0 < N; i0 += JOIN_THREADS) {
-        uint64_t i = i0 + threadIdx.x;
-        if (i < N && (A[i] >> bshift) != (A[i - 1] >> bshift))
-            atomicMin(&s_hi, (unsigned long long)i);
-        __syncthreads();
-        if (s_hi != ~0ull) break;
-        __syncthreads();
-    }
-    __syncthreads();
-    const uint64_t hi = (s_hi == ~0ull) ? N : (uint64_t)s_hi;
-    const uint64_t cnt = hi - lo;
-
+    const uint64_t r0 = s_r[0], r1 = s_r[1];
     Emitter em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
 
-    if (cnt <= JOIN_CAP) {
-        // ---- stage, build the hash of prefix entries, probe with suffix entries
-        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) ent[k] = A[lo + k];
+    uint64_t t0 = r0;
+    while (t0 < r1) {
+        const uint32_t cnt = (uint32_t)min64(JOIN_CAP, r1 - t0);
+        if (threadIdx.x == 0) s_cut = 0;
+        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) ent[k] = A[t0 + k];
+        for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = SLOT_EMPTY;
         __syncthreads();
-        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) {
-            uint64_t e = ent[k];
-            if ((e >> a.vbits) & 1) continue; // suffix entry
-            uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-            while (atomicCAS(&slot[h], SLOT_EMPTY, (unsigned short)k) != SLOT_EMPTY)
-                h = (h + 1) & (JOIN_SLOTS - 1);
+        uint64_t t1;
+        if (t0 + cnt == r1) {
+            t1 = r1;
+        } else {
+            // last bucket start inside the window: the window is cut there
+            for (uint32_t k = 1 + threadIdx.x; k < cnt; k += JOIN_THREADS)
+                if ((ent[k] >> bshift) != (ent[k - 1] >> bshift)) atomicMax(&s_cut, (unsigned long long)k);
+            __syncthreads();
+            t1 = t0 + s_cut;
         }
-        __syncthreads();
-        for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) {
-            uint64_t e = ent[k];
-            if (!((e >> a.vbits) & 1)) continue; // prefix entry
-            uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-            while (true) {
-                unsigned short s = slot[h];
-                if (s == SLOT_EMPTY) break;
-                uint64_t p = ent[s];
-                if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-                h = (h + 1) & (JOIN_SLOTS - 1);
+        if (t1 == t0) {
+            // ---- one bucket larger than a window (massively repeated fingerprints): find its
+            // end in global memory, then every suffix entry scans the bucket there.
+            const uint64_t bk = ent[0] >> bshift;
+            if (threadIdx.x == 0) s_end = r1;
+            __syncthreads();
+            for (uint64_t i0 = t0 + cnt; i0 < r1; i0 += JOIN_THREADS) {
+                const uint64_t i = i0 + threadIdx.x;
+                if (i < r1 && (A[i] >> bshift) != bk) atomicMin(&s_end, (unsigned long long)i);
+                __syncthreads();
+                if (s_end != r1) break;
+                __syncthreads();
+            }
+            __syncthreads();
+            const uint64_t be = s_end;
+            for (uint64_t i = t0 + threadIdx.x; i < be; i += JOIN_THREADS) {
+                const uint64_t e = A[i];
+                if (!((e >> a.vbits) & 1)) continue;
+                for (uint64_t j = t0; j < be; ++j) {
+                    const uint64_t p = A[j];
+                    if (((p >> a.vbits) & 1) == 0 && ((p ^ e) >> kshift) == 0)
+                        candidate<W>(a, e, p, vmask, em, nfalse);
+                }
+            }
+            t1 = be;
+        } else {
+            // ---- hash the prefix entries of [t0, t1), probe with the suffix entries
+            const uint32_t m = (uint32_t)(t1 - t0);
+            for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
+                const uint64_t e = ent[k];
+                if ((e >> a.vbits) & 1) continue;
+                uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
+                while (atomicCAS(&slot[h], SLOT_EMPTY, k) != SLOT_EMPTY)
+                    h = (h + 1) & (JOIN_SLOTS - 1);
+            }
+            __syncthreads();
+            for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
+                const uint64_t e = ent[k];
+                if (!((e >> a.vbits) & 1)) continue;
+                uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
+                while (true) {
+                    const uint32_t sl = slot[h];
+                    if (sl == SLOT_EMPTY) break;
+                    const uint64_t p = ent[sl];
+                    if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+                    h = (h + 1) & (JOIN_SLOTS - 1);
+                }
             }
         }
-    } else {
-        // ---- oversized run of buckets (only with massively repeated fingerprints): every
-        // suffix entry scans its own bucket in global memory.
-        for (uint64_t i = lo + threadIdx.x; i < hi; i += JOIN_THREADS) {
-            uint64_t e = A[i];
-            if (!((e >> a.vbits) & 1)) continue;
-            const uint64_t bk = e >> bshift;
-            uint64_t j0 = i;
-            while (j0 > lo && (A[j0 - 1] >> bshift) == bk) --j0;
-            for (uint64_t j = j0; j < hi && (A[j] >> bshift) == bk; ++j) {
-                uint64_t p = A[j];
-                if (((p >> a.vbits) & 1) == 0 && ((p ^ e) >> kshift) == 0)
-                    candidate<W>(a, e, p, vmask, em, nfalse);
-            }
+        __syncthreads();
+        // flush staged pairs when half full
+        const uint32_t c = bcount;
+        if (c >= JOIN_BUF / 2) {
+            const uint32_t mm = min(c, (uint32_t)JOIN_BUF);
+            if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)mm);
+            __syncthreads();
+            for (uint32_t t = threadIdx.x; t < mm; t += JOIN_THREADS)
+                if (gbase + t < a.cap) a.pairs[gbase + t] = buf[t];
+            __syncthreads();
+            if (threadIdx.x == 0) bcount = 0;
         }
+        __syncthreads();
+        t0 = t1;
     }
-    __syncthreads();
     const uint32_t m = min(bcount, (uint32_t)JOIN_BUF);
     if (m) {
         if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)m);
@@ -167,10 +208,17 @@ lasagna_status launch_join(const JoinArgs &args, cudaStream_t s)
     if (args.N == 0) return LASAGNA_OK;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const uint64_t blocks = ceil_div(args.N, JOIN_CHUNK);
-        const size_t smem = (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 2;
+        const size_t smem = (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 4;
         LSG_CUDA(cudaFuncSetAttribute(join_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)smem));
+        int per_sm = 0;
+        LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, join_kernel<W>,
+                                                               JOIN_THREADS, smem));
+        per_sm = std::max(per_sm, 1);
+        // persistent grid, but never more CTAs than ~one window of entries each
+        uint64_t blocks = std::min<uint64_t>((uint64_t)num_sms() * per_sm,
+                                             std::max<uint64_t>(1, args.N / JOIN_CHUNK));
+        blocks = std::min<uint64_t>(blocks, 1ull << args.T);
         join_kernel<W><<<(unsigned)blocks, JOIN_THREADS, smem, s>>>(args);
         LSG_LAUNCHED("join_kernel");
         return LASAGNA_OK;
