@@ -24,18 +24,24 @@ __device__ __forceinline__ uint64_t mod61(uint64_t x)
     return r >= Q61 ? r - Q61 : r;
 }
 
-// Horner step P <- P*5 + c (P < q, c <= 3: 5P + c < 2^64, no 128-bit product needed).
+// Lazily reduced arithmetic: values are kept in [0, 2^61 + 7) ("folded", congruent mod q);
+// fold(x) = (x & q) + (x >> 61) maps any x < 2^64 there with 4 32-bit ops and no compare.
+__device__ __forceinline__ uint64_t fold61(uint64_t x) { return (x & Q61) + (x >> 61); }
+// exact residue of a folded value
+__device__ __forceinline__ uint64_t exact61(uint64_t x) { return x >= Q61 ? x - Q61 : x; }
+
+// Horner step P <- P*5 + c on folded P (5(2^61+7) + 3 < 2^64: no 128-bit product).
 __device__ __forceinline__ uint64_t horner5(uint64_t P, uint32_t c)
 {
-    return mod61((P << 2) + P + c);
+    return fold61((P << 2) + P + c);
 }
 
 // Ascending-power step S <- S + c * pw (pw = 5^j mod q, pw2 = 2 pw mod q, c <= 3):
-// c*pw = (c&1)pw + (c&2 ? pw2 : 0), sum < 3q < 2^63.
+// c*pw = (c&1)pw + (c&2 ? pw2 : 0); folded S + c*pw < 2^61 + 7 + 2^62 < 2^64.
 __device__ __forceinline__ uint64_t addpow(uint64_t S, uint32_t c, uint64_t pw, uint64_t pw2)
 {
     uint64_t t = S + ((c & 1u) ? pw : 0ull) + ((c & 2u) ? pw2 : 0ull);
-    return mod61(t);
+    return fold61(t);
 }
 
 // Table key mixing: a bijection of the 64-bit word (multiplication by an odd constant mod

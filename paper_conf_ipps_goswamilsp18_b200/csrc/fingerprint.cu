@@ -15,27 +15,45 @@
 
 namespace lsg {
 
-struct FpStreams {
-    uint64_t P0, P1, S0, S1, pw, pw2;
-    __device__ __forceinline__ void init()
-    {
-        P0 = P1 = S0 = S1 = 0;
-        pw = 1;
-        pw2 = 2;
+// Place values M[j] = 5^j mod q and 2 M[j] mod q ("computed once for the entire
+// program"), j < 256, built at compile time into constant memory: every lane of a warp reads
+// the same j in the same step, so the constant cache broadcasts them.
+struct PowTable {
+    uint64_t m[256], m2[256];
+};
+constexpr uint64_t host_fold_exact(uint64_t x)
+{
+    uint64_t r = (x & Q61) + (x >> 61);
+    return r >= Q61 ? r - Q61 : r;
+}
+constexpr PowTable make_pow_table()
+{
+    PowTable t{};
+    uint64_t p = 1;
+    for (int j = 0; j < 256; ++j) {
+        t.m[j] = p;
+        t.m2[j] = host_fold_exact(p << 1);
+        p = host_fold_exact((p << 2) + p);
     }
+    return t;
+}
+__constant__ PowTable c_pow = make_pow_table();
+
+struct FpStreams {
+    uint64_t P0, P1, S0, S1; // folded (congruent mod q, < 2^61 + 7)
+    __device__ __forceinline__ void init() { P0 = P1 = S0 = S1 = 0; }
     // consume base j of r (ca) and of r' (cb)
-    __device__ __forceinline__ void step(uint32_t ca, uint32_t cb)
+    __device__ __forceinline__ void step(uint32_t ca, uint32_t cb, uint32_t j)
     {
+        const uint64_t pw = c_pow.m[j], pw2 = c_pow.m2[j];
         P0 = horner5(P0, ca);
         P1 = horner5(P1, cb);
         S1 = addpow(S1, ca ^ 2u, pw, pw2);
         S0 = addpow(S0, cb ^ 2u, pw, pw2);
-        pw = mod61((pw << 2) + pw);
-        pw2 = mod61(pw << 1);
     }
 };
 
-// Visit lengths l = 1..l_end; call emit(l, st) after base l-1.
+// Visit lengths l = 1..l_end; call emit(l, st) after base l-1 (values folded: use exact61).
 template <int W, typename Emit>
 __device__ __forceinline__ void roll_read(const uint64_t (&x)[W], const uint64_t (&y)[W],
                                           uint32_t l_end, Emit &&emit)
@@ -49,7 +67,7 @@ __device__ __forceinline__ void roll_read(const uint64_t (&x)[W], const uint64_t
         if (k0 >= l_end) break;
         const uint32_t kn = min(32u, l_end - k0);
         for (uint32_t j = 0; j < kn; ++j) {
-            st.step((uint32_t)(a & 3u), (uint32_t)(b & 3u));
+            st.step((uint32_t)(a & 3u), (uint32_t)(b & 3u), k0 + j);
             a >>= 2;
             b >>= 2;
             emit(k0 + j + 1, st);
@@ -72,8 +90,12 @@ fp_values_kernel(const uint64_t *__restrict__ packed, uint64_t n, uint32_t L, ui
         roll_read<W>(x, y, L, [&](uint32_t l, const FpStreams &st) {
             if (l < l_min) return;
             const uint64_t off = (uint64_t)(l - l_min) * V + 2 * i;
-            if (pfx) *reinterpret_cast<ulonglong2 *>(pfx + off) = make_ulonglong2(st.P0, st.P1);
-            if (sfx) *reinterpret_cast<ulonglong2 *>(sfx + off) = make_ulonglong2(st.S0, st.S1);
+            if (pfx)
+                *reinterpret_cast<ulonglong2 *>(pfx + off) =
+                    make_ulonglong2(exact61(st.P0), exact61(st.P1));
+            if (sfx)
+                *reinterpret_cast<ulonglong2 *>(sfx + off) =
+                    make_ulonglong2(exact61(st.S0), exact61(st.S1));
         });
     }
 }
@@ -121,8 +143,10 @@ table_kernel(TableArgs a)
             if (l < a.l_lo) return;
             const uint32_t s = l - a.l_lo;
             const uint64_t v0 = 2 * i, v1 = 2 * i + 1;
-            const uint64_t p0 = (mix(st.P0) & keep) | v0, s0 = (mix(st.S0) & keep) | tagS | v0;
-            const uint64_t p1 = (mix(st.P1) & keep) | v1, s1 = (mix(st.S1) & keep) | tagS | v1;
+            const uint64_t p0 = (mix(exact61(st.P0)) & keep) | v0;
+            const uint64_t s0 = (mix(exact61(st.S0)) & keep) | tagS | v0;
+            const uint64_t p1 = (mix(exact61(st.P1)) & keep) | v1;
+            const uint64_t s1 = (mix(exact61(st.S1)) & keep) | tagS | v1;
             ulonglong2 *dst = reinterpret_cast<ulonglong2 *>(a.tab + (uint64_t)s * N + 4 * i);
             dst[0] = make_ulonglong2(p0, s0);
             dst[1] = make_ulonglong2(p1, s1);

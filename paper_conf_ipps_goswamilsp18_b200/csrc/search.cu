@@ -24,7 +24,7 @@ namespace lsg {
 constexpr int JOIN_THREADS = 512;
 constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
 constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
-constexpr int JOIN_SLOTS = 8192;   // u32 hash slots (> JOIN_CAP: the probe always ends)
+constexpr int JOIN_SLOTS = 8192;   // hash chain heads (u32); chains through next[] (u16)
 constexpr int JOIN_BUF = 1024;     // staged output pairs
 constexpr uint32_t SLOT_EMPTY = 0xFFFFFFFFu;
 
@@ -89,6 +89,8 @@ join_kernel(JoinArgs a)
     uint64_t *ent = reinterpret_cast<uint64_t *>(jsm);                                   // [CAP]
     unsigned long long *buf = reinterpret_cast<unsigned long long *>(jsm + JOIN_CAP * 8); // [BUF]
     uint32_t *slot = reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);     // [SLOTS]
+    unsigned short *next =
+        reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4); // [CAP]
     __shared__ uint32_t bcount;
     __shared__ unsigned long long gbase, s_r[2], s_cut, s_end;
 
@@ -154,26 +156,25 @@ join_kernel(JoinArgs a)
             }
             t1 = be;
         } else {
-            // ---- hash the prefix entries of [t0, t1), probe with the suffix entries
+            // ---- hash the prefix entries of [t0, t1) (chained: one atomicExch per insert),
+            // then probe with the suffix entries
             const uint32_t m = (uint32_t)(t1 - t0);
             for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
                 const uint64_t e = ent[k];
                 if ((e >> a.vbits) & 1) continue;
-                uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-                while (atomicCAS(&slot[h], SLOT_EMPTY, k) != SLOT_EMPTY)
-                    h = (h + 1) & (JOIN_SLOTS - 1);
+                const uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
+                next[k] = (unsigned short)atomicExch(&slot[h], k);
             }
             __syncthreads();
             for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
                 const uint64_t e = ent[k];
                 if (!((e >> a.vbits) & 1)) continue;
-                uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-                while (true) {
-                    const uint32_t sl = slot[h];
-                    if (sl == SLOT_EMPTY) break;
+                uint32_t sl = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
+                while (sl != SLOT_EMPTY) {
                     const uint64_t p = ent[sl];
                     if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-                    h = (h + 1) & (JOIN_SLOTS - 1);
+                    sl = next[sl];
+                    if (sl == 0xFFFFu) break;
                 }
             }
         }
@@ -208,7 +209,8 @@ lasagna_status launch_join(const JoinArgs &args, cudaStream_t s)
     if (args.N == 0) return LASAGNA_OK;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 4;
+        const size_t smem =
+            (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 4 + (size_t)JOIN_CAP * 2;
         LSG_CUDA(cudaFuncSetAttribute(join_kernel<W>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)smem));
         int per_sm = 0;

@@ -94,49 +94,42 @@ onesweep_kernel(SortPassArgs a)
         if (tid < 256) dofs[tid] = ex;
     }
 
-    // load (warp-blocked: warp w owns keys [w*512, w*512+512), lane-strided) and rank
+    // load (warp-blocked: warp w owns keys [w*512, w*512+512), lane-strided)
     uint64_t key[SORT_KPT];
-    uint32_t rank[SORT_KPT];
     const uint64_t *src = a.in + seg_base + tile_lo;
 #pragma unroll
     for (int i = 0; i < SORT_KPT; ++i) {
         uint32_t idx = warp * (32 * SORT_KPT) + i * 32 + lane;
         key[i] = idx < cnt ? src[idx] : 0ull;
     }
+    // early counts: per-warp digit histograms (order-free atomics)
     uint32_t *mycnt = wcnt + warp * 256;
 #pragma unroll
     for (int i = 0; i < SORT_KPT; ++i) {
         uint32_t idx = warp * (32 * SORT_KPT) + i * 32 + lane;
-        bool valid = idx < cnt;
-        uint32_t d = valid ? (uint32_t)((key[i] >> a.shift) & dmask) : 256u + lane;
-        uint32_t peers = __match_any_sync(0xffffffffu, d);
-        uint32_t lower = __popc(peers & lanemask_lt());
-        uint32_t before = valid ? mycnt[d] : 0u;
-        __syncwarp();
-        if (valid && lower == 0) mycnt[d] = before + __popc(peers);
-        __syncwarp();
-        rank[i] = before + lower;
+        if (idx < cnt) atomicAdd(&mycnt[(uint32_t)((key[i] >> a.shift) & dmask)], 1u);
     }
     __syncthreads();
 
-    // per digit: exclusive over warps, then exclusive over digits (local tile offsets)
+    // per digit: totals, exclusive over digits (local tile offsets), then each warp's start
     uint32_t total = 0;
     if (tid < 256) {
-        uint32_t run = 0;
-        for (int w = 0; w < SORT_WARPS; ++w) {
-            uint32_t c = wcnt[w * 256 + tid];
-            wcnt[w * 256 + tid] = run;
-            run += c;
-        }
-        total = run;
+        for (int w = 0; w < SORT_WARPS; ++w) total += wcnt[w * 256 + tid];
     }
     {
         uint32_t ex = scan256(total, wsum);
-        if (tid < 256) lstart[tid] = ex;
+        if (tid < 256) {
+            lstart[tid] = ex;
+            uint32_t run = ex;
+            for (int w = 0; w < SORT_WARPS; ++w) {
+                uint32_t c = wcnt[w * 256 + tid];
+                wcnt[w * 256 + tid] = run;
+                run += c;
+            }
+        }
     }
-    __syncthreads();
 
-    // decoupled look-back: global offset of this tile's run of each digit
+    // decoupled look-back on the early counts: global offset of each digit's run of this tile
     if (tid < 256) {
         unsigned long long *my = a.status + (uint64_t)g * 256 + tid;
         const unsigned long long ep = (unsigned long long)a.epoch << 48;
@@ -160,15 +153,23 @@ onesweep_kernel(SortPassArgs a)
             gbase[tid] = dofs[tid] + (uint32_t)excl;
         }
     }
+    __syncthreads();
 
-    // scatter into the shared tile in stable digit order
+    // stable ranking straight into the tile's sorted position: keys are visited in their
+    // original order (i, lane); the group leader reserves popc(peers) slots of the warp's
+    // run of the digit with one shared atomic (issued in program order within the warp)
 #pragma unroll
     for (int i = 0; i < SORT_KPT; ++i) {
         uint32_t idx = warp * (32 * SORT_KPT) + i * 32 + lane;
-        if (idx < cnt) {
-            uint32_t d = (uint32_t)((key[i] >> a.shift) & dmask);
-            skeys[lstart[d] + wcnt[warp * 256 + d] + rank[i]] = key[i];
-        }
+        bool valid = idx < cnt;
+        uint32_t d = valid ? (uint32_t)((key[i] >> a.shift) & dmask) : 256u + lane;
+        uint32_t peers = __match_any_sync(0xffffffffu, d);
+        int leader = 31 - __clz((int)peers);
+        uint32_t lower = __popc(peers & lanemask_lt());
+        uint32_t base_pos = 0;
+        if (valid && lane == leader) base_pos = atomicAdd(&mycnt[d], __popc(peers));
+        base_pos = __shfl_sync(0xffffffffu, base_pos, leader);
+        if (valid) skeys[base_pos + lower] = key[i];
     }
     __syncthreads();
 
