@@ -28,33 +28,71 @@ constexpr int JOIN_SLOTS = 8192;   // hash chain heads (u32); chains through nex
 constexpr int JOIN_BUF = 1024;     // staged output pairs
 constexpr uint32_t SLOT_EMPTY = 0xFFFFFFFFu;
 
-struct Emitter {
-    unsigned long long *buf;  // shared
-    uint32_t *bcount;         // shared
+// Candidates are staged in shared memory and verified in a separate, fully parallel pass
+// (a fingerprint match is rare: verifying it inline would run the long verify path with one
+// or two active lanes per warp).
+struct Stager {
+    unsigned long long *buf; // shared: staged (u << 32 | b) records, ~0 = rejected
+    uint32_t *bcount;        // shared
     unsigned long long *pairs, cap, *count;
-    __device__ __forceinline__ void emit(unsigned long long rec)
-    {
-        uint32_t slot = atomicAdd(bcount, 1u);
-        if (slot < JOIN_BUF) buf[slot] = rec;
-        else {
-            unsigned long long gs = atomicAdd(count, 1ull);
-            if (gs < cap) pairs[gs] = rec;
-        }
-    }
 };
 
 template <int W>
 __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t s_ent, uint64_t p_ent,
-                                          uint64_t vmask, Emitter &em, unsigned long long &nfalse)
+                                          uint64_t vmask, Stager &sg, unsigned long long &nfalse)
 {
     const uint32_t u = (uint32_t)(s_ent & vmask), v = (uint32_t)(p_ent & vmask);
     const uint32_t b = v ^ 1u;
     if ((u >> 1) == (v >> 1) || u >= b) return; // R9: no same-read edge; each pair once
+    const unsigned long long rec = ((unsigned long long)u << 32) | b;
+    const uint32_t slot = atomicAdd(sg.bcount, 1u);
+    if (slot < JOIN_BUF) {
+        sg.buf[slot] = rec;
+        return;
+    }
+    // staging full: verify inline and emit straight to global memory
     if (!verify_overlap<W>(a.packed, a.stride, a.L, u, v, a.l)) {
         ++nfalse;
         return;
     }
-    em.emit(((unsigned long long)u << 32) | b);
+    const unsigned long long gs = atomicAdd(sg.count, 1ull);
+    if (gs < sg.cap) sg.pairs[gs] = rec;
+}
+
+// verify staged records [from, to) in parallel; rejected ones become ~0
+template <int W>
+__device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long long *buf,
+                                              uint32_t from, uint32_t to, unsigned long long &nfalse)
+{
+    for (uint32_t t = from + threadIdx.x; t < to; t += JOIN_THREADS) {
+        const unsigned long long rec = buf[t];
+        const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
+        if (!verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
+            buf[t] = ~0ull;
+            ++nfalse;
+        }
+    }
+}
+
+// write the accepted staged records [0, m) to the global pool (warp-aggregated slots)
+__device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint32_t m,
+                                             unsigned long long *pairs, unsigned long long cap,
+                                             unsigned long long *count)
+{
+    const int lane = threadIdx.x & 31;
+    for (uint32_t t0 = 0; t0 < m; t0 += JOIN_THREADS) {
+        const uint32_t t = t0 + threadIdx.x;
+        const unsigned long long rec = t < m ? buf[t] : ~0ull;
+        const bool ok = rec != ~0ull;
+        const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+        unsigned long long base = 0;
+        if (lane == 0 && bal) base = atomicAdd(count, (unsigned long long)__popc(bal));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (ok) {
+            const unsigned long long pos = base + __popc(bal & ((1u << lane) - 1));
+            if (pos < cap) pairs[pos] = rec;
+        }
+    }
 }
 
 // first index i in [lo, hi) with (A[i] >> shift) >= b (lower bound of bucket b), by one
@@ -91,8 +129,8 @@ join_kernel(JoinArgs a)
     uint32_t *slot = reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);     // [SLOTS]
     unsigned short *next =
         reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4); // [CAP]
-    __shared__ uint32_t bcount;
-    __shared__ unsigned long long gbase, s_r[2], s_cut, s_end;
+    __shared__ uint32_t bcount, vdone;
+    __shared__ unsigned long long s_r[2], s_cut, s_end;
 
     const uint64_t N = a.N;
     const uint32_t bshift = 64 - a.T;
@@ -102,7 +140,7 @@ join_kernel(JoinArgs a)
     const uint64_t B = 1ull << a.T;
     const int warp = threadIdx.x >> 5;
 
-    if (threadIdx.x == 0) bcount = 0;
+    if (threadIdx.x == 0) bcount = 0, vdone = 0;
     if (warp < 2) {
         const uint64_t b = (B * (blockIdx.x + warp)) / gridDim.x;
         const uint64_t r = (b >= B) ? N : warp_lower_bound(A, 0, N, bshift, b);
@@ -110,7 +148,7 @@ join_kernel(JoinArgs a)
     }
     __syncthreads();
     const uint64_t r0 = s_r[0], r1 = s_r[1];
-    Emitter em{buf, &bcount, a.pairs, a.cap, a.count};
+    Stager em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
 
     uint64_t t0 = r0;
@@ -179,27 +217,23 @@ join_kernel(JoinArgs a)
             }
         }
         __syncthreads();
-        // flush staged pairs when half full
-        const uint32_t c = bcount;
-        if (c >= JOIN_BUF / 2) {
-            const uint32_t mm = min(c, (uint32_t)JOIN_BUF);
-            if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)mm);
+        // verify this window's candidates, flush the staging buffer when half full
+        {
+            const uint32_t to = min(bcount, (uint32_t)JOIN_BUF);
+            verify_staged<W>(a, buf, vdone, to, nfalse);
             __syncthreads();
-            for (uint32_t t = threadIdx.x; t < mm; t += JOIN_THREADS)
-                if (gbase + t < a.cap) a.pairs[gbase + t] = buf[t];
-            __syncthreads();
-            if (threadIdx.x == 0) bcount = 0;
+            if (to >= JOIN_BUF / 2) {
+                flush_staged(buf, to, a.pairs, a.cap, a.count);
+                __syncthreads();
+                if (threadIdx.x == 0) bcount = 0, vdone = 0;
+            } else if (threadIdx.x == 0) {
+                vdone = to;
+            }
         }
         __syncthreads();
         t0 = t1;
     }
-    const uint32_t m = min(bcount, (uint32_t)JOIN_BUF);
-    if (m) {
-        if (threadIdx.x == 0) gbase = atomicAdd(a.count, (unsigned long long)m);
-        __syncthreads();
-        for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS)
-            if (gbase + t < a.cap) a.pairs[gbase + t] = buf[t];
-    }
+    flush_staged(buf, min(bcount, (uint32_t)JOIN_BUF), a.pairs, a.cap, a.count);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }

@@ -39,6 +39,19 @@ struct SortPassArgs {
     uint32_t epoch;
 };
 
+// look-back words are single 64-bit values (flag and count together): relaxed GPU-scope
+// accesses suffice (no other data is published through them)
+__device__ __forceinline__ void st_relaxed(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ uint32_t lanemask_lt()
 {
     uint32_t m;
@@ -77,7 +90,8 @@ onesweep_kernel(SortPassArgs a)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) s_tile = atomicAdd(a.tile_ctr, 1u);
-    for (int t = tid; t < SORT_WARPS * 256; t += SORT_THREADS) wcnt[t] = 0;
+    for (int t = tid; t < SORT_WARPS * 256 / 4; t += SORT_THREADS)
+        reinterpret_cast<uint4 *>(wcnt)[t] = make_uint4(0, 0, 0, 0);
     if (tid < 256) nhist[tid] = 0;
     __syncthreads();
     const uint32_t g = s_tile;
@@ -134,22 +148,22 @@ onesweep_kernel(SortPassArgs a)
         unsigned long long *my = a.status + (uint64_t)g * 256 + tid;
         const unsigned long long ep = (unsigned long long)a.epoch << 48;
         if (t == 0) {
-            *(volatile unsigned long long *)my = ep | ST_PREFIX | total;
+            st_relaxed(my, ep | ST_PREFIX | total);
             gbase[tid] = dofs[tid];
         } else {
-            *(volatile unsigned long long *)my = ep | total;
+            st_relaxed(my, ep | total);
             unsigned long long excl = 0;
             uint64_t p = (uint64_t)g - 1;
             while (true) {
                 unsigned long long w;
                 do {
-                    w = *(volatile unsigned long long *)(a.status + p * 256 + tid);
+                    w = ld_relaxed(a.status + p * 256 + tid);
                 } while ((w >> 48) != (unsigned long long)a.epoch);
                 excl += w & ST_VALUE;
                 if (w & ST_PREFIX) break;
                 --p;
             }
-            *(volatile unsigned long long *)my = ep | ST_PREFIX | (excl + total);
+            st_relaxed(my, ep | ST_PREFIX | (excl + total));
             gbase[tid] = dofs[tid] + (uint32_t)excl;
         }
     }
