@@ -176,8 +176,17 @@ onesweep_kernel(SortPassArgs a)
     for (int i = 0; i < SORT_KPT; ++i) {
         uint32_t idx = warp * (32 * SORT_KPT) + i * 32 + lane;
         bool valid = idx < cnt;
-        uint32_t d = valid ? (uint32_t)((key[i] >> a.shift) & dmask) : 256u + lane;
-        uint32_t peers = __match_any_sync(0xffffffffu, d);
+        uint32_t d = valid ? (uint32_t)((key[i] >> a.shift) & dmask) : 0u;
+        // peers with the same digit: bit-sliced multi-split with 8 ballots (cheaper than
+        // match.any on this part), restricted to valid lanes
+        uint32_t peers = __ballot_sync(0xffffffffu, valid);
+#pragma unroll
+        for (int bb = 0; bb < 8; ++bb) {
+            const bool bit = (d >> bb) & 1u;
+            const uint32_t m = __ballot_sync(0xffffffffu, bit);
+            peers &= bit ? m : ~m;
+        }
+        if (!valid) peers = 1u << lane;
         int leader = 31 - __clz((int)peers);
         uint32_t lower = __popc(peers & lanemask_lt());
         uint32_t base_pos = 0;
