@@ -14,141 +14,184 @@
 
 namespace lsg {
 
-__global__ void greedy_init(const unsigned long long *pairs, const unsigned long long *count,
-                            uint32_t *best0, uint32_t *best1)
+// Proposals are epoch-tagged 64-bit words best[x] = (epoch << 32) | ~partner combined with
+// atomicMax: within a round the largest word is the smallest partner, and words of earlier
+// rounds (smaller epochs) lose automatically, so best[] is never reset between rounds or
+// lengths (it is zeroed once per call).  No host synchronisation anywhere: every kernel
+// reads its pair count from device memory.
+__device__ __forceinline__ unsigned long long proposal(uint32_t epoch, uint32_t partner)
 {
-    const unsigned long long m = *count;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        unsigned long long r = pairs[i];
-        uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
-        best0[a] = NONE, best0[b] = NONE, best1[a] = NONE, best1[b] = NONE;
-    }
+    return ((unsigned long long)epoch << 32) | (unsigned long long)(~partner);
 }
 
 __global__ void greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
-                               const uint8_t *claimed, uint32_t *best)
+                               unsigned long long cap, const uint8_t *claimed,
+                               unsigned long long *best, uint32_t epoch,
+                               unsigned long long *out_count, unsigned long long *book)
 {
-    const unsigned long long m = *count;
+    const unsigned long long c = *count;
+    const unsigned long long m = c < cap ? c : cap;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *out_count = 0;
+        if (book) { // first round of a length: |P_l| bookkeeping
+            atomicAdd(&book[1], c);
+            atomicMax(&book[2], c);
+        }
+    }
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
          i += (uint64_t)gridDim.x * blockDim.x) {
-        unsigned long long r = pairs[i];
-        uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
+        const unsigned long long r = pairs[i];
+        const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
         if (claimed[a] | claimed[b]) continue;
-        atomicMin(&best[a], b);
-        atomicMin(&best[b], a);
+        atomicMax(&best[a], proposal(epoch, b));
+        atomicMax(&best[b], proposal(epoch, a));
     }
 }
 
-__global__ void greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
-                              uint8_t *claimed, const uint32_t *best, uint32_t *best_next,
-                              uint32_t *succ, uint8_t *olen, uint8_t l,
-                              unsigned long long *out, unsigned long long *out_count,
-                              unsigned long long *accepted)
+__device__ __forceinline__ void accept_pair(uint32_t a, uint32_t b, uint8_t *claimed, uint32_t *succ,
+                                            uint8_t *olen, uint8_t l)
 {
-    const unsigned long long m = *count;
+    claimed[a] = 1, claimed[b] = 1;
+    succ[a] = b ^ 1u, succ[b] = a ^ 1u; // edges a -> b^1 and (complement) b -> a^1
+    olen[a] = l, olen[b] = l;
+}
+
+__global__ void greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
+                              unsigned long long cap, uint8_t *claimed,
+                              const unsigned long long *best, uint32_t epoch, uint32_t *succ,
+                              uint8_t *olen, uint8_t l, unsigned long long *out,
+                              unsigned long long *out_count, unsigned long long *book)
+{
+    const unsigned long long c = *count;
+    const unsigned long long m = c < cap ? c : cap;
     uint32_t acc = 0;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
          i += (uint64_t)gridDim.x * blockDim.x) {
-        unsigned long long r = pairs[i];
-        uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
+        const unsigned long long r = pairs[i];
+        const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
         if (claimed[a] | claimed[b]) continue; // dead: an end was taken in an earlier round
-        if (best[a] == b && best[b] == a) {
-            claimed[a] = 1, claimed[b] = 1;
-            succ[a] = b ^ 1u, succ[b] = a ^ 1u;
-            olen[a] = l, olen[b] = l;
+        if (best[a] == proposal(epoch, b) && best[b] == proposal(epoch, a)) {
+            accept_pair(a, b, claimed, succ, olen, l);
             ++acc;
         } else {
-            best_next[a] = NONE, best_next[b] = NONE;
             out[atomicAdd(out_count, 1ull)] = r;
         }
     }
     for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if ((threadIdx.x & 31) == 0 && acc) atomicAdd(accepted, (unsigned long long)acc);
+    if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&book[0], (unsigned long long)acc);
 }
 
 constexpr int TAIL_MAX = 4096;
+constexpr int FINISH_THREADS = 1024;
 
-// Sequential definition on the remaining pairs: bitonic sort by (a, b) in shared memory,
-// then one thread visits them in order.
-__global__ void __launch_bounds__(1024)
-greedy_tail(const unsigned long long *pairs, const unsigned long long *count, uint8_t *claimed,
-            uint32_t *succ, uint8_t *olen, uint8_t l, unsigned long long *accepted)
+// Finishes one length on a single CTA: locally-dominant rounds with block barriers while more
+// than TAIL_MAX pairs are live, then the sequential definition itself (bitonic sort by
+// (a, b) in shared memory, one thread visits the pairs in order).
+__global__ void __launch_bounds__(FINISH_THREADS)
+greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
+              unsigned long long *other, unsigned long long *other_count, uint8_t *claimed,
+              unsigned long long *best, uint32_t epoch, uint32_t fast_rounds, uint32_t *succ,
+              uint8_t *olen, uint8_t l, unsigned long long *book)
 {
     __shared__ unsigned long long s[TAIL_MAX];
-    const unsigned long long cnt_ = *count;
-    const uint32_t m = (uint32_t)(cnt_ < (unsigned long long)TAIL_MAX ? cnt_ : (unsigned long long)TAIL_MAX);
-    uint32_t P = 1;
-    while (P < m) P <<= 1;
-    for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) s[i] = i < m ? pairs[i] : ~0ull;
-    __syncthreads();
-    for (uint32_t k = 2; k <= P; k <<= 1)
-        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
-            for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) {
-                uint32_t ixj = i ^ j;
-                if (ixj > i) {
-                    bool up = (i & k) == 0;
-                    unsigned long long x = s[i], y = s[ixj];
-                    if ((x > y) == up) s[i] = y, s[ixj] = x;
-                }
-            }
-            __syncthreads();
-        }
-    if (threadIdx.x == 0) {
-        unsigned long long acc = 0;
-        for (uint32_t i = 0; i < m; ++i) {
-            uint32_t a = (uint32_t)(s[i] >> 32), b = (uint32_t)s[i];
+    __shared__ uint32_t s_live, s_acc;
+    uint32_t live = (uint32_t)*cur_count;
+    uint32_t rounds = fast_rounds;
+    if (threadIdx.x == 0) s_acc = 0;
+    while (live > (uint32_t)TAIL_MAX) {
+        for (uint32_t i = threadIdx.x; i < live; i += FINISH_THREADS) {
+            const unsigned long long r = cur[i];
+            const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
             if (claimed[a] | claimed[b]) continue;
-            claimed[a] = 1, claimed[b] = 1;
-            succ[a] = b ^ 1u, succ[b] = a ^ 1u;
-            olen[a] = l, olen[b] = l;
-            ++acc;
+            atomicMax(&best[a], proposal(epoch, b));
+            atomicMax(&best[b], proposal(epoch, a));
         }
-        if (acc) atomicAdd(accepted, acc);
+        if (threadIdx.x == 0) s_live = 0;
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < live; i += FINISH_THREADS) {
+            const unsigned long long r = cur[i];
+            const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
+            if (claimed[a] | claimed[b]) continue;
+            if (best[a] == proposal(epoch, b) && best[b] == proposal(epoch, a)) {
+                accept_pair(a, b, claimed, succ, olen, l);
+                atomicAdd(&s_acc, 1u);
+            } else {
+                other[atomicAdd(&s_live, 1u)] = r;
+            }
+        }
+        __syncthreads();
+        live = s_live;
+        unsigned long long *t = cur;
+        cur = other;
+        other = t;
+        ++epoch;
+        ++rounds;
+        __syncthreads();
     }
+    if (live) {
+        uint32_t P = 1;
+        while (P < live) P <<= 1;
+        for (uint32_t i = threadIdx.x; i < P; i += FINISH_THREADS) s[i] = i < live ? cur[i] : ~0ull;
+        __syncthreads();
+        for (uint32_t k = 2; k <= P; k <<= 1)
+            for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+                for (uint32_t i = threadIdx.x; i < P; i += FINISH_THREADS) {
+                    const uint32_t ixj = i ^ j;
+                    if (ixj > i) {
+                        const bool up = (i & k) == 0;
+                        const unsigned long long x = s[i], y = s[ixj];
+                        if ((x > y) == up) s[i] = y, s[ixj] = x;
+                    }
+                }
+                __syncthreads();
+            }
+        if (threadIdx.x == 0) {
+            uint32_t acc = 0;
+            for (uint32_t i = 0; i < live; ++i) {
+                const uint32_t a = (uint32_t)(s[i] >> 32), b = (uint32_t)s[i];
+                if (claimed[a] | claimed[b]) continue;
+                accept_pair(a, b, claimed, succ, olen, l);
+                ++acc;
+            }
+            s_acc += acc;
+            ++rounds;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (s_acc) atomicAdd(&book[0], (unsigned long long)s_acc);
+        atomicMax(&book[3], (unsigned long long)rounds);
+    }
+    (void)other_count;
 }
 
+constexpr uint32_t FAST_ROUNDS = 3;
+constexpr uint32_t EPOCHS_PER_LENGTH = 1u << 22; // fast rounds + at most ~4M finishing rounds
 
-// Greedy over the m pairs of length l in bufs.pool (count in *bufs.cnt, device; m its host
-// copy).  Synchronises the stream once per round.
-lasagna_status greedy_length(GreedyBufs &g, uint64_t m, uint8_t l, uint32_t *succ, uint8_t *olen,
-                             cudaStream_t s, uint32_t *rounds_out)
+// Greedy over the pairs of length l in g.pool (count in *g.cnt, device).  Fully
+// asynchronous: FAST_ROUNDS grid-wide rounds, then one CTA finishes the (few) survivors.
+lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *olen,
+                             cudaStream_t s)
 {
-    *rounds_out = 0;
-    if (m == 0) return LASAGNA_OK;
     const int sms = num_sms();
-    auto blocks_for = [&](uint64_t k) {
-        return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(k, 256), (uint64_t)sms * 8));
-    };
+    const unsigned blocks = (unsigned)std::max<uint64_t>(
+        1, std::min<uint64_t>(ceil_div(g.cap, 256), (uint64_t)sms * 8));
     unsigned long long *in = g.pool, *out = g.pool2, *cin = g.cnt, *cout = g.cnt2;
-    uint32_t *best = g.best0, *bnext = g.best1;
-    greedy_init<<<blocks_for(m), 256, 0, s>>>(in, cin, g.best0, g.best1);
-    LSG_LAUNCHED("greedy_init");
-    uint32_t rounds = 0;
-    uint64_t live = m;
-    while (live > 0) {
-        if (rounds >= 4 && live <= (uint64_t)TAIL_MAX) {
-            greedy_tail<<<1, 1024, 0, s>>>(in, cin, g.claimed, succ, olen, l, g.accepted);
-            LSG_LAUNCHED("greedy_tail");
-            ++rounds;
-            break;
-        }
-        LSG_CUDA(cudaMemsetAsync(cout, 0, sizeof(unsigned long long), s));
-        greedy_propose<<<blocks_for(live), 256, 0, s>>>(in, cin, g.claimed, best);
+    const uint32_t e0 = g.epoch;
+    g.epoch += EPOCHS_PER_LENGTH;
+    for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
+        greedy_propose<<<blocks, 256, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, cout,
+                                              r == 0 ? g.book : nullptr);
         LSG_LAUNCHED("greedy_propose");
-        greedy_accept<<<blocks_for(live), 256, 0, s>>>(in, cin, g.claimed, best, bnext, succ, olen,
-                                                       l, out, cout, g.accepted);
+        greedy_accept<<<blocks, 256, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, succ, olen,
+                                             l, out, cout, g.book);
         LSG_LAUNCHED("greedy_accept");
-        ++rounds;
-        unsigned long long h = 0;
-        LSG_CUDA(cudaMemcpyAsync(&h, cout, sizeof(h), cudaMemcpyDeviceToHost, s));
-        LSG_CUDA(cudaStreamSynchronize(s));
-        live = h;
         std::swap(in, out);
         std::swap(cin, cout);
-        std::swap(best, bnext);
     }
-    *rounds_out = rounds;
+    greedy_finish<<<1, FINISH_THREADS, 0, s>>>(in, cin, out, cout, g.claimed, g.best,
+                                               e0 + FAST_ROUNDS, FAST_ROUNDS, succ, olen, l, g.book);
+    LSG_LAUNCHED("greedy_finish");
     return LASAGNA_OK;
 }
 

@@ -63,13 +63,14 @@ lasagna_status launch_keys_to_output(const uint64_t *keys, uint64_t m, uint32_t 
 struct GreedyBufs {
     unsigned long long *pool, *pool2; // pair lists (ping-pong)
     unsigned long long *cnt, *cnt2;   // their fills (device)
-    unsigned long long *accepted;     // running total (device)
-    uint32_t *best0, *best1;
+    unsigned long long *book;         // device: [0] accepted, [1] sum |P_l|, [2] max |P_l|, [3] max rounds
+    unsigned long long *best;         // u64 [V]: epoch-tagged proposals, zeroed once per call
     uint8_t *claimed;
     unsigned long long cap;
+    uint32_t epoch;                   // next free epoch (host side)
 };
-lasagna_status greedy_length(GreedyBufs &g, uint64_t m, uint8_t l, uint32_t *succ, uint8_t *olen,
-                             cudaStream_t s, uint32_t *rounds_out);
+lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *olen,
+                             cudaStream_t s);
 lasagna_status launch_gather_pairs(const uint64_t *order, uint64_t off, uint64_t m,
                                    const uint32_t *pa, const uint32_t *pb,
                                    unsigned long long *pool, unsigned long long *cnt,

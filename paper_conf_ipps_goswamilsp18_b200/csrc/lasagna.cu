@@ -73,11 +73,12 @@ static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Layout {
     uint32_t G;          // lengths per group
     uint64_t pool_cap;   // pair pool capacity (pairs)
-    size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best0, best1, claimed,
-        total;
+    size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, total;
 };
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
+// u64 counters after the sort tile counters
+enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_BOOK = 4, CTR64_N = 8 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -100,11 +101,10 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     l.pool = take(pool_cap * 8);
     l.pool2 = take(pool_cap * 8);
     if (greedy) {
-        l.best0 = take(g.V * 4);
-        l.best1 = take(g.V * 4);
+        l.best = take(g.V * 8);
         l.claimed = take(g.V);
     } else {
-        l.best0 = l.best1 = l.claimed = 0; // overlaps: pairs sorted in pool/pool2
+        l.best = l.claimed = 0; // overlaps: pairs sorted in pool/pool2
     }
     l.total = off;
     return l;
@@ -154,7 +154,7 @@ struct Run {
     SortCtx sctx;
     uint64_t *tab[2];
     uint32_t *hist;
-    unsigned long long *ctr64; // [0] pool count, [1] false matches, [2] accepted, [3] cnt2
+    unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
     void bind(void *workspace)
@@ -254,13 +254,14 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     return LASAGNA_OK;
 }
 
-// Join (search + verify) of length l; *m_out = pairs found (host, synchronises).
+// Join (search + verify) of length l into the pool; if m_out, synchronise and report the
+// pair count.
 static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, uint32_t l_lo,
                                     int which, uint64_t *m_out)
 {
     const Geometry &g = r.g;
     const uint32_t s = l - l_lo;
-    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, sizeof(unsigned long long), r.s));
+    LSG_CUDA(cudaMemsetAsync(r.ctr64 + CTR_POOL, 0, sizeof(unsigned long long), r.s));
     JoinArgs ja;
     ja.packed = packed;
     ja.keys = r.tab[which] + (uint64_t)s * g.N;
@@ -272,14 +273,16 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.T = g.T;
     ja.pairs = r.pool;
     ja.cap = r.lay.pool_cap;
-    ja.count = r.ctr64;
-    ja.false_matches = r.ctr64 + 1;
+    ja.count = r.ctr64 + CTR_POOL;
+    ja.false_matches = r.ctr64 + CTR_FALSE;
     lasagna_status rc = launch_join(ja, r.s);
     if (rc != LASAGNA_OK) return rc;
-    unsigned long long m = 0;
-    LSG_CUDA(cudaMemcpyAsync(&m, r.ctr64, sizeof(m), cudaMemcpyDeviceToHost, r.s));
-    LSG_CUDA(cudaStreamSynchronize(r.s));
-    *m_out = m;
+    if (m_out) {
+        unsigned long long m = 0;
+        LSG_CUDA(cudaMemcpyAsync(&m, r.ctr64 + CTR_POOL, sizeof(m), cudaMemcpyDeviceToHost, r.s));
+        LSG_CUDA(cudaStreamSynchronize(r.s));
+        *m_out = m;
+    }
     return LASAGNA_OK;
 }
 
@@ -444,13 +447,13 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     GreedyBufs gb;
     gb.pool = r.pool;
     gb.pool2 = r.pool2;
-    gb.cnt = r.ctr64;
-    gb.cnt2 = r.ctr64 + 3;
-    gb.accepted = r.ctr64 + 2;
-    gb.best0 = r.at<uint32_t>(r.lay.best0);
-    gb.best1 = r.at<uint32_t>(r.lay.best1);
+    gb.cnt = r.ctr64 + CTR_POOL;
+    gb.cnt2 = r.ctr64 + CTR_POOL2;
+    gb.book = r.ctr64 + CTR_BOOK;
+    gb.best = r.at<unsigned long long>(r.lay.best);
     gb.claimed = claimed;
     gb.cap = cap;
+    gb.epoch = 1;
 
     lasagna_stats st;
     memset(&st, 0, sizeof st);
@@ -462,12 +465,14 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     const uint64_t launches0 = launch_count();
 
     if ((rc = sort_ctx_reset(r.sctx, s)) != LASAGNA_OK) return rc;
-    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, 8 * sizeof(unsigned long long), s));
+    LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, CTR64_N * sizeof(unsigned long long), s));
     LSG_CUDA(cudaMemsetAsync(succ, 0xFF, g.V * 4, s));
     LSG_CUDA(cudaMemsetAsync(olen, 0, g.V, s));
     LSG_CUDA(cudaMemsetAsync(claimed, 0, g.V, s));
+    LSG_CUDA(cudaMemsetAsync(gb.best, 0, g.V * 8, s));
 
-    uint64_t total_pairs = 0;
+    // Everything below is stream-ordered with no host round trip: the join of length l and
+    // its greedy claim read/write counts in device memory (one synchronisation at the end).
     for (int64_t l_hi = (int64_t)L - 1; l_hi >= (int64_t)l_min; l_hi -= G) {
         const uint32_t l_lo = (uint32_t)std::max<int64_t>(l_min, l_hi - (int64_t)G + 1);
         int which = 0;
@@ -475,37 +480,33 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
             return rc;
         ++st.passes;
         for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
-            uint64_t m = 0;
             if ((rc = tm.start(PH_SEARCH)) != LASAGNA_OK) return rc;
             // no pruning: the claimed bits are not consulted, so every length's full pair
             // list is found (|P| = overlap edges / 2 is reported)
-            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, &m)) != LASAGNA_OK)
+            if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr)) != LASAGNA_OK)
                 return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
-            if (m > cap) {
-                uint64_t need = m + m / 4;
-                *workspace_bytes = layout(g, G, need, true).total;
-                set_error("length %lld produced %llu pairs > pool %llu", (long long)l,
-                          (unsigned long long)m, (unsigned long long)cap);
-                return LASAGNA_ENOSPC;
-            }
-            total_pairs += m;
-            uint32_t rounds = 0;
             ++st.search_launches;
             if ((rc = tm.start(PH_GREEDY)) != LASAGNA_OK) return rc;
-            if ((rc = greedy_length(gb, m, (uint8_t)l, succ, olen, s, &rounds)) != LASAGNA_OK)
-                return rc;
+            if ((rc = greedy_length(gb, (uint8_t)l, succ, olen, s)) != LASAGNA_OK) return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
-            st.rounds_max = std::max(st.rounds_max, rounds);
         }
     }
+    unsigned long long h[CTR64_N];
+    LSG_CUDA(cudaMemcpyAsync(h, r.ctr64, sizeof h, cudaMemcpyDeviceToHost, s));
+    LSG_CUDA(cudaStreamSynchronize(s));
+    const unsigned long long *book = h + CTR_BOOK;
+    if (book[2] > cap) {
+        const uint64_t need = book[2] + book[2] / 4;
+        *workspace_bytes = layout(g, G, need, true).total;
+        set_error("a length produced %llu pairs > pool %llu", book[2], (unsigned long long)cap);
+        return LASAGNA_ENOSPC;
+    }
     if (stats) {
-        unsigned long long h[3];
-        LSG_CUDA(cudaMemcpyAsync(h, r.ctr64, sizeof h, cudaMemcpyDeviceToHost, s));
-        LSG_CUDA(cudaStreamSynchronize(s));
-        st.n_pairs = total_pairs;
-        st.fp_false_matches = h[1];
-        st.n_greedy = h[2];
+        st.n_pairs = book[1];
+        st.n_greedy = book[0];
+        st.rounds_max = (uint32_t)book[3];
+        st.fp_false_matches = h[CTR_FALSE];
         if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
         st.kernel_launches = launch_count() - launches0;
         *stats = st;
@@ -678,7 +679,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     }
     const uint64_t V = 2 * n;
     const uint64_t c1 = std::max<uint64_t>(count, 1);
-    // keys, keys2 | pool, pool2 | status | ctrs | hist | best0, best1 | claimed
+    // keys, keys2 | pool, pool2 | status | ctrs | hist | best | claimed
     size_t off = 0;
     auto take = [&](size_t b) {
         size_t o = off;
@@ -687,8 +688,8 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     };
     const size_t o_keys = take(c1 * 8), o_keys2 = take(c1 * 8), o_pool = take(c1 * 8),
                  o_pool2 = take(c1 * 8), o_status = take(sort_status_bytes(c1, 1)),
-                 o_ctrs = take(CTR_BYTES), o_hist = take(8 * 256 * 4), o_best0 = take(V * 4 + 4),
-                 o_best1 = take(V * 4 + 4), o_claimed = take(V + 1);
+                 o_ctrs = take(CTR_BYTES), o_hist = take(8 * 256 * 4), o_best = take(V * 8 + 8),
+                 o_claimed = take(V + 1);
     if (!workspace) {
         *workspace_bytes = off;
         return LASAGNA_OK;
@@ -736,27 +737,27 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     GreedyBufs gb;
     gb.pool = reinterpret_cast<unsigned long long *>(ws + o_pool);
     gb.pool2 = reinterpret_cast<unsigned long long *>(ws + o_pool2);
-    gb.cnt = ctr64;
-    gb.cnt2 = ctr64 + 3;
-    gb.accepted = ctr64 + 2;
-    gb.best0 = reinterpret_cast<uint32_t *>(ws + o_best0);
-    gb.best1 = reinterpret_cast<uint32_t *>(ws + o_best1);
+    gb.cnt = ctr64 + CTR_POOL;
+    gb.cnt2 = ctr64 + CTR_POOL2;
+    gb.book = ctr64 + CTR_BOOK;
+    gb.best = reinterpret_cast<unsigned long long *>(ws + o_best);
     gb.claimed = claimed;
     gb.cap = c1;
+    gb.epoch = 1;
+    LSG_CUDA(cudaMemsetAsync(gb.best, 0, V * 8, s));
     uint64_t pos = 0;
-    uint32_t total_rounds = 0;
     for (int d = 0; d < 256; ++d) { // digit d = 255 - l: longest lengths first
         const uint64_t m = h[d];
         if (!m) continue;
         const uint8_t l = (uint8_t)(255 - d);
         if ((rc = launch_gather_pairs(keys[which], pos, m, pa, pb, gb.pool, gb.cnt, s)) != LASAGNA_OK)
             return rc;
-        uint32_t r = 0;
-        if ((rc = greedy_length(gb, m, l, succ, olen, s, &r)) != LASAGNA_OK) return rc;
-        total_rounds += r;
+        if ((rc = greedy_length(gb, l, succ, olen, s)) != LASAGNA_OK) return rc;
         pos += m;
     }
+    unsigned long long bk[4];
+    LSG_CUDA(cudaMemcpyAsync(bk, gb.book, sizeof bk, cudaMemcpyDeviceToHost, s));
     LSG_CUDA(cudaStreamSynchronize(s));
-    if (rounds) *rounds = total_rounds;
+    if (rounds) *rounds = (uint32_t)bk[3];
     return LASAGNA_OK;
 }
