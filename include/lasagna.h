@@ -170,6 +170,49 @@ LASAGNA_API lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, c
                                     size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
                                     uint32_t *rounds, void *stream);
 
+/* ---------------------------------------------------------------------------------------
+ * Sharded phases: the building blocks of the multi-GPU driver (one process per GPU, tables
+ * partitioned by hash range; paper_conf_ipps_goswamilsp18_b200/dist.py).  The key layout is
+ * the one lasagna_greedy_graph uses internally for a read set of n_total reads:
+ *   key = mix(F) top (63 - vbits) bits | tag << vbits | global vertex id
+ *   (tag 0 = prefix entry, 1 = suffix entry; vbits = lasagna_vertex_bits(n_total)),
+ * and the join needs the keys of one length sorted by their top lasagna_key_sort_bits(n_total)
+ * bits.  A hash-range shard is any set of keys sharing their top bits.
+ */
+LASAGNA_API uint32_t lasagna_vertex_bits(uint64_t n_total);
+LASAGNA_API uint32_t lasagna_key_sort_bits(uint64_t n_total);
+
+/* a2/a3 for the reads [read_offset, read_offset + n_local) of an n_total-read set whose packed
+ * rows start at `packed`: tab[(l - l_lo) * 4 n_local + 4i + 2o + tag] for l in [l_lo, l_hi]
+ * (at most 64 lengths), i local read, o orientation.  Asynchronous. */
+LASAGNA_API lasagna_status lasagna_table_keys(const uint64_t *packed, uint64_t n_local,
+                                              uint64_t read_offset, uint64_t n_total, uint32_t L,
+                                              uint32_t l_lo, uint32_t l_hi, uint64_t *tab,
+                                              void *stream);
+
+/* counts[s*256 + d] = number of keys of segment s (n_seg segments of seg_len keys) whose
+ * bits [shift, shift+bits) equal d (bits <= 8).  counts is zeroed by the call.  Async. */
+LASAGNA_API lasagna_status lasagna_digit_counts(const uint64_t *keys, uint64_t seg_len,
+                                                uint32_t n_seg, uint32_t shift, uint32_t bits,
+                                                uint32_t *counts, void *stream);
+
+/* a4, segmented: n_seg independent arrays of seg_len keys (contiguous), each sorted stably
+ * by bits [bit_lo, bit_hi); result in keys.  Workspace query as usual.  Async. */
+LASAGNA_API lasagna_status lasagna_sort_segments(uint64_t *keys, uint64_t *scratch,
+                                                 uint64_t seg_len, uint32_t n_seg, uint32_t bit_lo,
+                                                 uint32_t bit_hi, void *workspace,
+                                                 size_t *workspace_bytes, void *stream);
+
+/* a5 on one length l: `keys` (count entries, any hash-range shard of length l's table, sorted
+ * by the top lasagna_key_sort_bits(n_total) bits); packed_all = the packed rows of ALL n_total
+ * reads (verification).  Appends the verified read-end pairs (a << 32) | b, a < b, to pairs
+ * (at most capacity are stored); counters (device u64[2]) accumulate [0] pairs found (may
+ * exceed capacity: overflow) and [1] rejected fingerprint matches.  Async. */
+LASAGNA_API lasagna_status lasagna_join(const uint64_t *keys, uint64_t count,
+                                        const uint64_t *packed_all, uint64_t n_total, uint32_t L,
+                                        uint32_t l, uint64_t *pairs, uint64_t capacity,
+                                        uint64_t *counters, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -128,9 +128,11 @@ table_kernel(TableArgs a)
 {
     extern __shared__ uint32_t shist[]; // [G][256]
     const uint32_t G = a.l_hi - a.l_lo + 1;
-    for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x) shist[t] = 0;
+    const bool with_hist = a.hist != nullptr;
+    if (with_hist)
+        for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x) shist[t] = 0;
     __syncthreads();
-    const uint64_t N = 4 * a.n; // 2V entries per length
+    const uint64_t N = 4 * a.n; // 2V entries per length (of this read range)
     const uint64_t keep = ~((2ull << a.vbits) - 1);
     const uint64_t tagS = 1ull << a.vbits;
     const uint32_t dmask = (1u << a.d_bits) - 1;
@@ -142,7 +144,7 @@ table_kernel(TableArgs a)
         roll_read<W>(x, y, a.l_hi, [&](uint32_t l, const FpStreams &st) {
             if (l < a.l_lo) return;
             const uint32_t s = l - a.l_lo;
-            const uint64_t v0 = 2 * i, v1 = 2 * i + 1;
+            const uint64_t v0 = 2 * (a.read_offset + i), v1 = v0 + 1; // global vertex ids
             const uint64_t p0 = (mix(exact61(st.P0)) & keep) | v0;
             const uint64_t s0 = (mix(exact61(st.S0)) & keep) | tagS | v0;
             const uint64_t p1 = (mix(exact61(st.P1)) & keep) | v1;
@@ -150,23 +152,26 @@ table_kernel(TableArgs a)
             ulonglong2 *dst = reinterpret_cast<ulonglong2 *>(a.tab + (uint64_t)s * N + 4 * i);
             dst[0] = make_ulonglong2(p0, s0);
             dst[1] = make_ulonglong2(p1, s1);
-            uint32_t *h = shist + s * 256;
-            atomicAdd(&h[(uint32_t)((p0 >> a.d_shift) & dmask)], 1u);
-            atomicAdd(&h[(uint32_t)((s0 >> a.d_shift) & dmask)], 1u);
-            atomicAdd(&h[(uint32_t)((p1 >> a.d_shift) & dmask)], 1u);
-            atomicAdd(&h[(uint32_t)((s1 >> a.d_shift) & dmask)], 1u);
+            if (with_hist) {
+                uint32_t *h = shist + s * 256;
+                atomicAdd(&h[(uint32_t)((p0 >> a.d_shift) & dmask)], 1u);
+                atomicAdd(&h[(uint32_t)((s0 >> a.d_shift) & dmask)], 1u);
+                atomicAdd(&h[(uint32_t)((p1 >> a.d_shift) & dmask)], 1u);
+                atomicAdd(&h[(uint32_t)((s1 >> a.d_shift) & dmask)], 1u);
+            }
         });
     }
     __syncthreads();
-    for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x)
-        if (shist[t]) atomicAdd(&a.hist[t], shist[t]);
+    if (with_hist)
+        for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x)
+            if (shist[t]) atomicAdd(&a.hist[t], shist[t]);
 }
 
 lasagna_status launch_table(const TableArgs &args, cudaStream_t s)
 {
     if (args.n == 0) return LASAGNA_OK;
     const uint32_t G = args.l_hi - args.l_lo + 1;
-    const size_t smem = (size_t)G * 256 * sizeof(uint32_t);
+    const size_t smem = args.hist ? (size_t)G * 256 * sizeof(uint32_t) : 0;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
         if (smem > 48 * 1024)

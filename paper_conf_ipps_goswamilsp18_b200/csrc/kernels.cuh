@@ -16,13 +16,14 @@ lasagna_status launch_fp_values(const uint64_t *packed, uint64_t n, uint32_t L, 
 
 struct TableArgs {
     const uint64_t *packed;
-    uint64_t n;
+    uint64_t n;               // reads in this range
+    uint64_t read_offset;     // global id of the first read (vertex ids are global)
     uint32_t L, stride;
     uint32_t l_lo, l_hi;      // group of lengths (segment s = l - l_lo)
     uint32_t vbits;           // b_v: vertex-id bits at the bottom of a key
     uint32_t d_shift, d_bits; // first LSD digit (histogram produced on the fly)
     uint64_t *tab;            // [G][2V]: entry 2v = prefix key of v, 2v+1 = suffix key of v
-    uint32_t *hist;           // [G][256]
+    uint32_t *hist;           // [G][256] first-digit histogram, or null
 };
 lasagna_status launch_table(const TableArgs &a, cudaStream_t s);
 
@@ -40,6 +41,8 @@ void digit_plan(uint32_t lo, uint32_t hi, uint32_t *P, uint32_t *shifts, uint32_
 lasagna_status sort_segments(uint64_t *bufs[2], uint64_t seg_len, uint32_t n_seg, uint32_t lo,
                              uint32_t hi, uint32_t *hist, bool hist0_ready, SortCtx &ctx,
                              cudaStream_t s, int *which);
+lasagna_status launch_hist(const uint64_t *keys, uint64_t seg_len, uint32_t n_seg, uint32_t shift,
+                           uint32_t bits, uint32_t *hist, cudaStream_t s);
 
 // ---- a5 (search.cu)
 struct JoinArgs {

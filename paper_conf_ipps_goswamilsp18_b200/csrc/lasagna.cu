@@ -232,6 +232,7 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     TableArgs ta;
     ta.packed = packed;
     ta.n = g.n;
+    ta.read_offset = 0;
     ta.L = g.L;
     ta.stride = stride_for(g.L);
     ta.l_lo = l_lo;
@@ -618,47 +619,8 @@ lasagna_status lasagna_sort_u64(uint64_t *keys, uint64_t *scratch, uint64_t coun
                                 uint32_t bit_lo, uint32_t bit_hi, void *workspace,
                                 size_t *workspace_bytes, void *stream)
 {
-    g_err[0] = 0;
-    if (!workspace_bytes || bit_lo >= bit_hi || bit_hi > 64) {
-        set_error("bad bit range or NULL workspace_bytes");
-        return LASAGNA_EINVAL;
-    }
-    const size_t need = align256(sort_status_bytes(count, 1)) + align256(CTR_BYTES) +
-                        align256(8 * 256 * 4);
-    if (!workspace) {
-        *workspace_bytes = need;
-        return LASAGNA_OK;
-    }
-    if (*workspace_bytes < need) {
-        *workspace_bytes = need;
-        set_error("workspace too small");
-        return LASAGNA_ENOSPC;
-    }
-    if (count == 0) return LASAGNA_OK;
-    if (!keys || !scratch || !aligned(keys, 8) || !aligned(scratch, 8) || !aligned(workspace, 256)) {
-        set_error("NULL or misaligned pointer");
-        return LASAGNA_EINVAL;
-    }
-    if (count > 0xFFFFFFFFull) {
-        set_error("count must be < 2^32");
-        return LASAGNA_ERANGE;
-    }
-    cudaStream_t s = (cudaStream_t)stream;
-    char *ws = (char *)workspace;
-    SortCtx c;
-    c.status = reinterpret_cast<unsigned long long *>(ws);
-    c.status_bytes = sort_status_bytes(count, 1);
-    c.tile_ctrs = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes));
-    uint32_t *hist = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes) + align256(CTR_BYTES));
-    lasagna_status rc = sort_ctx_reset(c, s);
-    if (rc != LASAGNA_OK) return rc;
-    uint64_t *bufs[2] = {keys, scratch};
-    int which = 0;
-    rc = sort_segments(bufs, count, 1, bit_lo, bit_hi, hist, false, c, s, &which);
-    if (rc != LASAGNA_OK) return rc;
-    if (which == 1)
-        LSG_CUDA(cudaMemcpyAsync(keys, scratch, count * 8, cudaMemcpyDeviceToDevice, s));
-    return LASAGNA_OK;
+    return lasagna_sort_segments(keys, scratch, count, 1, bit_lo, bit_hi, workspace,
+                                 workspace_bytes, stream);
 }
 
 } // extern "C"
@@ -761,3 +723,137 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     if (rounds) *rounds = (uint32_t)bk[3];
     return LASAGNA_OK;
 }
+
+// ==================================================================== sharded phases
+// Building blocks of the multi-GPU driver (paper_conf_ipps_goswamilsp18_b200/dist.py): the
+// same kernels as lasagna_greedy_graph, with global vertex ids and caller-managed buffers.
+extern "C" {
+
+uint32_t lasagna_vertex_bits(uint64_t n_total) { return geometry(n_total, 2, 1).vbits; }
+
+uint32_t lasagna_key_sort_bits(uint64_t n_total) { return geometry(n_total, 2, 1).T; }
+
+lasagna_status lasagna_table_keys(const uint64_t *packed, uint64_t n_local, uint64_t read_offset,
+                                  uint64_t n_total, uint32_t L, uint32_t l_lo, uint32_t l_hi,
+                                  uint64_t *tab, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n_total, L, l_lo);
+    if (rc != LASAGNA_OK) return rc;
+    if (l_hi < l_lo || l_hi >= L || l_hi - l_lo + 1 > 64 || read_offset + n_local > n_total) {
+        set_error("bad length group [%u, %u] or read range", l_lo, l_hi);
+        return LASAGNA_EINVAL;
+    }
+    if (n_local == 0) return LASAGNA_OK;
+    if (!packed || !tab || !aligned(packed, 16) || !aligned(tab, 16)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    Geometry g = geometry(n_total, L, l_lo);
+    TableArgs ta;
+    ta.packed = packed;
+    ta.n = n_local;
+    ta.read_offset = read_offset;
+    ta.L = L;
+    ta.stride = stride_for(L);
+    ta.l_lo = l_lo;
+    ta.l_hi = l_hi;
+    ta.vbits = g.vbits;
+    ta.d_shift = 0;
+    ta.d_bits = 1;
+    ta.tab = tab;
+    ta.hist = nullptr;
+    return launch_table(ta, (cudaStream_t)stream);
+}
+
+lasagna_status lasagna_digit_counts(const uint64_t *keys, uint64_t seg_len, uint32_t n_seg,
+                                    uint32_t shift, uint32_t bits, uint32_t *counts, void *stream)
+{
+    g_err[0] = 0;
+    if (bits < 1 || bits > 8 || shift + bits > 64 || !counts || (seg_len && !keys)) {
+        set_error("bad digit or NULL pointer");
+        return LASAGNA_EINVAL;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    LSG_CUDA(cudaMemsetAsync(counts, 0, (size_t)n_seg * 256 * 4, s));
+    return launch_hist(keys, seg_len, n_seg, shift, bits, counts, s);
+}
+
+lasagna_status lasagna_sort_segments(uint64_t *keys, uint64_t *scratch, uint64_t seg_len,
+                                     uint32_t n_seg, uint32_t bit_lo, uint32_t bit_hi,
+                                     void *workspace, size_t *workspace_bytes, void *stream)
+{
+    g_err[0] = 0;
+    if (!workspace_bytes || bit_lo >= bit_hi || bit_hi > 64 || n_seg == 0) {
+        set_error("bad bit range, segment count or NULL workspace_bytes");
+        return LASAGNA_EINVAL;
+    }
+    const size_t need = align256(sort_status_bytes(seg_len, n_seg)) + align256(CTR_BYTES) +
+                        align256((size_t)8 * n_seg * 256 * 4);
+    if (!workspace) {
+        *workspace_bytes = need;
+        return LASAGNA_OK;
+    }
+    if (*workspace_bytes < need) {
+        *workspace_bytes = need;
+        set_error("workspace too small");
+        return LASAGNA_ENOSPC;
+    }
+    if (seg_len == 0) return LASAGNA_OK;
+    if (!keys || !scratch || !aligned(keys, 8) || !aligned(scratch, 8) || !aligned(workspace, 256)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    if (seg_len > 0xFFFFFFFFull) {
+        set_error("segment length must be < 2^32");
+        return LASAGNA_ERANGE;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    char *ws = (char *)workspace;
+    SortCtx c;
+    c.status = reinterpret_cast<unsigned long long *>(ws);
+    c.status_bytes = sort_status_bytes(seg_len, n_seg);
+    c.tile_ctrs = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes));
+    uint32_t *hist = reinterpret_cast<uint32_t *>(ws + align256(c.status_bytes) + align256(CTR_BYTES));
+    lasagna_status rc = sort_ctx_reset(c, s);
+    if (rc != LASAGNA_OK) return rc;
+    uint64_t *bufs[2] = {keys, scratch};
+    int which = 0;
+    rc = sort_segments(bufs, seg_len, n_seg, bit_lo, bit_hi, hist, false, c, s, &which);
+    if (rc != LASAGNA_OK) return rc;
+    if (which == 1)
+        LSG_CUDA(cudaMemcpyAsync(keys, scratch, seg_len * n_seg * 8, cudaMemcpyDeviceToDevice, s));
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_join(const uint64_t *keys, uint64_t count, const uint64_t *packed_all,
+                            uint64_t n_total, uint32_t L, uint32_t l, uint64_t *pairs,
+                            uint64_t capacity, uint64_t *counters, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = check_shape(n_total, L, l);
+    if (rc != LASAGNA_OK) return rc;
+    if (!counters || (count && (!keys || !packed_all)) || (capacity && !pairs) ||
+        !aligned(counters, 8) || (packed_all && !aligned(packed_all, 16))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    if (count == 0) return LASAGNA_OK;
+    Geometry g = geometry(n_total, L, l);
+    JoinArgs ja;
+    ja.packed = packed_all;
+    ja.keys = keys;
+    ja.N = count;
+    ja.L = L;
+    ja.stride = stride_for(L);
+    ja.l = l;
+    ja.vbits = g.vbits;
+    ja.T = g.T;
+    ja.pairs = reinterpret_cast<unsigned long long *>(pairs);
+    ja.cap = capacity;
+    ja.count = reinterpret_cast<unsigned long long *>(counters);
+    ja.false_matches = reinterpret_cast<unsigned long long *>(counters) + 1;
+    return launch_join(ja, (cudaStream_t)stream);
+}
+
+} // extern "C"

@@ -137,13 +137,16 @@ join_kernel(JoinArgs a)
     const uint32_t kshift = a.vbits + 1; // key bits above tag + vid
     const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint64_t *A = a.keys;
-    const uint64_t B = 1ull << a.T;
     const int warp = threadIdx.x >> 5;
 
     if (threadIdx.x == 0) bcount = 0, vdone = 0;
+    // CTA c owns the buckets that start in [c N/grid, (c+1) N/grid): its range starts at the
+    // first entry of the bucket holding entry c N/grid (balanced by entries, whatever the
+    // key distribution — e.g. one hash range of a multi-GPU shard)
     if (warp < 2) {
-        const uint64_t b = (B * (blockIdx.x + warp)) / gridDim.x;
-        const uint64_t r = (b >= B) ? N : warp_lower_bound(A, 0, N, bshift, b);
+        const uint64_t q = (N * (blockIdx.x + warp)) / gridDim.x;
+        uint64_t r = N;
+        if (q < N) r = warp_lower_bound(A, 0, q + 1, bshift, A[q] >> bshift);
         if ((threadIdx.x & 31) == 0) s_r[warp] = r;
     }
     __syncthreads();
@@ -254,7 +257,6 @@ lasagna_status launch_join(const JoinArgs &args, cudaStream_t s)
         // persistent grid, but never more CTAs than ~one window of entries each
         uint64_t blocks = std::min<uint64_t>((uint64_t)num_sms() * per_sm,
                                              std::max<uint64_t>(1, args.N / JOIN_CHUNK));
-        blocks = std::min<uint64_t>(blocks, 1ull << args.T);
         join_kernel<W><<<(unsigned)blocks, JOIN_THREADS, smem, s>>>(args);
         LSG_LAUNCHED("join_kernel");
         return LASAGNA_OK;

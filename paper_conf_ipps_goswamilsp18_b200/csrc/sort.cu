@@ -229,6 +229,16 @@ __global__ void hist_kernel(const uint64_t *__restrict__ in, uint64_t seg_len, u
         if (h[t]) atomicAdd(&hist[(uint64_t)seg * 256 + t], h[t]);
 }
 
+lasagna_status launch_hist(const uint64_t *keys, uint64_t seg_len, uint32_t n_seg, uint32_t shift,
+                           uint32_t bits, uint32_t *hist, cudaStream_t s)
+{
+    if (seg_len == 0 || n_seg == 0) return LASAGNA_OK;
+    dim3 grid((unsigned)std::min<uint64_t>(ceil_div(seg_len, 256 * 16), 1024), n_seg);
+    hist_kernel<<<grid, 256, 0, s>>>(keys, seg_len, shift, bits, hist);
+    LSG_LAUNCHED("hist_kernel");
+    return LASAGNA_OK;
+}
+
 // ---------------------------------------------------------------- host side
 size_t sort_status_bytes(uint64_t seg_len, uint32_t n_seg)
 {

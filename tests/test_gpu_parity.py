@@ -316,3 +316,43 @@ def test_greedy_pairs_adversarial_chain(lz, k):
     succ, olen, rounds = lz.greedy_pairs(n, pl, pa, pb)
     assert _np(succ, np.uint32).tolist() == esucc
     assert _np(olen, np.uint8).tolist() == eolen
+
+
+@gpu
+@pytest.mark.parametrize("reads,l_min", [(["AC"], 1), (["ACGTAC", "GTACGT"], 1), (["AAAA", "AAAA", "TTTT"], 1),
+                                         (["ACGT" * 8 + "A"], 16)])
+def test_degenerate_shapes(lz, reads, l_min):
+    import torch
+    arr = to_array(reads)
+    n, L = arr.shape
+    packed = lz.load_reads(torch.from_numpy(arr).cuda())
+    r = lz.greedy_graph(packed, n, L, l_min)
+    esucc, eolen, m, _ = oracle.greedy_graph(arr, l_min)
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    pl, pa, pb = lz.overlaps(packed, n, L, l_min)
+    epl, epa, epb = oracle.overlaps(arr, l_min)
+    assert np.array_equal(_np(pa, np.uint32), epa) and np.array_equal(_np(pb, np.uint32), epb)
+
+
+@gpu
+def test_empty_read_set(lz):
+    import torch
+    packed = torch.empty((0, 4), dtype=torch.int64, device="cuda")
+    r = lz.greedy_graph(packed, 0, 100, 63)
+    assert r.succ.numel() == 0 and r.stats["n_pairs"] == 0
+    pl, pa, pb = lz.overlaps(packed, 0, 100, 63)
+    assert pl.numel() == 0
+
+
+@gpu
+def test_planner_and_small_workspace(lz):
+    """a8: the planner shrinks the length group to the budget; a workspace below one length
+    is ENOSPC with the needed size reported."""
+    n, L, l_min = 20_000, 100, 63
+    lp_all, ws_all = lz.plan(n, L, l_min, 1 << 40)
+    assert lp_all == L - l_min
+    lp_small, ws_small = lz.plan(n, L, l_min, ws_all // 4)
+    assert 1 <= lp_small < lp_all and ws_small <= ws_all // 4
+    lp0, need = lz.plan(n, L, l_min, 1 << 10)
+    assert lp0 == 0 and need > (1 << 10)
