@@ -26,7 +26,6 @@ constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
 constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
 constexpr int JOIN_SLOTS = 8192;   // hash chain heads (u32); chains through next[] (u16)
 constexpr int JOIN_BUF = 1024;     // staged output pairs
-constexpr uint32_t SLOT_EMPTY = 0xFFFFFFFFu;
 
 // Candidates are staged in shared memory and verified in a separate, fully parallel pass
 // (a fingerprint match is rare: verifying it inline would run the long verify path with one
@@ -154,20 +153,36 @@ join_kernel(JoinArgs a)
     Stager em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
 
+    // hash slots hold (window epoch << 16) | entry index: a slot written in an earlier window
+    // reads as empty, so the table is never cleared
+    for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+    uint32_t epoch = 0;
     uint64_t t0 = r0;
     while (t0 < r1) {
+        if (++epoch == 0x10000u) { // 16-bit tags wrapped: clear once and restart the epochs
+            __syncthreads();
+            for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+            epoch = 1;
+        }
         const uint32_t cnt = (uint32_t)min64(JOIN_CAP, r1 - t0);
-        if (threadIdx.x == 0) s_cut = 0;
         for (uint32_t k = threadIdx.x; k < cnt; k += JOIN_THREADS) ent[k] = A[t0 + k];
-        for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = SLOT_EMPTY;
         __syncthreads();
         uint64_t t1;
         if (t0 + cnt == r1) {
             t1 = r1;
         } else {
-            // last bucket start inside the window: the window is cut there
-            for (uint32_t k = 1 + threadIdx.x; k < cnt; k += JOIN_THREADS)
-                if ((ent[k] >> bshift) != (ent[k - 1] >> bshift)) atomicMax(&s_cut, (unsigned long long)k);
+            // the window is cut at the start of its last bucket (binary search: the staged
+            // entries are sorted by bucket)
+            if (threadIdx.x == 0) {
+                const uint64_t bl = ent[cnt - 1] >> bshift;
+                uint32_t lo = 0, hi = cnt - 1;
+                while (lo < hi) {
+                    const uint32_t mid = (lo + hi) >> 1;
+                    if ((ent[mid] >> bshift) < bl) lo = mid + 1;
+                    else hi = mid;
+                }
+                s_cut = lo;
+            }
             __syncthreads();
             t1 = t0 + s_cut;
         }
@@ -200,22 +215,24 @@ join_kernel(JoinArgs a)
             // ---- hash the prefix entries of [t0, t1) (chained: one atomicExch per insert),
             // then probe with the suffix entries
             const uint32_t m = (uint32_t)(t1 - t0);
+            const uint32_t tag = (epoch & 0xFFFFu) << 16;
             for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
                 const uint64_t e = ent[k];
                 if ((e >> a.vbits) & 1) continue;
                 const uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-                next[k] = (unsigned short)atomicExch(&slot[h], k);
+                const uint32_t old = atomicExch(&slot[h], tag | k);
+                next[k] = (old >> 16) == (tag >> 16) ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
             }
             __syncthreads();
             for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
                 const uint64_t e = ent[k];
                 if (!((e >> a.vbits) & 1)) continue;
-                uint32_t sl = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
-                while (sl != SLOT_EMPTY) {
+                const uint32_t sv = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
+                uint32_t sl = (sv >> 16) == (tag >> 16) ? (sv & 0xFFFFu) : 0xFFFFu;
+                while (sl != 0xFFFFu) {
                     const uint64_t p = ent[sl];
                     if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
                     sl = next[sl];
-                    if (sl == 0xFFFFu) break;
                 }
             }
         }

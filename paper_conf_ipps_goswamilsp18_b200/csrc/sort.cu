@@ -12,6 +12,8 @@
 //
 // Segmented: n_seg independent arrays of seg_len keys each (one per overlap length) are
 // sorted by one launch.
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 namespace lsg {
@@ -79,6 +81,8 @@ __device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t *wsum /* [8] sh
     return x - v + add;
 }
 
+// RANK = 0: bit-sliced multi-split (8 ballots); RANK = 1: match.any
+template <int RANK>
 __global__ void __launch_bounds__(SORT_THREADS, 2)
 onesweep_kernel(SortPassArgs a)
 {
@@ -179,14 +183,19 @@ onesweep_kernel(SortPassArgs a)
         uint32_t d = valid ? (uint32_t)((key[i] >> a.shift) & dmask) : 0u;
         // peers with the same digit: bit-sliced multi-split with 8 ballots (cheaper than
         // match.any on this part), restricted to valid lanes
-        uint32_t peers = __ballot_sync(0xffffffffu, valid);
+        uint32_t peers;
+        if constexpr (RANK == 0) {
+            peers = __ballot_sync(0xffffffffu, valid);
 #pragma unroll
-        for (int bb = 0; bb < 8; ++bb) {
-            const bool bit = (d >> bb) & 1u;
-            const uint32_t m = __ballot_sync(0xffffffffu, bit);
-            peers &= bit ? m : ~m;
+            for (int bb = 0; bb < 8; ++bb) {
+                const bool bit = (d >> bb) & 1u;
+                const uint32_t m = __ballot_sync(0xffffffffu, bit);
+                peers &= bit ? m : ~m;
+            }
+            if (!valid) peers = 1u << lane;
+        } else {
+            peers = __match_any_sync(0xffffffffu, valid ? d : 256u + lane);
         }
-        if (!valid) peers = 1u << lane;
         int leader = 31 - __clz((int)peers);
         uint32_t lower = __popc(peers & lanemask_lt());
         uint32_t base_pos = 0;
@@ -290,8 +299,12 @@ lasagna_status sort_segments(uint64_t *bufs[2], uint64_t seg_len, uint32_t n_seg
         LSG_LAUNCHED("hist_kernel");
     }
     const size_t smem = (size_t)SORT_TILE * 8 + (size_t)SORT_WARPS * 256 * 4;
-    LSG_CUDA(cudaFuncSetAttribute(onesweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)smem));
+    static const int rank_mode = [] {
+        const char *e = getenv("LASAGNA_SORT_RANK");
+        return (e && e[0] == 'm') ? 1 : 0;
+    }();
+    auto kern = rank_mode ? onesweep_kernel<1> : onesweep_kernel<0>;
+    LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t tps = (uint32_t)ceil_div(seg_len, SORT_TILE);
     if (sort_status_bytes(seg_len, n_seg) > ctx.status_bytes) {
         set_error("sort status buffer too small");
@@ -320,7 +333,7 @@ lasagna_status sort_segments(uint64_t *bufs[2], uint64_t seg_len, uint32_t n_seg
         a.tile_ctr = ctx.tile_ctrs + ctx.epoch;
         a.epoch = ctx.epoch;
         uint64_t grid = (uint64_t)tps * n_seg;
-        onesweep_kernel<<<(unsigned)grid, SORT_THREADS, smem, s>>>(a);
+        kern<<<(unsigned)grid, SORT_THREADS, smem, s>>>(a);
         LSG_LAUNCHED("onesweep_kernel");
         cur ^= 1;
     }
