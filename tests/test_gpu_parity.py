@@ -352,7 +352,8 @@ def test_planner_and_small_workspace(lz):
     n, L, l_min = 20_000, 100, 63
     lp_all, ws_all = lz.plan(n, L, l_min, 1 << 40)
     assert lp_all == L - l_min
-    lp_small, ws_small = lz.plan(n, L, l_min, ws_all // 4)
-    assert 1 <= lp_small < lp_all and ws_small <= ws_all // 4
     lp0, need = lz.plan(n, L, l_min, 1 << 10)
     assert lp0 == 0 and need > (1 << 10)
+    budget = (need + ws_all) // 2
+    lp_small, ws_small = lz.plan(n, L, l_min, budget)
+    assert 1 <= lp_small < lp_all and ws_small <= budget
