@@ -62,6 +62,37 @@ lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsign
 lasagna_status launch_keys_to_output(const uint64_t *keys, uint64_t m, uint32_t vbits, uint8_t l,
                                      uint32_t *pa, uint32_t *pb, uint8_t *pl, cudaStream_t s);
 
+// ---- bucketed a3/a4/a5 (partition.cu)
+struct ScatterArgs {
+    const uint64_t *packed;
+    uint64_t n, read_offset;
+    uint32_t L, stride, l_lo, l_hi, vbits;
+    uint64_t *out;      // [G][256][cap] level-1 regions (top 8 key bits)
+    uint32_t *fill;     // [G][256]
+    uint64_t cap;
+    uint32_t *overflow;
+};
+lasagna_status launch_scatter_table(const ScatterArgs &a, cudaStream_t s);
+struct RefineArgs {
+    const uint64_t *in;
+    const uint32_t *fill_in;
+    uint64_t cap_in;
+    uint32_t dshift;    // this level's digit: bits [dshift, dshift + 8)
+    uint64_t *out;      // [regions][256][cap_out]
+    uint32_t *fill_out; // [regions][256]
+    uint64_t cap_out;
+    uint32_t *overflow;
+};
+lasagna_status launch_refine(const RefineArgs &a, uint64_t n_regions, cudaStream_t s);
+struct BucketJoinArgs {
+    JoinArgs j;               // packed, L, stride, l, vbits, pairs, cap, count, false_matches
+    const uint64_t *buckets;  // [n_buckets][bucket_cap]
+    const uint32_t *fills;    // [n_buckets]
+    uint64_t bucket_cap, n_buckets;
+    uint32_t *overflow;
+};
+lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s);
+
 // ---- a6/a7 (greedy.cu)
 struct GreedyBufs {
     unsigned long long *pool, *pool2; // pair lists (ping-pong)

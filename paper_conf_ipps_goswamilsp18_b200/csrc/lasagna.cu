@@ -6,6 +6,7 @@
 #include <vector>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "kernels.cuh"
@@ -42,7 +43,21 @@ lasagna_status cuda_status(cudaError_t e, const char *what)
 struct Geometry {
     uint64_t n, V, N;
     uint32_t L, l_min, n_len, vbits, T;
+    // bucketed path (partition.cu): P = T/8 MSD levels, region capacities with slack
+    uint32_t P;
+    uint64_t cap1, cap2;
 };
+
+// capacity of a region expecting `mean` keys: mean + 8 sigma + 32 (multinomial occupancy;
+// a region that still overflows makes the call fall back to the exact LSD path)
+static uint64_t region_cap(double mean)
+{
+    // LASAGNA_TEST_TIGHT_REGIONS=1 (tests only): half-size regions force the overflow fallback
+    static const bool tight = getenv("LASAGNA_TEST_TIGHT_REGIONS") != nullptr;
+    if (tight) return ((uint64_t)(mean / 2) + 2) & ~1ull;
+    uint64_t c = (uint64_t)std::ceil(mean + 8.0 * std::sqrt(mean) + 32.0);
+    return (c + 1) & ~1ull;
+}
 
 static uint32_t ceil_log2(uint64_t x)
 {
@@ -65,6 +80,9 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     int P = (int)std::ceil((lg - 11.5) / 8.0);
     P = std::max(1, std::min(P, 4));
     g.T = std::min<uint32_t>(8u * (uint32_t)P, 63u - g.vbits);
+    g.P = g.T / 8;
+    g.cap1 = region_cap((double)g.N / 256.0);
+    g.cap2 = region_cap((double)g.N / 65536.0);
     return g;
 }
 
@@ -73,12 +91,13 @@ static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Layout {
     uint32_t G;          // lengths per group
     uint64_t pool_cap;   // pair pool capacity (pairs)
-    size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, total;
+    size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, fill1,
+        fill2, total;
 };
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
-enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_BOOK = 4, CTR64_N = 8 };
+enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR64_N = 8 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -91,9 +110,15 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
         off += align256(bytes);
         return o;
     };
-    const size_t tabb = (size_t)G * g.N * 8;
-    l.tabA = take(tabb);
-    l.tabB = take(tabb);
+    // tabA/tabB: the exact path's LSD ping-pong buffers, or the bucketed path's level-1 and
+    // level-2 regions (with slack)
+    const size_t exact_b = (size_t)G * g.N * 8;
+    const size_t lvl1_b = (size_t)G * 256 * g.cap1 * 8;
+    const size_t lvl2_b = g.P >= 2 ? (size_t)G * 65536 * g.cap2 * 8 : 0;
+    l.tabA = take(std::max(exact_b, lvl1_b));
+    l.tabB = take(std::max(exact_b, lvl2_b));
+    l.fill1 = take((size_t)G * 256 * 4);
+    l.fill2 = take(g.P >= 2 ? (size_t)G * 65536 * 4 : 4);
     l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
     l.status = take(l.status_bytes);
     l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
@@ -108,6 +133,17 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     }
     l.total = off;
     return l;
+}
+
+// The bucketed path (partition.cu) serves T <= 16 (P <= 2); LASAGNA_PATH=exact forces the
+// exact LSD-sort path (also the fallback when a slack region overflows).
+static bool use_bucketed(const Geometry &g)
+{
+    static const bool force_exact = [] {
+        const char *e = getenv("LASAGNA_PATH");
+        return e && e[0] == 'e';
+    }();
+    return !force_exact && g.P >= 1 && g.P <= 2;
 }
 
 static uint64_t default_pool_cap(const Geometry &g)
@@ -154,6 +190,8 @@ struct Run {
     SortCtx sctx;
     uint64_t *tab[2];
     uint32_t *hist;
+    bool bucketed;              // partition.cu path (else exact LSD sort + contiguous join)
+    uint32_t *fill1, *fill2;
     unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
@@ -163,6 +201,8 @@ struct Run {
         tab[0] = at<uint64_t>(lay.tabA);
         tab[1] = at<uint64_t>(lay.tabB);
         hist = at<uint32_t>(lay.hist);
+        fill1 = at<uint32_t>(lay.fill1);
+        fill2 = at<uint32_t>(lay.fill2);
         sctx.status = at<unsigned long long>(lay.status);
         sctx.status_bytes = lay.status_bytes;
         sctx.tile_ctrs = at<uint32_t>(lay.ctrs);
@@ -221,9 +261,55 @@ struct PhaseTimer {
 };
 
 // Build + sort the key tables of lengths [l_lo, l_hi]; returns which tab buffer is sorted.
+static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint32_t l_lo,
+                                           uint32_t l_hi, PhaseTimer &tm, lasagna_stats *st)
+{
+    const Geometry &g = r.g;
+    const uint32_t G = l_hi - l_lo + 1;
+    unsigned int *ovf = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
+    LSG_CUDA(cudaMemsetAsync(r.fill1, 0, (size_t)G * 256 * 4, r.s));
+    ScatterArgs sa;
+    sa.packed = packed;
+    sa.n = g.n;
+    sa.read_offset = 0;
+    sa.L = g.L;
+    sa.stride = stride_for(g.L);
+    sa.l_lo = l_lo;
+    sa.l_hi = l_hi;
+    sa.vbits = g.vbits;
+    sa.out = r.tab[0];
+    sa.fill = r.fill1;
+    sa.cap = g.cap1;
+    sa.overflow = ovf;
+    lasagna_status rc;
+    if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
+    if ((rc = launch_scatter_table(sa, r.s)) != LASAGNA_OK) return rc;
+    if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+    if (g.P >= 2) {
+        RefineArgs ra;
+        ra.in = r.tab[0];
+        ra.fill_in = r.fill1;
+        ra.cap_in = g.cap1;
+        ra.dshift = 48;
+        ra.out = r.tab[1];
+        ra.fill_out = r.fill2;
+        ra.cap_out = g.cap2;
+        ra.overflow = ovf;
+        if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
+        if ((rc = launch_refine(ra, (uint64_t)G * 256, r.s)) != LASAGNA_OK) return rc;
+        if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+        if (st) st->sort_launches += 1;
+    }
+    return LASAGNA_OK;
+}
+
 static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo, uint32_t l_hi,
                                   int *which, PhaseTimer &tm, lasagna_stats *st)
 {
+    if (r.bucketed) {
+        *which = 0;
+        return build_group_bucketed(r, packed, l_lo, l_hi, tm, st);
+    }
     const Geometry &g = r.g;
     const uint32_t G = l_hi - l_lo + 1;
     uint32_t P, shifts[8], bits[8];
@@ -276,7 +362,26 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.cap = r.lay.pool_cap;
     ja.count = r.ctr64 + CTR_POOL;
     ja.false_matches = r.ctr64 + CTR_FALSE;
-    lasagna_status rc = launch_join(ja, r.s);
+    lasagna_status rc;
+    if (r.bucketed) {
+        BucketJoinArgs bj;
+        bj.j = ja;
+        bj.overflow = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
+        if (g.P >= 2) {
+            bj.buckets = r.tab[1] + (uint64_t)s * 65536 * g.cap2;
+            bj.fills = r.fill2 + (uint64_t)s * 65536;
+            bj.bucket_cap = g.cap2;
+            bj.n_buckets = 65536;
+        } else {
+            bj.buckets = r.tab[0] + (uint64_t)s * 256 * g.cap1;
+            bj.fills = r.fill1 + (uint64_t)s * 256;
+            bj.bucket_cap = g.cap1;
+            bj.n_buckets = 256;
+        }
+        rc = launch_bucket_join(bj, r.s);
+    } else {
+        rc = launch_join(ja, r.s);
+    }
     if (rc != LASAGNA_OK) return rc;
     if (m_out) {
         unsigned long long m = 0;
@@ -456,6 +561,9 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     gb.cap = cap;
     gb.epoch = 1;
 
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    r.bucketed = attempt == 0 && use_bucketed(g);
+    gb.epoch = 1;
     lasagna_stats st;
     memset(&st, 0, sizeof st);
     st.lengths_per_pass = G;
@@ -496,6 +604,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     unsigned long long h[CTR64_N];
     LSG_CUDA(cudaMemcpyAsync(h, r.ctr64, sizeof h, cudaMemcpyDeviceToHost, s));
     LSG_CUDA(cudaStreamSynchronize(s));
+    if (r.bucketed && h[CTR_OVERFLOW]) continue; // a slack region overflowed: exact path
     const unsigned long long *book = h + CTR_BOOK;
     if (book[2] > cap) {
         const uint64_t need = book[2] + book[2] / 4;
@@ -513,6 +622,9 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
         *stats = st;
     }
     return LASAGNA_OK;
+  }
+    set_error("internal: no path completed");
+    return LASAGNA_ECUDA;
 }
 
 lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
@@ -558,6 +670,8 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
     r.lay = layout(g, G, cap, false);
     r.s = s;
     r.bind(workspace);
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    r.bucketed = attempt == 0 && use_bucketed(g);
     PhaseTimer tm;
     tm.on = false;
     if ((rc = sort_ctx_reset(r.sctx, s)) != LASAGNA_OK) return rc;
@@ -599,7 +713,10 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
             total += m;
         }
     }
+    unsigned long long ovf = 0;
+    LSG_CUDA(cudaMemcpyAsync(&ovf, r.ctr64 + CTR_OVERFLOW, 8, cudaMemcpyDeviceToHost, s));
     LSG_CUDA(cudaStreamSynchronize(s));
+    if (r.bucketed && ovf) continue; // a slack region overflowed: redo on the exact path
     *n_pairs = total;
     if (worst > cap) {
         *workspace_bytes = layout(g, G, worst + worst / 4, false).total;
@@ -613,6 +730,9 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
         return LASAGNA_ENOSPC;
     }
     return LASAGNA_OK;
+  }
+    set_error("internal: no path completed");
+    return LASAGNA_ECUDA;
 }
 
 lasagna_status lasagna_sort_u64(uint64_t *keys, uint64_t *scratch, uint64_t count,

@@ -17,82 +17,9 @@
 //
 // Traffic: the sorted array is streamed once (8 B per entry, 16 B per vertex); random
 // accesses are limited to the verification loads of fingerprint matches.
-#include "kernels.cuh"
+#include "joinwin.cuh"
 
 namespace lsg {
-
-constexpr int JOIN_THREADS = 512;
-constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
-constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
-constexpr int JOIN_SLOTS = 8192;   // hash chain heads (u32); chains through next[] (u16)
-constexpr int JOIN_BUF = 1024;     // staged output pairs
-
-// Candidates are staged in shared memory and verified in a separate, fully parallel pass
-// (a fingerprint match is rare: verifying it inline would run the long verify path with one
-// or two active lanes per warp).
-struct Stager {
-    unsigned long long *buf; // shared: staged (u << 32 | b) records, ~0 = rejected
-    uint32_t *bcount;        // shared
-    unsigned long long *pairs, cap, *count;
-};
-
-template <int W>
-__device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t s_ent, uint64_t p_ent,
-                                          uint64_t vmask, Stager &sg, unsigned long long &nfalse)
-{
-    const uint32_t u = (uint32_t)(s_ent & vmask), v = (uint32_t)(p_ent & vmask);
-    const uint32_t b = v ^ 1u;
-    if ((u >> 1) == (v >> 1) || u >= b) return; // R9: no same-read edge; each pair once
-    const unsigned long long rec = ((unsigned long long)u << 32) | b;
-    const uint32_t slot = atomicAdd(sg.bcount, 1u);
-    if (slot < JOIN_BUF) {
-        sg.buf[slot] = rec;
-        return;
-    }
-    // staging full: verify inline and emit straight to global memory
-    if (!verify_overlap<W>(a.packed, a.stride, a.L, u, v, a.l)) {
-        ++nfalse;
-        return;
-    }
-    const unsigned long long gs = atomicAdd(sg.count, 1ull);
-    if (gs < sg.cap) sg.pairs[gs] = rec;
-}
-
-// verify staged records [from, to) in parallel; rejected ones become ~0
-template <int W>
-__device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long long *buf,
-                                              uint32_t from, uint32_t to, unsigned long long &nfalse)
-{
-    for (uint32_t t = from + threadIdx.x; t < to; t += JOIN_THREADS) {
-        const unsigned long long rec = buf[t];
-        const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
-        if (!verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
-            buf[t] = ~0ull;
-            ++nfalse;
-        }
-    }
-}
-
-// write the accepted staged records [0, m) to the global pool (warp-aggregated slots)
-__device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint32_t m,
-                                             unsigned long long *pairs, unsigned long long cap,
-                                             unsigned long long *count)
-{
-    const int lane = threadIdx.x & 31;
-    for (uint32_t t0 = 0; t0 < m; t0 += JOIN_THREADS) {
-        const uint32_t t = t0 + threadIdx.x;
-        const unsigned long long rec = t < m ? buf[t] : ~0ull;
-        const bool ok = rec != ~0ull;
-        const uint32_t bal = __ballot_sync(0xffffffffu, ok);
-        unsigned long long base = 0;
-        if (lane == 0 && bal) base = atomicAdd(count, (unsigned long long)__popc(bal));
-        base = __shfl_sync(0xffffffffu, base, 0);
-        if (ok) {
-            const unsigned long long pos = base + __popc(bal & ((1u << lane) - 1));
-            if (pos < cap) pairs[pos] = rec;
-        }
-    }
-}
 
 // first index i in [lo, hi) with (A[i] >> shift) >= b (lower bound of bucket b), by one
 // warp: each round the 32 lanes probe 32 evenly spaced positions (32-ary search).
@@ -133,8 +60,6 @@ join_kernel(JoinArgs a)
 
     const uint64_t N = a.N;
     const uint32_t bshift = 64 - a.T;
-    const uint32_t kshift = a.vbits + 1; // key bits above tag + vid
-    const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint64_t *A = a.keys;
     const int warp = threadIdx.x >> 5;
 
@@ -201,55 +126,13 @@ join_kernel(JoinArgs a)
             }
             __syncthreads();
             const uint64_t be = s_end;
-            for (uint64_t i = t0 + threadIdx.x; i < be; i += JOIN_THREADS) {
-                const uint64_t e = A[i];
-                if (!((e >> a.vbits) & 1)) continue;
-                for (uint64_t j = t0; j < be; ++j) {
-                    const uint64_t p = A[j];
-                    if (((p >> a.vbits) & 1) == 0 && ((p ^ e) >> kshift) == 0)
-                        candidate<W>(a, e, p, vmask, em, nfalse);
-                }
-            }
+            oversized_join<W>(a, A, t0, be, em, nfalse);
             t1 = be;
         } else {
-            // ---- hash the prefix entries of [t0, t1) (chained: one atomicExch per insert),
-            // then probe with the suffix entries
-            const uint32_t m = (uint32_t)(t1 - t0);
-            const uint32_t tag = (epoch & 0xFFFFu) << 16;
-            for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
-                const uint64_t e = ent[k];
-                if ((e >> a.vbits) & 1) continue;
-                const uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
-                const uint32_t old = atomicExch(&slot[h], tag | k);
-                next[k] = (old >> 16) == (tag >> 16) ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
-            }
-            __syncthreads();
-            for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
-                const uint64_t e = ent[k];
-                if (!((e >> a.vbits) & 1)) continue;
-                const uint32_t sv = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
-                uint32_t sl = (sv >> 16) == (tag >> 16) ? (sv & 0xFFFFu) : 0xFFFFu;
-                while (sl != 0xFFFFu) {
-                    const uint64_t p = ent[sl];
-                    if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-                    sl = next[sl];
-                }
-            }
+            hash_join_window<W>(a, ent, (uint32_t)(t1 - t0), slot, next, epoch, em, nfalse);
         }
         __syncthreads();
-        // verify this window's candidates, flush the staging buffer when half full
-        {
-            const uint32_t to = min(bcount, (uint32_t)JOIN_BUF);
-            verify_staged<W>(a, buf, vdone, to, nfalse);
-            __syncthreads();
-            if (to >= JOIN_BUF / 2) {
-                flush_staged(buf, to, a.pairs, a.cap, a.count);
-                __syncthreads();
-                if (threadIdx.x == 0) bcount = 0, vdone = 0;
-            } else if (threadIdx.x == 0) {
-                vdone = to;
-            }
-        }
+        window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
         __syncthreads();
         t0 = t1;
     }

@@ -357,3 +357,49 @@ def test_planner_and_small_workspace(lz):
     budget = (need + ws_all) // 2
     lp_small, ws_small = lz.plan(n, L, l_min, budget)
     assert 1 <= lp_small < lp_all and ws_small <= budget
+
+
+@gpu
+def test_region_overflow_falls_back_to_exact_path(tmp_path):
+    """Slack regions that overflow (forced here) are detected and the call redoes the work on
+    the exact LSD path: the result is still bit-exact."""
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, torch, readgen, oracle\n"
+        "import paper_conf_ipps_goswamilsp18_b200 as lz\n"
+        "reads = readgen.config_reads('cfg1', n=8000)\n"
+        "packed = lz.load_reads(torch.from_numpy(reads).cuda())\n"
+        "r = lz.greedy_graph(packed, 8000, 100, 63)\n"
+        "es, eo, m, _ = oracle.greedy_graph(reads, 63)\n"
+        "assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), es)\n"
+        "assert np.array_equal(r.olen.cpu().numpy(), eo)\n"
+        "pl, pa, pb = lz.overlaps(packed, 8000, 100, 63)\n"
+        "assert pl.numel() == m\n"
+        "print('ok')\n")
+    env = dict(os.environ, LASAGNA_TEST_TIGHT_REGIONS="1", PYTHONPATH=ROOT)
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                         cwd=ROOT, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+
+
+@gpu
+@pytest.mark.parametrize("path", ["exact"])
+def test_exact_path_cfg1(path):
+    """The exact LSD-sort path (LASAGNA_PATH=exact) stays bit-exact too."""
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, torch, readgen, oracle\n"
+        "import paper_conf_ipps_goswamilsp18_b200 as lz\n"
+        "reads = readgen.config_reads('cfg1')\n"
+        "packed = lz.load_reads(torch.from_numpy(reads).cuda())\n"
+        "r = lz.greedy_graph(packed, 20000, 100, 63)\n"
+        "es, eo, m, _ = oracle.greedy_graph(reads, 63)\n"
+        "assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), es)\n"
+        "assert np.array_equal(r.olen.cpu().numpy(), eo)\n"
+        "print('ok')\n")
+    env = dict(os.environ, LASAGNA_PATH=path, PYTHONPATH=ROOT)
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                         cwd=ROOT, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
