@@ -163,6 +163,48 @@ __host__ __device__ inline uint32_t stride_for(uint32_t L)
     return w <= 1 ? 1 : w <= 2 ? 2 : w <= 4 ? 4 : 8;
 }
 
+// ----------------------------------------------------------------- bulk async copies (TMA engine)
+// 1-D cp.async.bulk global -> shared with an mbarrier completing on the transferred bytes
+// (SASS UBLKCP): the copy engine moves the next tile while the CTA works on the current one.
+__device__ __forceinline__ uint32_t smem_u32(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
+                 : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init()
+{
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async()
+{
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// one elected thread: expect `bytes` on `bar` and start the copy
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes,
+                                          unsigned long long *bar)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, "
+                 "[%3];" ::"r"(smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t phase)
+{
+    asm volatile("{\n\t.reg .pred p;\n"
+                 "WAIT_%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                 "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+                 "r"(phase)
+                 : "memory");
+}
+
 // ----------------------------------------------------------------- host-side error plumbing
 void set_error(const char *fmt, ...);
 lasagna_status cuda_status(cudaError_t e, const char *what);
@@ -201,7 +243,7 @@ lasagna_status dispatch_W(uint32_t L, F &&f)
 
 __host__ __device__ __forceinline__ uint64_t min64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
-inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+__host__ __device__ inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
 inline int num_sms()
 {

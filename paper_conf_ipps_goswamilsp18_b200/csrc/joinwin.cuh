@@ -119,6 +119,35 @@ __device__ __forceinline__ void hash_join_window(const JoinArgs &a, const uint64
     }
 }
 
+// split form: prefix entries ent[0..nP), suffix entries ent[s0..s0+nS) (no tag tests, no
+// divergence between the insert and probe passes)
+template <int W>
+__device__ __forceinline__ void hash_join_split(const JoinArgs &a, const uint64_t *ent, uint32_t nP,
+                                                uint32_t s0, uint32_t nS, uint32_t *slot,
+                                                unsigned short *next, uint32_t epoch, Stager &em,
+                                                unsigned long long &nfalse)
+{
+    const uint32_t kshift = a.vbits + 1;
+    const uint64_t vmask = (1ull << a.vbits) - 1;
+    const uint32_t tag = (epoch & 0xFFFFu) << 16;
+    for (uint32_t k = threadIdx.x; k < nP; k += JOIN_THREADS) {
+        const uint32_t h = (uint32_t)(ent[k] >> kshift) & (JOIN_SLOTS - 1);
+        const uint32_t old = atomicExch(&slot[h], tag | k);
+        next[k] = (old >> 16) == (tag >> 16) ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
+    }
+    __syncthreads();
+    for (uint32_t k = threadIdx.x; k < nS; k += JOIN_THREADS) {
+        const uint64_t e = ent[s0 + k];
+        const uint32_t sv = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
+        uint32_t sl = (sv >> 16) == (tag >> 16) ? (sv & 0xFFFFu) : 0xFFFFu;
+        while (sl != 0xFFFFu) {
+            const uint64_t p = ent[sl];
+            if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+            sl = next[sl];
+        }
+    }
+}
+
 // a run [lo, hi) of global entries too large for a window (massively repeated fingerprints):
 // every suffix entry scans the whole run in global memory
 template <int W>

@@ -27,7 +27,7 @@ namespace lsg {
 
 constexpr int SC_THREADS = 512; // reads per scatter CTA (one per thread)
 constexpr int RF_THREADS = 512;
-constexpr int RF_KPT = 16;
+constexpr int RF_KPT = 8;
 constexpr int RF_TILE = RF_THREADS * RF_KPT;
 
 // exclusive scan over the first 256 threads of a block of >= 256 threads (8 warps used);
@@ -149,29 +149,53 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
 }
 
 // ------------------------------------------------------------------ level k -> k+1
+// One CTA owns one region and streams it: the bulk-copy engine prefetches tile t+1 into the
+// other half of a double buffer while tile t is ranked (shared atomics: order inside a
+// sub-region is irrelevant), staged by digit and written out in digit runs.
 __global__ void __launch_bounds__(RF_THREADS, 2)
 refine_kernel(RefineArgs a)
 {
-    extern __shared__ __align__(16) uint64_t rstage[]; // [RF_TILE]
+    extern __shared__ __align__(128) uint64_t rsm[];
+    uint64_t *inb = rsm;                 // [2][RF_TILE]
+    uint64_t *rstage = rsm + 2 * RF_TILE; // [RF_TILE]
+    __shared__ __align__(8) unsigned long long mbar[2];
     __shared__ uint32_t cnt[256], lstart[256], running[256], wsum[8];
     const uint64_t r = blockIdx.x;
     const uint32_t fill = a.fill_in[r];
     const uint64_t count = min64(fill, a.cap_in);
     const uint64_t *src = a.in + r * a.cap_in;
     uint64_t *dst = a.out + r * 256 * a.cap_out;
+    const uint32_t ntiles = (uint32_t)ceil_div(count, RF_TILE);
     if (threadIdx.x < 256) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
+    if (threadIdx.x == 0) {
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
+        fence_mbar_init();
+    }
     __syncthreads();
-    for (uint64_t t0 = 0; t0 < count; t0 += RF_TILE) {
+    // bytes of tile t (rounded up to 16: the region capacity is even, so the rounding stays
+    // inside the region)
+    auto tile_bytes = [&](uint32_t t) {
+        const uint64_t m = min64(RF_TILE, count - (uint64_t)t * RF_TILE);
+        return (uint32_t)(((m * 8) + 15) & ~15ull);
+    };
+    if (threadIdx.x == 0 && ntiles) bulk_load(inb, src, tile_bytes(0), &mbar[0]);
+    for (uint32_t t = 0; t < ntiles; ++t) {
+        const uint32_t bsel = t & 1;
+        const uint64_t t0 = (uint64_t)t * RF_TILE;
         const uint32_t m = (uint32_t)min64(RF_TILE, count - t0);
-        uint64_t key[RF_KPT];
+        if (threadIdx.x == 0 && t + 1 < ntiles) {
+            fence_proxy_async();
+            bulk_load(inb + (bsel ^ 1) * RF_TILE, src + t0 + RF_TILE, tile_bytes(t + 1),
+                      &mbar[bsel ^ 1]);
+        }
+        mbar_wait(&mbar[bsel], (t >> 1) & 1);
+        const uint64_t *tin = inb + bsel * RF_TILE;
         uint32_t rk[RF_KPT];
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
-            if (idx < m) {
-                key[q] = src[t0 + idx];
-                rk[q] = atomicAdd(&cnt[(uint32_t)(key[q] >> a.dshift) & 255u], 1u);
-            }
+            if (idx < m) rk[q] = atomicAdd(&cnt[(uint32_t)(tin[idx] >> a.dshift) & 255u], 1u);
         }
         __syncthreads();
         uint32_t c = 0;
@@ -185,13 +209,16 @@ refine_kernel(RefineArgs a)
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
-            if (idx < m) rstage[lstart[(uint32_t)(key[q] >> a.dshift) & 255u] + rk[q]] = key[q];
+            if (idx < m) {
+                const uint64_t k = tin[idx];
+                rstage[lstart[(uint32_t)(k >> a.dshift) & 255u] + rk[q]] = k;
+            }
         }
         __syncthreads();
-        for (uint32_t t = threadIdx.x; t < m; t += RF_THREADS) {
-            const uint64_t k = rstage[t];
+        for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
+            const uint64_t k = rstage[u];
             const uint32_t d = (uint32_t)(k >> a.dshift) & 255u;
-            const uint64_t pos = (uint64_t)running[d] + (t - lstart[d]);
+            const uint64_t pos = (uint64_t)running[d] + (u - lstart[d]);
             if (pos < a.cap_out) dst[(uint64_t)d * a.cap_out + pos] = k;
             else *a.overflow = 1u;
         }
@@ -209,7 +236,7 @@ refine_kernel(RefineArgs a)
 lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStream_t s)
 {
     if (n_regions == 0) return LASAGNA_OK;
-    const size_t smem = (size_t)RF_TILE * 8;
+    const size_t smem = (size_t)3 * RF_TILE * 8;
     LSG_CUDA(cudaFuncSetAttribute(refine_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)smem));
     refine_kernel<<<(unsigned)n_regions, RF_THREADS, smem, s>>>(args);
@@ -232,7 +259,7 @@ bucket_join_kernel(BucketJoinArgs b)
         reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4);
     uint32_t *sfill =
         reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4 + JOIN_CAP * 2);
-    __shared__ uint32_t bcount, vdone, s_nb, s_total;
+    __shared__ uint32_t bcount, vdone, s_nb, s_total, s_np, s_ns;
     const JoinArgs &a = b.j;
     const uint64_t nb = b.n_buckets;
     const uint64_t b0 = nb * blockIdx.x / gridDim.x, b1 = nb * (blockIdx.x + 1) / gridDim.x;
@@ -270,15 +297,38 @@ bucket_join_kernel(BucketJoinArgs b)
                 const uint64_t bk = c0 + k;
                 oversized_join<W>(a, b.buckets + bk * b.bucket_cap, 0, total, em, nfalse);
             } else {
-                uint32_t off = 0;
+                // stage the window split by list: prefix entries from the front, suffix
+                // entries from the back (warp-aggregated slots)
+                if (threadIdx.x == 0) s_np = 0, s_ns = 0;
+                __syncthreads();
+                const int lane = threadIdx.x & 31;
                 for (uint32_t q = 0; q < nbw; ++q) {
                     const uint32_t f = sfill[k + q];
                     const uint64_t *srcb = b.buckets + (c0 + k + q) * b.bucket_cap;
-                    for (uint32_t t = threadIdx.x; t < f; t += JOIN_THREADS) ent[off + t] = srcb[t];
-                    off += f;
+                    for (uint32_t t0 = 0; t0 < f; t0 += JOIN_THREADS) {
+                        const uint32_t t = t0 + threadIdx.x;
+                        const bool ok = t < f;
+                        const uint64_t e = ok ? srcb[t] : 0;
+                        const bool isS = ok && ((e >> a.vbits) & 1);
+                        const uint32_t bS = __ballot_sync(0xffffffffu, isS);
+                        const uint32_t bP = __ballot_sync(0xffffffffu, ok && !isS);
+                        uint32_t baseP = 0, baseS = 0;
+                        if (lane == 0) {
+                            if (bP) baseP = atomicAdd(&s_np, (uint32_t)__popc(bP));
+                            if (bS) baseS = atomicAdd(&s_ns, (uint32_t)__popc(bS));
+                        }
+                        baseP = __shfl_sync(0xffffffffu, baseP, 0);
+                        baseS = __shfl_sync(0xffffffffu, baseS, 0);
+                        const uint32_t lt = (1u << lane) - 1;
+                        if (ok) {
+                            if (isS) ent[JOIN_CAP - 1 - (baseS + __popc(bS & lt))] = e;
+                            else ent[baseP + __popc(bP & lt)] = e;
+                        }
+                    }
                 }
                 __syncthreads();
-                hash_join_window<W>(a, ent, total, slot, next, epoch, em, nfalse);
+                const uint32_t nP = s_np, nS = s_ns;
+                hash_join_split<W>(a, ent, nP, JOIN_CAP - nS, nS, slot, next, epoch, em, nfalse);
             }
             __syncthreads();
             window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
