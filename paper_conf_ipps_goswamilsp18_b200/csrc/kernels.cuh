@@ -67,10 +67,11 @@ struct ScatterArgs {
     const uint64_t *packed;
     uint64_t n, read_offset;
     uint32_t L, stride, l_lo, l_hi, vbits;
-    uint64_t *out;      // [G][256][cap] level-1 regions (top 8 key bits)
-    uint32_t *fill;     // [G][256]
+    uint64_t *out;      // [G][256][cap] level-1 regions (top 8 key bits); split: [G][256][2][cap]
+    uint32_t *fill;     // [G][256] (split: [G][256][2])
     uint64_t cap;
     uint32_t *overflow;
+    bool split;         // final level: prefix and suffix entries in separate halves
 };
 lasagna_status launch_scatter_table(const ScatterArgs &a, cudaStream_t s);
 struct RefineArgs {
@@ -78,17 +79,19 @@ struct RefineArgs {
     const uint32_t *fill_in;
     uint64_t cap_in;
     uint32_t dshift;    // this level's digit: bits [dshift, dshift + 8)
-    uint64_t *out;      // [regions][256][cap_out]
-    uint32_t *fill_out; // [regions][256]
+    uint64_t *out;      // [regions][256][cap_out] (split: [regions][256][2][cap_out])
+    uint32_t *fill_out; // [regions][256] (split: [regions][256][2])
     uint64_t cap_out;
+    uint32_t vbits;
     uint32_t *overflow;
+    bool split;
 };
 lasagna_status launch_refine(const RefineArgs &a, uint64_t n_regions, cudaStream_t s);
 struct BucketJoinArgs {
     JoinArgs j;               // packed, L, stride, l, vbits, pairs, cap, count, false_matches
-    const uint64_t *buckets;  // [n_buckets][bucket_cap]
-    const uint32_t *fills;    // [n_buckets]
-    uint64_t bucket_cap, n_buckets;
+    const uint64_t *buckets;  // [n_buckets][2][half_cap]: prefix half, suffix half
+    const uint32_t *fills;    // [n_buckets][2]
+    uint64_t half_cap, n_buckets;
     uint32_t *overflow;
 };
 lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s);

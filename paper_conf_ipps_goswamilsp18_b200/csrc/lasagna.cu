@@ -45,7 +45,8 @@ struct Geometry {
     uint32_t L, l_min, n_len, vbits, T;
     // bucketed path (partition.cu): P = T/8 MSD levels, region capacities with slack
     uint32_t P;
-    uint64_t cap1, cap2;
+    uint64_t cap1;          // level-1 region capacity (unsplit, P = 2)
+    uint64_t half1, half2;  // half-bucket capacities of the final level (P = 1 / P = 2)
 };
 
 // capacity of a region expecting `mean` keys: mean + 8 sigma + 32 (multinomial occupancy;
@@ -82,7 +83,8 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     g.T = std::min<uint32_t>(8u * (uint32_t)P, 63u - g.vbits);
     g.P = g.T / 8;
     g.cap1 = region_cap((double)g.N / 256.0);
-    g.cap2 = region_cap((double)g.N / 65536.0);
+    g.half1 = region_cap((double)g.N / 512.0);
+    g.half2 = region_cap((double)g.N / 131072.0);
     return g;
 }
 
@@ -113,12 +115,12 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     // tabA/tabB: the exact path's LSD ping-pong buffers, or the bucketed path's level-1 and
     // level-2 regions (with slack)
     const size_t exact_b = (size_t)G * g.N * 8;
-    const size_t lvl1_b = (size_t)G * 256 * g.cap1 * 8;
-    const size_t lvl2_b = g.P >= 2 ? (size_t)G * 65536 * g.cap2 * 8 : 0;
+    const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half1 : 256 * g.cap1) * 8;
+    const size_t lvl2_b = g.P >= 2 ? (size_t)G * 131072 * g.half2 * 8 : 0;
     l.tabA = take(std::max(exact_b, lvl1_b));
     l.tabB = take(std::max(exact_b, lvl2_b));
-    l.fill1 = take((size_t)G * 256 * 4);
-    l.fill2 = take(g.P >= 2 ? (size_t)G * 65536 * 4 : 4);
+    l.fill1 = take((size_t)G * 512 * 4);
+    l.fill2 = take(g.P >= 2 ? (size_t)G * 131072 * 4 : 4);
     l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
     l.status = take(l.status_bytes);
     l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
@@ -267,7 +269,7 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     const Geometry &g = r.g;
     const uint32_t G = l_hi - l_lo + 1;
     unsigned int *ovf = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
-    LSG_CUDA(cudaMemsetAsync(r.fill1, 0, (size_t)G * 256 * 4, r.s));
+    LSG_CUDA(cudaMemsetAsync(r.fill1, 0, (size_t)G * 512 * 4, r.s));
     ScatterArgs sa;
     sa.packed = packed;
     sa.n = g.n;
@@ -279,7 +281,8 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.vbits = g.vbits;
     sa.out = r.tab[0];
     sa.fill = r.fill1;
-    sa.cap = g.cap1;
+    sa.split = g.P == 1; // one level: the level-1 regions are the (split) buckets
+    sa.cap = sa.split ? g.half1 : g.cap1;
     sa.overflow = ovf;
     lasagna_status rc;
     if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
@@ -293,7 +296,9 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
         ra.dshift = 48;
         ra.out = r.tab[1];
         ra.fill_out = r.fill2;
-        ra.cap_out = g.cap2;
+        ra.cap_out = g.half2;
+        ra.vbits = g.vbits;
+        ra.split = true;
         ra.overflow = ovf;
         if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
         if ((rc = launch_refine(ra, (uint64_t)G * 256, r.s)) != LASAGNA_OK) return rc;
@@ -368,14 +373,14 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.j = ja;
         bj.overflow = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
         if (g.P >= 2) {
-            bj.buckets = r.tab[1] + (uint64_t)s * 65536 * g.cap2;
-            bj.fills = r.fill2 + (uint64_t)s * 65536;
-            bj.bucket_cap = g.cap2;
+            bj.buckets = r.tab[1] + (uint64_t)s * 131072 * g.half2;
+            bj.fills = r.fill2 + (uint64_t)s * 131072;
+            bj.half_cap = g.half2;
             bj.n_buckets = 65536;
         } else {
-            bj.buckets = r.tab[0] + (uint64_t)s * 256 * g.cap1;
-            bj.fills = r.fill1 + (uint64_t)s * 256;
-            bj.bucket_cap = g.cap1;
+            bj.buckets = r.tab[0] + (uint64_t)s * 512 * g.half1;
+            bj.fills = r.fill1 + (uint64_t)s * 512;
+            bj.half_cap = g.half1;
             bj.n_buckets = 256;
         }
         rc = launch_bucket_join(bj, r.s);

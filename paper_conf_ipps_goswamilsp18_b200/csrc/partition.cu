@@ -30,9 +30,10 @@ constexpr int RF_THREADS = 512;
 constexpr int RF_KPT = 8;
 constexpr int RF_TILE = RF_THREADS * RF_KPT;
 
-// exclusive scan over the first 256 threads of a block of >= 256 threads (8 warps used);
-// every thread of the block must call it.  wsum: 8 shared words.
-__device__ __forceinline__ uint32_t block_scan256(uint32_t v, uint32_t *wsum)
+// exclusive scan of v over the first NB threads (NB a multiple of 32, <= 512); every thread of
+// the block must call it.  wsum: 16 shared words.
+template <int NB>
+__device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t *wsum)
 {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t x = v;
@@ -41,22 +42,33 @@ __device__ __forceinline__ uint32_t block_scan256(uint32_t v, uint32_t *wsum)
         uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
         if (lane >= o) x += y;
     }
-    if (threadIdx.x < 256 && lane == 31) wsum[warp] = x;
+    if (threadIdx.x < NB && lane == 31) wsum[warp] = x;
     __syncthreads();
     uint32_t add = 0;
-    if (threadIdx.x < 256)
+    if (threadIdx.x < NB)
         for (int w = 0; w < warp; ++w) add += wsum[w];
     __syncthreads();
     return x - v + add;
 }
 
+// partition bin of a key: its digit, or (SPLIT, the final level) digit * 2 + list tag so that
+// each bucket stores its prefix entries and its suffix entries in two halves
+template <bool SPLIT>
+__device__ __forceinline__ uint32_t bin_of(uint64_t key, uint32_t dshift, uint32_t vbits)
+{
+    const uint32_t d = (uint32_t)(key >> dshift) & 255u;
+    if constexpr (SPLIT) return (d << 1) | (uint32_t)((key >> vbits) & 1);
+    else return d;
+}
+
 // ------------------------------------------------------------------ level 1: fused with a2
-template <int W>
+template <int W, bool SPLIT>
 __global__ void __launch_bounds__(SC_THREADS, 2)
 scatter_table_kernel(ScatterArgs a)
 {
+    constexpr int NB = SPLIT ? 512 : 256;
     __shared__ uint64_t stage[SC_THREADS * 4];
-    __shared__ uint32_t cnt[256], lstart[256], base[256], wsum[8];
+    __shared__ uint32_t cnt[NB], lstart[NB], base[NB], wsum[16];
     __shared__ uint32_t s_total;
 
     const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
@@ -69,7 +81,7 @@ scatter_table_kernel(ScatterArgs a)
 #pragma unroll
         for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
     }
-    if (threadIdx.x < 256) cnt[threadIdx.x] = 0;
+    if (threadIdx.x < NB) cnt[threadIdx.x] = 0;
     __syncthreads();
     const uint64_t keep = ~((2ull << a.vbits) - 1);
     const uint64_t tagS = 1ull << a.vbits;
@@ -98,23 +110,23 @@ scatter_table_kernel(ScatterArgs a)
                 kk[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
-                    dd[q] = (uint32_t)(kk[q] >> 56);
+                    dd[q] = bin_of<SPLIT>(kk[q], 56, a.vbits);
                     rk[q] = atomicAdd(&cnt[dd[q]], 1u);
                 }
             }
             __syncthreads();
             const uint32_t seg = l - a.l_lo;
             uint32_t c = 0;
-            if (threadIdx.x < 256) {
+            if (threadIdx.x < NB) {
                 c = cnt[threadIdx.x];
                 cnt[threadIdx.x] = 0;
                 base[threadIdx.x] =
-                    c ? atomicAdd(&a.fill[(uint64_t)seg * 256 + threadIdx.x], c) : 0u;
+                    c ? atomicAdd(&a.fill[(uint64_t)seg * NB + threadIdx.x], c) : 0u;
             }
-            const uint32_t ex = block_scan256(c, wsum);
-            if (threadIdx.x < 256) {
+            const uint32_t ex = block_scan<NB>(c, wsum);
+            if (threadIdx.x < NB) {
                 lstart[threadIdx.x] = ex;
-                if (threadIdx.x == 255) s_total = ex + c;
+                if (threadIdx.x == NB - 1) s_total = ex + c;
             }
             __syncthreads();
             if (valid) {
@@ -123,10 +135,10 @@ scatter_table_kernel(ScatterArgs a)
             }
             __syncthreads();
             const uint32_t total = s_total;
-            uint64_t *dst = a.out + (uint64_t)seg * 256 * a.cap;
+            uint64_t *dst = a.out + (uint64_t)seg * NB * a.cap;
             for (uint32_t t = threadIdx.x; t < total; t += SC_THREADS) {
                 const uint64_t key = stage[t];
-                const uint32_t d = (uint32_t)(key >> 56);
+                const uint32_t d = bin_of<SPLIT>(key, 56, a.vbits);
                 const uint64_t pos = (uint64_t)base[d] + (t - lstart[d]);
                 if (pos < a.cap) dst[(uint64_t)d * a.cap + pos] = key;
                 else *a.overflow = 1u;
@@ -142,7 +154,10 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
         const uint64_t blocks = ceil_div(args.n, SC_THREADS);
-        scatter_table_kernel<W><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
+        if (args.split)
+            scatter_table_kernel<W, true><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
+        else
+            scatter_table_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
         LSG_LAUNCHED("scatter_table_kernel");
         return LASAGNA_OK;
     });
@@ -152,21 +167,23 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
 // One CTA owns one region and streams it: the bulk-copy engine prefetches tile t+1 into the
 // other half of a double buffer while tile t is ranked (shared atomics: order inside a
 // sub-region is irrelevant), staged by digit and written out in digit runs.
+template <bool SPLIT>
 __global__ void __launch_bounds__(RF_THREADS, 2)
 refine_kernel(RefineArgs a)
 {
+    constexpr int NB = SPLIT ? 512 : 256;
     extern __shared__ __align__(128) uint64_t rsm[];
     uint64_t *inb = rsm;                 // [2][RF_TILE]
     uint64_t *rstage = rsm + 2 * RF_TILE; // [RF_TILE]
     __shared__ __align__(8) unsigned long long mbar[2];
-    __shared__ uint32_t cnt[256], lstart[256], running[256], wsum[8];
+    __shared__ uint32_t cnt[NB], lstart[NB], running[NB], wsum[16];
     const uint64_t r = blockIdx.x;
     const uint32_t fill = a.fill_in[r];
     const uint64_t count = min64(fill, a.cap_in);
     const uint64_t *src = a.in + r * a.cap_in;
-    uint64_t *dst = a.out + r * 256 * a.cap_out;
+    uint64_t *dst = a.out + r * NB * a.cap_out;
     const uint32_t ntiles = (uint32_t)ceil_div(count, RF_TILE);
-    if (threadIdx.x < 256) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
+    if (threadIdx.x < NB) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
         mbar_init(&mbar[0], 1);
         mbar_init(&mbar[1], 1);
@@ -195,39 +212,39 @@ refine_kernel(RefineArgs a)
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
-            if (idx < m) rk[q] = atomicAdd(&cnt[(uint32_t)(tin[idx] >> a.dshift) & 255u], 1u);
+            if (idx < m) rk[q] = atomicAdd(&cnt[bin_of<SPLIT>(tin[idx], a.dshift, a.vbits)], 1u);
         }
         __syncthreads();
         uint32_t c = 0;
-        if (threadIdx.x < 256) {
+        if (threadIdx.x < NB) {
             c = cnt[threadIdx.x];
             cnt[threadIdx.x] = 0;
         }
-        const uint32_t ex = block_scan256(c, wsum);
-        if (threadIdx.x < 256) lstart[threadIdx.x] = ex;
+        const uint32_t ex = block_scan<NB>(c, wsum);
+        if (threadIdx.x < NB) lstart[threadIdx.x] = ex;
         __syncthreads();
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
             if (idx < m) {
                 const uint64_t k = tin[idx];
-                rstage[lstart[(uint32_t)(k >> a.dshift) & 255u] + rk[q]] = k;
+                rstage[lstart[bin_of<SPLIT>(k, a.dshift, a.vbits)] + rk[q]] = k;
             }
         }
         __syncthreads();
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
-            const uint32_t d = (uint32_t)(k >> a.dshift) & 255u;
+            const uint32_t d = bin_of<SPLIT>(k, a.dshift, a.vbits);
             const uint64_t pos = (uint64_t)running[d] + (u - lstart[d]);
             if (pos < a.cap_out) dst[(uint64_t)d * a.cap_out + pos] = k;
             else *a.overflow = 1u;
         }
         __syncthreads();
-        if (threadIdx.x < 256) running[threadIdx.x] += c;
+        if (threadIdx.x < NB) running[threadIdx.x] += c;
         __syncthreads();
     }
-    if (threadIdx.x < 256) {
-        a.fill_out[r * 256 + threadIdx.x] = running[threadIdx.x];
+    if (threadIdx.x < NB) {
+        a.fill_out[r * NB + threadIdx.x] = running[threadIdx.x];
         if (running[threadIdx.x] > a.cap_out) *a.overflow = 1u;
     }
     if (threadIdx.x == 0 && fill > a.cap_in) *a.overflow = 1u;
@@ -237,109 +254,207 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 {
     if (n_regions == 0) return LASAGNA_OK;
     const size_t smem = (size_t)3 * RF_TILE * 8;
-    LSG_CUDA(cudaFuncSetAttribute(refine_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)smem));
-    refine_kernel<<<(unsigned)n_regions, RF_THREADS, smem, s>>>(args);
+    auto kern = args.split ? refine_kernel<true> : refine_kernel<false>;
+    LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    kern<<<(unsigned)n_regions, RF_THREADS, smem, s>>>(args);
     LSG_LAUNCHED("refine_kernel");
     return LASAGNA_OK;
 }
 
 // ------------------------------------------------------------------ a5 over the buckets
-constexpr int BJ_FILLS = 2048; // bucket fills staged per chunk
+// Buckets are stored split: prefix entries [b][0][0..fillP), suffix entries [b][1][0..fillS).
+// A window = consecutive whole buckets whose halves fit the staging buffers; the copy engine
+// (cp.async.bulk) stages window w+1 while window w is joined.  A half's copy is rounded up
+// to 16 bytes, so an odd fill drags one stale slot along: it is overwritten with a sentinel
+// key (~0: tag bits set, never equal to a real key of the other list) after the copy lands.
+constexpr int BJ_HALF = 2048;   // staged prefix (and suffix) entries per window
+constexpr int BJ_MAXB = 64;     // buckets per window
+constexpr int BJ_FILLS = 1024;  // buckets whose fills are staged at once
+constexpr int BJ_SLOTS = 4096;
+
+struct WinDesc {
+    uint32_t nb, nP, nS;             // buckets, staged prefix / suffix slots (padded)
+    uint32_t odd[2 * BJ_MAXB];       // staging offsets of the sentinel slots (or ~0)
+};
+
+template <int W>
+__device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const uint64_t *P,
+                                                     uint32_t nP, const uint64_t *S, uint32_t nS,
+                                                     Stager &em, unsigned long long &nfalse)
+{
+    const uint32_t kshift = a.vbits + 1;
+    const uint64_t vmask = (1ull << a.vbits) - 1;
+    for (uint32_t i = threadIdx.x; i < nS; i += JOIN_THREADS) {
+        const uint64_t e = S[i];
+        for (uint32_t j = 0; j < nP; ++j) {
+            const uint64_t p = P[j];
+            if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+        }
+    }
+}
 
 template <int W>
 __global__ void __launch_bounds__(JOIN_THREADS, 2)
 bucket_join_kernel(BucketJoinArgs b)
 {
-    extern __shared__ __align__(16) unsigned char jsm[];
-    uint64_t *ent = reinterpret_cast<uint64_t *>(jsm);                                   // [CAP]
-    unsigned long long *buf = reinterpret_cast<unsigned long long *>(jsm + JOIN_CAP * 8); // [BUF]
-    uint32_t *slot = reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8);     // [SLOTS]
-    unsigned short *next =
-        reinterpret_cast<unsigned short *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4);
-    uint32_t *sfill =
-        reinterpret_cast<uint32_t *>(jsm + (JOIN_CAP + JOIN_BUF) * 8 + JOIN_SLOTS * 4 + JOIN_CAP * 2);
-    __shared__ uint32_t bcount, vdone, s_nb, s_total, s_np, s_ns;
+    extern __shared__ __align__(128) unsigned char jsm[];
+    uint64_t *pst = reinterpret_cast<uint64_t *>(jsm);                    // [2][BJ_HALF]
+    uint64_t *sst = pst + 2 * BJ_HALF;                                   // [2][BJ_HALF]
+    unsigned long long *buf = reinterpret_cast<unsigned long long *>(sst + 2 * BJ_HALF); // [BUF]
+    uint32_t *slot = reinterpret_cast<uint32_t *>(buf + JOIN_BUF);       // [BJ_SLOTS]
+    unsigned short *next = reinterpret_cast<unsigned short *>(slot + BJ_SLOTS); // [BJ_HALF]
+    uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
+    __shared__ WinDesc wd[2];
+    __shared__ __align__(8) unsigned long long mbar[2];
+    __shared__ uint32_t bcount, vdone, s_over;
     const JoinArgs &a = b.j;
-    const uint64_t nb = b.n_buckets;
-    const uint64_t b0 = nb * blockIdx.x / gridDim.x, b1 = nb * (blockIdx.x + 1) / gridDim.x;
-    if (threadIdx.x == 0) bcount = 0, vdone = 0;
-    for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+    const uint64_t nbk = b.n_buckets;
+    const uint64_t b0 = nbk * blockIdx.x / gridDim.x, b1 = nbk * (blockIdx.x + 1) / gridDim.x;
+    const uint32_t kshift = a.vbits + 1;
+    const uint64_t vmask = (1ull << a.vbits) - 1;
+    if (threadIdx.x == 0) {
+        bcount = 0, vdone = 0;
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
+        fence_mbar_init();
+    }
+    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
     Stager em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
-    uint32_t epoch = 0;
+    uint32_t epoch = 0, phases = 0; // bit w: parity of the next phase of mbar[w]
+
     for (uint64_t c0 = b0; c0 < b1; c0 += BJ_FILLS) {
         const uint32_t nc = (uint32_t)min64(BJ_FILLS, b1 - c0);
         __syncthreads();
-        for (uint32_t t = threadIdx.x; t < nc; t += JOIN_THREADS) {
-            const uint32_t f = b.fills[c0 + t];
-            if (f > b.bucket_cap) *b.overflow = 1u;
-            sfill[t] = (uint32_t)min64(f, b.bucket_cap);
+        for (uint32_t t = threadIdx.x; t < 2 * nc; t += JOIN_THREADS) {
+            const uint32_t f = b.fills[2 * c0 + t];
+            if (f > b.half_cap) *b.overflow = 1u;
+            sfill[t] = (uint32_t)min64(f, b.half_cap);
         }
         __syncthreads();
-        uint32_t k = 0;
-        while (k < nc) {
-            // window: buckets [k, k + nb_w) with total <= JOIN_CAP (at least one bucket)
-            if (threadIdx.x == 0) {
-                uint32_t tot = sfill[k], e = k + 1;
-                while (e < nc && tot + sfill[e] <= (uint32_t)JOIN_CAP) tot += sfill[e++];
-                s_nb = e - k;
-                s_total = tot;
+        // plan window starting at bucket k of the chunk into descriptor slot w and start its
+        // copies (thread 0 only); returns the next bucket.  An oversized bucket (a half larger
+        // than BJ_HALF) forms a window of its own with nb = 0 and is joined in global memory.
+        auto plan = [&](uint32_t k, int w) -> uint32_t {
+            WinDesc &d = wd[w];
+            uint32_t nP = 0, nS = 0, nb = 0, bytes = 0;
+            if (sfill[2 * k] > (uint32_t)BJ_HALF || sfill[2 * k + 1] > (uint32_t)BJ_HALF) {
+                d.nb = 0;
+                d.nP = k; // bucket index within the chunk
+                return k + 1;
             }
-            __syncthreads();
-            const uint32_t nbw = s_nb, total = s_total;
-            if (++epoch == 0x10000u) {
-                for (uint32_t t = threadIdx.x; t < JOIN_SLOTS; t += JOIN_THREADS) slot[t] = 0;
-                epoch = 1;
-                __syncthreads();
+            uint32_t e = k;
+            while (e < nc && nb < (uint32_t)BJ_MAXB) {
+                const uint32_t fp = sfill[2 * e], fs = sfill[2 * e + 1];
+                const uint32_t pp = (fp + 1) & ~1u, ps = (fs + 1) & ~1u;
+                if (fp > (uint32_t)BJ_HALF || fs > (uint32_t)BJ_HALF) break;
+                if (nP + pp > (uint32_t)BJ_HALF || nS + ps > (uint32_t)BJ_HALF) break;
+                d.odd[2 * nb] = (fp & 1) ? nP + fp : ~0u;
+                d.odd[2 * nb + 1] = (fs & 1) ? nS + fs : ~0u;
+                if (pp) bytes += pp * 8;
+                if (ps) bytes += ps * 8;
+                nP += pp, nS += ps, ++nb, ++e;
             }
-            if (total > (uint32_t)JOIN_CAP) {
-                const uint64_t bk = c0 + k;
-                oversized_join<W>(a, b.buckets + bk * b.bucket_cap, 0, total, em, nfalse);
+            d.nb = nb, d.nP = nP, d.nS = nS;
+            if (bytes) {
+                // expect all bytes first, then start the copies
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(
+                                 smem_u32(&mbar[w])),
+                             "r"(bytes)
+                             : "memory");
+                uint32_t oP = 0, oS = 0;
+                for (uint32_t q = k; q < e; ++q) {
+                    const uint32_t pp = (sfill[2 * q] + 1) & ~1u, ps = (sfill[2 * q + 1] + 1) & ~1u;
+                    const uint64_t *gb = b.buckets + (c0 + q) * 2 * b.half_cap;
+                    if (pp)
+                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
+                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + oP)),
+                                     "l"(gb), "r"(pp * 8), "r"(smem_u32(&mbar[w]))
+                                     : "memory");
+                    if (ps)
+                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
+                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(sst + w * BJ_HALF + oS)),
+                                     "l"(gb + b.half_cap), "r"(ps * 8), "r"(smem_u32(&mbar[w]))
+                                     : "memory");
+                    oP += pp, oS += ps;
+                }
             } else {
-                // stage the window split by list: prefix entries from the front, suffix
-                // entries from the back (warp-aggregated slots)
-                if (threadIdx.x == 0) s_np = 0, s_ns = 0;
-                __syncthreads();
-                const int lane = threadIdx.x & 31;
-                for (uint32_t q = 0; q < nbw; ++q) {
-                    const uint32_t f = sfill[k + q];
-                    const uint64_t *srcb = b.buckets + (c0 + k + q) * b.bucket_cap;
-                    for (uint32_t t0 = 0; t0 < f; t0 += JOIN_THREADS) {
-                        const uint32_t t = t0 + threadIdx.x;
-                        const bool ok = t < f;
-                        const uint64_t e = ok ? srcb[t] : 0;
-                        const bool isS = ok && ((e >> a.vbits) & 1);
-                        const uint32_t bS = __ballot_sync(0xffffffffu, isS);
-                        const uint32_t bP = __ballot_sync(0xffffffffu, ok && !isS);
-                        uint32_t baseP = 0, baseS = 0;
-                        if (lane == 0) {
-                            if (bP) baseP = atomicAdd(&s_np, (uint32_t)__popc(bP));
-                            if (bS) baseS = atomicAdd(&s_ns, (uint32_t)__popc(bS));
-                        }
-                        baseP = __shfl_sync(0xffffffffu, baseP, 0);
-                        baseS = __shfl_sync(0xffffffffu, baseS, 0);
-                        const uint32_t lt = (1u << lane) - 1;
-                        if (ok) {
-                            if (isS) ent[JOIN_CAP - 1 - (baseS + __popc(bS & lt))] = e;
-                            else ent[baseP + __popc(bP & lt)] = e;
-                        }
-                    }
+                // nothing to copy: complete the phase by a plain arrive
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&mbar[w]))
+                             : "memory");
+            }
+            return e;
+        };
+        __shared__ uint32_t s_k[2];
+        if (threadIdx.x == 0) {
+            fence_proxy_async();
+            s_k[0] = plan(0, 0);
+        }
+        __syncthreads();
+        int w = 0;
+        uint32_t kcur = 0;
+        while (kcur < nc) {
+            const uint32_t knext = s_k[w];
+            // prefetch the next window into the other buffer
+            if (threadIdx.x == 0 && knext < nc) {
+                fence_proxy_async();
+                s_k[w ^ 1] = plan(knext, w ^ 1);
+            }
+            WinDesc &d = wd[w];
+            if (d.nb == 0) {
+                // oversized bucket: no copy was issued, join it in global memory
+                const uint64_t bk = c0 + d.nP;
+                const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
+                oversized_join_split<W>(a, gb, sfill[2 * d.nP], gb + b.half_cap,
+                                        sfill[2 * d.nP + 1], em, nfalse);
+                if (threadIdx.x == 0) s_over = 1;
+            } else {
+                mbar_wait(&mbar[w], (phases >> w) & 1u);
+                phases ^= 1u << w;
+                uint64_t *P = pst + w * BJ_HALF, *S = sst + w * BJ_HALF;
+                for (uint32_t t = threadIdx.x; t < 2 * d.nb; t += JOIN_THREADS) {
+                    const uint32_t o = d.odd[t];
+                    if (o != ~0u) ((t & 1) ? S : P)[o] = ~0ull;
+                }
+                if (++epoch == 0x10000u) {
+                    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+                    epoch = 1;
                 }
                 __syncthreads();
-                const uint32_t nP = s_np, nS = s_ns;
-                hash_join_split<W>(a, ent, nP, JOIN_CAP - nS, nS, slot, next, epoch, em, nfalse);
+                const uint32_t tag = epoch << 16;
+                const uint32_t nP = d.nP, nS = d.nS;
+                for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
+                    const uint64_t e = P[k2];
+                    if (e == ~0ull) continue;
+                    const uint32_t h = (uint32_t)(e >> kshift) & (BJ_SLOTS - 1);
+                    const uint32_t old = atomicExch(&slot[h], tag | k2);
+                    next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
+                }
+                __syncthreads();
+                for (uint32_t k2 = threadIdx.x; k2 < nS; k2 += JOIN_THREADS) {
+                    const uint64_t e = S[k2];
+                    if (e == ~0ull) continue;
+                    const uint32_t sv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
+                    uint32_t sl = (sv >> 16) == epoch ? (sv & 0xFFFFu) : 0xFFFFu;
+                    while (sl != 0xFFFFu) {
+                        const uint64_t p = P[sl];
+                        if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+                        sl = next[sl];
+                    }
+                }
             }
             __syncthreads();
             window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
             __syncthreads();
-            k += nbw;
+            kcur = knext;
+            w ^= 1;
         }
     }
     __syncthreads();
     flush_staged(buf, min(bcount, (uint32_t)JOIN_BUF), a.pairs, a.cap, a.count);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
+    (void)s_over;
 }
 
 lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
@@ -347,8 +462,8 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (args.n_buckets == 0) return LASAGNA_OK;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)(JOIN_CAP + JOIN_BUF) * 8 + (size_t)JOIN_SLOTS * 4 +
-                            (size_t)JOIN_CAP * 2 + (size_t)BJ_FILLS * 4;
+        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
+                            (size_t)BJ_SLOTS * 4 + (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
         LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0;
