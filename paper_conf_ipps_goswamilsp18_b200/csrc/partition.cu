@@ -20,6 +20,8 @@
 //
 // Traffic per entry: 8 B written by the scatter, 8 + 8 B per refine level, 8 B read by the
 // join (T = 16: 32 B, against 48 B for table + 2 LSD passes + join).
+#include <cstdlib>
+
 #include "fingerprint.cuh"
 #include "joinwin.cuh"
 
@@ -27,8 +29,7 @@ namespace lsg {
 
 constexpr int SC_THREADS = 512; // reads per scatter CTA (one per thread)
 constexpr int RF_THREADS = 512;
-constexpr int RF_KPT = 8;
-constexpr int RF_TILE = RF_THREADS * RF_KPT;
+
 
 // exclusive scan of v over the first NB threads (NB a multiple of 32, <= 512); every thread of
 // the block must call it.  wsum: 16 shared words.
@@ -68,7 +69,8 @@ scatter_table_kernel(ScatterArgs a)
 {
     constexpr int NB = SPLIT ? 512 : 256;
     __shared__ uint64_t stage[SC_THREADS * 4];
-    __shared__ uint32_t cnt[NB], lstart[NB], base[NB], wsum[16];
+    __shared__ uint32_t cnt[NB], lstart[NB], wsum[16];
+    __shared__ long long gofs[NB]; // per bin: element offset of stage slot 0's destination, -1 = overflow
     __shared__ uint32_t s_total;
 
     const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
@@ -116,17 +118,23 @@ scatter_table_kernel(ScatterArgs a)
             }
             __syncthreads();
             const uint32_t seg = l - a.l_lo;
-            uint32_t c = 0;
+            uint32_t c = 0, bs = 0;
             if (threadIdx.x < NB) {
                 c = cnt[threadIdx.x];
                 cnt[threadIdx.x] = 0;
-                base[threadIdx.x] =
-                    c ? atomicAdd(&a.fill[(uint64_t)seg * NB + threadIdx.x], c) : 0u;
+                bs = c ? atomicAdd(&a.fill[(uint64_t)seg * NB + threadIdx.x], c) : 0u;
             }
             const uint32_t ex = block_scan<NB>(c, wsum);
             if (threadIdx.x < NB) {
                 lstart[threadIdx.x] = ex;
                 if (threadIdx.x == NB - 1) s_total = ex + c;
+                if ((uint64_t)bs + c > a.cap) {
+                    gofs[threadIdx.x] = -1;
+                    *a.overflow = 1u;
+                } else {
+                    gofs[threadIdx.x] = (long long)(((uint64_t)seg * NB + threadIdx.x) * a.cap + bs) -
+                                        (long long)ex;
+                }
             }
             __syncthreads();
             if (valid) {
@@ -135,13 +143,10 @@ scatter_table_kernel(ScatterArgs a)
             }
             __syncthreads();
             const uint32_t total = s_total;
-            uint64_t *dst = a.out + (uint64_t)seg * NB * a.cap;
             for (uint32_t t = threadIdx.x; t < total; t += SC_THREADS) {
                 const uint64_t key = stage[t];
-                const uint32_t d = bin_of<SPLIT>(key, 56, a.vbits);
-                const uint64_t pos = (uint64_t)base[d] + (t - lstart[d]);
-                if (pos < a.cap) dst[(uint64_t)d * a.cap + pos] = key;
-                else *a.overflow = 1u;
+                const long long go = gofs[bin_of<SPLIT>(key, 56, a.vbits)];
+                if (go >= 0) a.out[go + t] = key;
             }
             // the next round's first barrier orders these reads before stage/lstart reuse
         }
@@ -167,21 +172,22 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
 // One CTA owns one region and streams it: the bulk-copy engine prefetches tile t+1 into the
 // other half of a double buffer while tile t is ranked (shared atomics: order inside a
 // sub-region is irrelevant), staged by digit and written out in digit runs.
-template <bool SPLIT>
-__global__ void __launch_bounds__(RF_THREADS, 2)
+template <bool SPLIT, int RF_KPT>
+__global__ void __launch_bounds__(RF_THREADS, 1)
 refine_kernel(RefineArgs a)
 {
+    constexpr int RF_TILE = RF_THREADS * RF_KPT;
     constexpr int NB = SPLIT ? 512 : 256;
     extern __shared__ __align__(128) uint64_t rsm[];
     uint64_t *inb = rsm;                 // [2][RF_TILE]
     uint64_t *rstage = rsm + 2 * RF_TILE; // [RF_TILE]
     __shared__ __align__(8) unsigned long long mbar[2];
     __shared__ uint32_t cnt[NB], lstart[NB], running[NB], wsum[16];
+    __shared__ long long gofs[NB];
     const uint64_t r = blockIdx.x;
     const uint32_t fill = a.fill_in[r];
     const uint64_t count = min64(fill, a.cap_in);
     const uint64_t *src = a.in + r * a.cap_in;
-    uint64_t *dst = a.out + r * NB * a.cap_out;
     const uint32_t ntiles = (uint32_t)ceil_div(count, RF_TILE);
     if (threadIdx.x < NB) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
@@ -221,7 +227,17 @@ refine_kernel(RefineArgs a)
             cnt[threadIdx.x] = 0;
         }
         const uint32_t ex = block_scan<NB>(c, wsum);
-        if (threadIdx.x < NB) lstart[threadIdx.x] = ex;
+        if (threadIdx.x < NB) {
+            lstart[threadIdx.x] = ex;
+            const uint32_t run = running[threadIdx.x];
+            if ((uint64_t)run + c > a.cap_out) {
+                gofs[threadIdx.x] = -1;
+                *a.overflow = 1u;
+            } else {
+                gofs[threadIdx.x] =
+                    (long long)((r * NB + threadIdx.x) * a.cap_out + run) - (long long)ex;
+            }
+        }
         __syncthreads();
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
@@ -234,10 +250,8 @@ refine_kernel(RefineArgs a)
         __syncthreads();
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
-            const uint32_t d = bin_of<SPLIT>(k, a.dshift, a.vbits);
-            const uint64_t pos = (uint64_t)running[d] + (u - lstart[d]);
-            if (pos < a.cap_out) dst[(uint64_t)d * a.cap_out + pos] = k;
-            else *a.overflow = 1u;
+            const long long go = gofs[bin_of<SPLIT>(k, a.dshift, a.vbits)];
+            if (go >= 0) a.out[go + u] = k;
         }
         __syncthreads();
         if (threadIdx.x < NB) running[threadIdx.x] += c;
@@ -253,8 +267,14 @@ refine_kernel(RefineArgs a)
 lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStream_t s)
 {
     if (n_regions == 0) return LASAGNA_OK;
-    const size_t smem = (size_t)3 * RF_TILE * 8;
-    auto kern = args.split ? refine_kernel<true> : refine_kernel<false>;
+    // tile of 8 keys per thread (2 CTAs per SM) or 16 (LASAGNA_RF_KPT=16, 1 CTA per SM)
+    static const int kpt = [] {
+        const char *e = getenv("LASAGNA_RF_KPT");
+        return (e && atoi(e) == 16) ? 16 : 8;
+    }();
+    const size_t smem = (size_t)3 * RF_THREADS * kpt * 8;
+    auto kern = kpt == 16 ? (args.split ? refine_kernel<true, 16> : refine_kernel<false, 16>)
+                          : (args.split ? refine_kernel<true, 8> : refine_kernel<false, 8>);
     LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     kern<<<(unsigned)n_regions, RF_THREADS, smem, s>>>(args);
     LSG_LAUNCHED("refine_kernel");
