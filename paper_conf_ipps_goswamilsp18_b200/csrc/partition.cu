@@ -267,10 +267,11 @@ refine_kernel(RefineArgs a)
 lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStream_t s)
 {
     if (n_regions == 0) return LASAGNA_OK;
-    // tile of 8 keys per thread (2 CTAs per SM) or 16 (LASAGNA_RF_KPT=16, 1 CTA per SM)
+    // tile of 16 keys per thread (one 512-thread CTA per SM, measured faster than 8 keys at
+    // two CTAs per SM: 22 vs 30 ms at cfg3); LASAGNA_RF_KPT=8 selects the smaller tile
     static const int kpt = [] {
         const char *e = getenv("LASAGNA_RF_KPT");
-        return (e && atoi(e) == 16) ? 16 : 8;
+        return (e && atoi(e) == 8) ? 8 : 16;
     }();
     const size_t smem = (size_t)3 * RF_THREADS * kpt * 8;
     auto kern = kpt == 16 ? (args.split ? refine_kernel<true, 16> : refine_kernel<false, 16>)
