@@ -478,8 +478,186 @@ bucket_join_kernel(BucketJoinArgs b)
     (void)s_over;
 }
 
+// ------------------------------------------------------------------ a5, one warp per bucket
+// When a bucket half fits a warp's shared-memory slice, every warp joins whole buckets on
+// its own (no block barriers): the prefix half is hashed in the warp's slice (chained,
+// epoch-tagged heads: never cleared), the suffix half is streamed straight from global
+// memory and probed, candidates are staged per warp and verified 32 at a time.
+constexpr int WJ_WARPS = 4;
+constexpr int WJ_CAND = 64;
+constexpr int WJ_BATCH = 8; // global loads in flight per lane
+
+template <int W>
+__global__ void __launch_bounds__(WJ_WARPS * 32)
+warp_join_kernel(BucketJoinArgs b, uint32_t pcap, uint32_t nheads)
+{
+    extern __shared__ __align__(16) unsigned char wsm[];
+    const JoinArgs &a = b.j;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 + (size_t)pcap * 2 + WJ_CAND * 8;
+    unsigned char *base = wsm + warp * ((per_warp + 15) & ~(size_t)15);
+    uint64_t *P = reinterpret_cast<uint64_t *>(base);
+    uint32_t *heads = reinterpret_cast<uint32_t *>(base + (size_t)pcap * 8);
+    unsigned short *next = reinterpret_cast<unsigned short *>(base + (size_t)pcap * 8 + nheads * 4);
+    unsigned long long *cand =
+        reinterpret_cast<unsigned long long *>(base + (size_t)pcap * 8 + nheads * 4 + pcap * 2);
+    const uint32_t kshift = a.vbits + 1;
+    const uint64_t vmask = (1ull << a.vbits) - 1;
+    const uint32_t hmask = nheads - 1;
+    const uint32_t lt = (1u << lane) - 1;
+    for (uint32_t t = lane; t < nheads; t += 32) heads[t] = 0;
+    uint32_t ncand = 0, epoch = 0;
+    unsigned long long nfalse = 0;
+
+    // verify the first 32 staged candidates (lane i takes cand[i]) and append the accepted
+    // ones to the global pool; ncand is warp-uniform
+    auto drain32 = [&](uint32_t k) {
+        __syncwarp();
+        bool ok = false;
+        unsigned long long rec = 0;
+        if ((uint32_t)lane < k) {
+            rec = cand[lane];
+            const uint32_t u = (uint32_t)(rec >> 32), bb = (uint32_t)rec;
+            ok = verify_overlap<W>(a.packed, a.stride, a.L, u, bb ^ 1u, a.l);
+            nfalse += ok ? 0 : 1;
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+        unsigned long long gb = 0;
+        if (lane == 0 && bal) gb = atomicAdd(a.count, (unsigned long long)__popc(bal));
+        gb = __shfl_sync(0xffffffffu, gb, 0);
+        if (ok) {
+            const unsigned long long pos = gb + __popc(bal & lt);
+            if (pos < a.cap) a.pairs[pos] = rec;
+        }
+        __syncwarp();
+        // move the remainder down
+        if ((uint32_t)lane + 32 < ncand) cand[lane] = cand[lane + 32];
+        __syncwarp();
+    };
+
+    const uint64_t total_warps = (uint64_t)gridDim.x * WJ_WARPS;
+    for (uint64_t bk = (uint64_t)blockIdx.x * WJ_WARPS + warp; bk < b.n_buckets; bk += total_warps) {
+        uint32_t fP = 0, fS = 0;
+        if (lane == 0) {
+            fP = b.fills[2 * bk];
+            fS = b.fills[2 * bk + 1];
+            if (fP > b.half_cap || fS > b.half_cap) *b.overflow = 1u;
+        }
+        fP = (uint32_t)min64(__shfl_sync(0xffffffffu, fP, 0), b.half_cap);
+        fS = (uint32_t)min64(__shfl_sync(0xffffffffu, fS, 0), b.half_cap);
+        if (fP == 0 || fS == 0) continue;
+        if (++epoch == 0x10000u) {
+            for (uint32_t t = lane; t < nheads; t += 32) heads[t] = 0;
+            epoch = 1;
+            __syncwarp();
+        }
+        const uint32_t tag = epoch << 16;
+        const uint64_t *gP = b.buckets + bk * 2 * b.half_cap;
+        const uint64_t *gS = gP + b.half_cap;
+        // stage + hash the prefix half (8 loads per lane in flight before the inserts)
+        for (uint32_t t0 = 0; t0 < fP; t0 += 32 * WJ_BATCH) {
+            uint64_t ev[WJ_BATCH];
+#pragma unroll
+            for (int q = 0; q < WJ_BATCH; ++q) {
+                const uint32_t t = t0 + q * 32 + lane;
+                ev[q] = t < fP ? gP[t] : 0;
+            }
+#pragma unroll
+            for (int q = 0; q < WJ_BATCH; ++q) {
+                const uint32_t t = t0 + q * 32 + lane;
+                if (t < fP) {
+                    P[t] = ev[q];
+                    const uint32_t old =
+                        atomicExch(&heads[(uint32_t)(ev[q] >> kshift) & hmask], tag | t);
+                    next[t] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
+                }
+            }
+        }
+        __syncwarp();
+        // probe with the suffix half, straight from global memory
+        uint64_t sv[WJ_BATCH];
+        for (uint32_t t0 = 0; t0 < fS; t0 += 32) {
+            const uint32_t qq = (t0 / 32) % WJ_BATCH;
+            if (qq == 0) {
+#pragma unroll
+                for (int q = 0; q < WJ_BATCH; ++q) {
+                    const uint32_t t = t0 + q * 32 + lane;
+                    sv[q] = t < fS ? gS[t] : 0;
+                }
+            }
+            const uint32_t t = t0 + lane;
+            uint64_t e = 0;
+#pragma unroll
+            for (int q = 0; q < WJ_BATCH; ++q)
+                if ((uint32_t)q == qq) e = sv[q];
+            uint32_t sl = 0xFFFFu;
+            if (t < fS) {
+                const uint32_t hv = heads[(uint32_t)(e >> kshift) & hmask];
+                sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
+            }
+            while (__any_sync(0xffffffffu, sl != 0xFFFFu)) {
+                bool c = false;
+                unsigned long long rec = 0;
+                if (sl != 0xFFFFu) {
+                    const uint64_t p = P[sl];
+                    if (((p ^ e) >> kshift) == 0) {
+                        const uint32_t u = (uint32_t)(e & vmask), v = (uint32_t)(p & vmask);
+                        const uint32_t bb = v ^ 1u;
+                        if ((u >> 1) != (v >> 1) && u < bb) { // R9; each pair once
+                            c = true;
+                            rec = ((unsigned long long)u << 32) | bb;
+                        }
+                    }
+                    sl = next[sl];
+                }
+                const uint32_t bal = __ballot_sync(0xffffffffu, c);
+                if (bal) {
+                    if (c) cand[ncand + __popc(bal & lt)] = rec;
+                    ncand += __popc(bal);
+                    if (ncand >= 32) {
+                        drain32(32);
+                        ncand -= 32;
+                    }
+                }
+            }
+        }
+        __syncwarp();
+    }
+    if (ncand) {
+        drain32(ncand);
+        ncand = 0;
+    }
+    for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
+    if (lane == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
+}
+
 lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
 {
+    if (args.n_buckets == 0) return LASAGNA_OK;
+    static const bool block_join = getenv("LASAGNA_BLOCK_JOIN") != nullptr;
+    const uint32_t pcap = (uint32_t)((args.half_cap + 1) & ~1ull);
+    if (!block_join && pcap <= 2048) {
+        uint32_t nheads = 256; // ~1 prefix entry per chain head
+        while (nheads * 2 <= pcap) nheads <<= 1;
+        const size_t per_warp =
+            ((size_t)pcap * 8 + (size_t)nheads * 4 + (size_t)pcap * 2 + WJ_CAND * 8 + 15) & ~(size_t)15;
+        const size_t smem = per_warp * WJ_WARPS;
+        return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
+            constexpr int W = decltype(wc)::value;
+            LSG_CUDA(cudaFuncSetAttribute(warp_join_kernel<W>,
+                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            int per_sm = 0;
+            LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, warp_join_kernel<W>,
+                                                                   WJ_WARPS * 32, smem));
+            per_sm = std::max(per_sm, 1);
+            const uint64_t blocks = std::max<uint64_t>(
+                1, std::min<uint64_t>((uint64_t)num_sms() * per_sm,
+                                      ceil_div(args.n_buckets, WJ_WARPS)));
+            warp_join_kernel<W><<<(unsigned)blocks, WJ_WARPS * 32, smem, s>>>(args, pcap, nheads);
+            LSG_LAUNCHED("warp_join_kernel");
+            return LASAGNA_OK;
+        });
+    }
     if (args.n_buckets == 0) return LASAGNA_OK;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
