@@ -494,13 +494,14 @@ warp_join_kernel(BucketJoinArgs b, uint32_t pcap, uint32_t nheads)
     extern __shared__ __align__(16) unsigned char wsm[];
     const JoinArgs &a = b.j;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 + (size_t)pcap * 2 + WJ_CAND * 8;
-    unsigned char *base = wsm + warp * ((per_warp + 15) & ~(size_t)15);
+    const size_t next_b = ((size_t)pcap * 2 + 15) & ~(size_t)15;
+    const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 + next_b + WJ_CAND * 8;
+    unsigned char *base = wsm + warp * per_warp;
     uint64_t *P = reinterpret_cast<uint64_t *>(base);
     uint32_t *heads = reinterpret_cast<uint32_t *>(base + (size_t)pcap * 8);
     unsigned short *next = reinterpret_cast<unsigned short *>(base + (size_t)pcap * 8 + nheads * 4);
     unsigned long long *cand =
-        reinterpret_cast<unsigned long long *>(base + (size_t)pcap * 8 + nheads * 4 + pcap * 2);
+        reinterpret_cast<unsigned long long *>(base + (size_t)pcap * 8 + nheads * 4 + next_b);
     const uint32_t kshift = a.vbits + 1;
     const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint32_t hmask = nheads - 1;
@@ -639,8 +640,8 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (!block_join && pcap <= 2048) {
         uint32_t nheads = 256; // ~1 prefix entry per chain head
         while (nheads * 2 <= pcap) nheads <<= 1;
-        const size_t per_warp =
-            ((size_t)pcap * 8 + (size_t)nheads * 4 + (size_t)pcap * 2 + WJ_CAND * 8 + 15) & ~(size_t)15;
+        const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 +
+                                (((size_t)pcap * 2 + 15) & ~(size_t)15) + WJ_CAND * 8;
         const size_t smem = per_warp * WJ_WARPS;
         return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
             constexpr int W = decltype(wc)::value;
