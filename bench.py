@@ -138,14 +138,25 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict) ->
     n_len = L - l_min
     G = stats["lengths_per_pass"]
     verify = 64.0 * (stats["n_pairs"] + stats["fp_false_matches"]) / max(1, n_len)
-    per = {
-        # one onesweep pass over a group: every key read once and written once
-        "onesweep_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
-        # one join launch (one length): the sorted table streamed once + verification loads
-        "join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
-        # table: 4 keys (32 B) written per read per length, the packed read loaded once
-        "table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
-    }
+    bucketed = bool(stats.get("bucketed", 1))
+    if bucketed:
+        per = {
+            # level-1 partition fused with the fingerprints: every key written once
+            "scatter_table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
+            # level-2 partition: every key read once and written once
+            "refine_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
+            # one join launch (one length): every key read once + verification loads
+            "bucket_join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
+        }
+    else:
+        per = {
+            # one onesweep pass over a group: every key read once and written once
+            "onesweep_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
+            # one join launch (one length): the sorted table streamed once + verification loads
+            "join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
+            # table: 4 keys (32 B) written per read per length, the packed read loaded once
+            "table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
+        }
     name = max(per, key=lambda k: per[k][0])
     ms, launches, bytes_per_launch = per[name]
     launches = max(1, launches)
@@ -265,7 +276,7 @@ def main() -> None:
     # ---- device-resident timed region
     sampler = ClockSampler(_bus_id(torch, 0))
     agg = {k: 0.0 for k in ["ms_table", "ms_sort", "ms_search", "ms_greedy"]}
-    cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes"]}
+    cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes"]}  # summed over steps
     sampler.start()
     torch.cuda.synchronize()
     launches0 = lz.kernel_launches()

@@ -573,6 +573,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     memset(&st, 0, sizeof st);
     st.lengths_per_pass = G;
     st.key_sort_bits = g.T;
+    st.bucketed = r.bucketed ? 1u : 0u;
     PhaseTimer tm;
     tm.on = stats != nullptr;
     tm.s = s;

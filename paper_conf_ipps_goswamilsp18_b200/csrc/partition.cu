@@ -635,9 +635,11 @@ warp_join_kernel(BucketJoinArgs b, uint32_t pcap, uint32_t nheads)
 lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
 {
     if (args.n_buckets == 0) return LASAGNA_OK;
-    static const bool block_join = getenv("LASAGNA_BLOCK_JOIN") != nullptr;
+    // the block join (windows of whole buckets, bulk-copy staged) measured faster than the
+    // warp-per-bucket join at cfg3 (38 vs 50 ms); LASAGNA_WARP_JOIN=1 selects the latter
+    static const bool warp_join = getenv("LASAGNA_WARP_JOIN") != nullptr;
     const uint32_t pcap = (uint32_t)((args.half_cap + 1) & ~1ull);
-    if (!block_join && pcap <= 2048) {
+    if (warp_join && pcap <= 2048) {
         uint32_t nheads = 256; // ~1 prefix entry per chain head
         while (nheads * 2 <= pcap) nheads <<= 1;
         const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 +

@@ -31,6 +31,7 @@ class _Stats(ctypes.Structure):
                 ("rounds_max", ctypes.c_uint32), ("passes", ctypes.c_uint32),
                 ("lengths_per_pass", ctypes.c_uint32), ("key_sort_bits", ctypes.c_uint32),
                 ("sort_launches", ctypes.c_uint32), ("search_launches", ctypes.c_uint32),
+                ("bucketed", ctypes.c_uint32),
                 ("ms_table", ctypes.c_float), ("ms_sort", ctypes.c_float),
                 ("ms_search", ctypes.c_float),
                 ("ms_greedy", ctypes.c_float)]
