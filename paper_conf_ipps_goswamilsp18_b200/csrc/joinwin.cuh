@@ -167,23 +167,36 @@ __device__ __forceinline__ void oversized_join(const JoinArgs &a, const uint64_t
     }
 }
 
-// after a window: verify its staged candidates; flush the staging buffer when half full.
-// Must be called by all threads after a __syncthreads().
+// after a window (called by all threads after a __syncthreads()): once at least one candidate
+// per thread is staged, verify them all in parallel (the long verify path runs with full
+// warps) and flush the accepted ones.  Cheaper windows just leave the buffer as it is.
 template <int W>
 __device__ __forceinline__ void window_epilogue(const JoinArgs &a, unsigned long long *buf,
                                                 uint32_t *bcount, uint32_t *vdone,
                                                 unsigned long long &nfalse)
 {
     const uint32_t to = min(*bcount, (uint32_t)JOIN_BUF);
-    verify_staged<W>(a, buf, *vdone, to, nfalse);
-    __syncthreads();
-    if (to >= JOIN_BUF / 2) {
+    if (to >= (uint32_t)JOIN_THREADS) {
+        verify_staged<W>(a, buf, 0, to, nfalse);
+        __syncthreads();
         flush_staged(buf, to, a.pairs, a.cap, a.count);
         __syncthreads();
-        if (threadIdx.x == 0) *bcount = 0, *vdone = 0;
-    } else if (threadIdx.x == 0) {
-        *vdone = to;
+        if (threadIdx.x == 0) *bcount = 0;
+        __syncthreads();
     }
+    (void)vdone;
+}
+
+// end of a join kernel: verify and flush whatever is still staged
+template <int W>
+__device__ __forceinline__ void final_flush(const JoinArgs &a, unsigned long long *buf,
+                                            uint32_t *bcount, unsigned long long &nfalse)
+{
+    __syncthreads();
+    const uint32_t to = min(*bcount, (uint32_t)JOIN_BUF);
+    verify_staged<W>(a, buf, 0, to, nfalse);
+    __syncthreads();
+    flush_staged(buf, to, a.pairs, a.cap, a.count);
 }
 
 } // namespace lsg

@@ -464,15 +464,13 @@ bucket_join_kernel(BucketJoinArgs b)
                     }
                 }
             }
-            __syncthreads();
+            __syncthreads(); // window w done: its buffer may be refilled
             window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
-            __syncthreads();
             kcur = knext;
             w ^= 1;
         }
     }
-    __syncthreads();
-    flush_staged(buf, min(bcount, (uint32_t)JOIN_BUF), a.pairs, a.cap, a.count);
+    final_flush<W>(a, buf, &bcount, nfalse);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
     (void)s_over;

@@ -136,7 +136,7 @@ join_kernel(JoinArgs a)
         __syncthreads();
         t0 = t1;
     }
-    flush_staged(buf, min(bcount, (uint32_t)JOIN_BUF), a.pairs, a.cap, a.count);
+    final_flush<W>(a, buf, &bcount, nfalse);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
