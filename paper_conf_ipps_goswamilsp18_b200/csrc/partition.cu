@@ -153,16 +153,126 @@ scatter_table_kernel(ScatterArgs a)
     }
 }
 
+// Two lengths per partition round (non-split level 1): half the barriers, half the scans and
+// reservation atomics of the one-length round; bins k * 256 + digit for the round's k-th length.
+template <int W>
+__global__ void __launch_bounds__(SC_THREADS, 2)
+scatter_table2_kernel(ScatterArgs a)
+{
+    constexpr int NB = 256, NB2 = 512;
+    __shared__ uint64_t stage[SC_THREADS * 8];
+    __shared__ uint32_t cnt[NB2], lstart[NB2], wsum[16];
+    __shared__ long long gofs[NB2];
+    __shared__ uint32_t s_total;
+
+    const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
+    const bool valid = i < a.n;
+    uint64_t x[W], y[W];
+    if (valid) {
+        load_read<W>(a.packed, a.stride, i, x);
+        rc_words<W>(x, a.L, y);
+    } else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
+    }
+    cnt[threadIdx.x] = 0; // NB2 == SC_THREADS
+    __syncthreads();
+    const uint64_t keep = ~((2ull << a.vbits) - 1);
+    const uint64_t tagS = 1ull << a.vbits;
+    const uint64_t v0 = 2 * (a.read_offset + i);
+    FpStreams st;
+    st.init();
+    uint64_t k0[4], k1[4];
+    uint32_t r0[4], r1[4];
+    uint32_t kc = 0, lfirst = 0; // keys buffered this round (block-uniform)
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+        uint64_t xa = x[w], yb = y[w];
+        const uint32_t kb = 32u * w;
+        if (kb >= a.l_hi) break;
+        const uint32_t kn = min(32u, a.l_hi - kb);
+        for (uint32_t j = 0; j < kn; ++j) {
+            st.step((uint32_t)(xa & 3u), (uint32_t)(yb & 3u), kb + j);
+            xa >>= 2;
+            yb >>= 2;
+            const uint32_t l = kb + j + 1;
+            if (l < a.l_lo) continue;
+            if (kc == 0) {
+                lfirst = l;
+                if (valid) {
+                    k0[0] = (mix(exact61(st.P0)) & keep) | v0;
+                    k0[1] = (mix(exact61(st.S0)) & keep) | tagS | v0;
+                    k0[2] = (mix(exact61(st.P1)) & keep) | (v0 + 1);
+                    k0[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) r0[q] = atomicAdd(&cnt[(uint32_t)(k0[q] >> 56)], 1u);
+                }
+            } else {
+                if (valid) {
+                    k1[0] = (mix(exact61(st.P0)) & keep) | v0;
+                    k1[1] = (mix(exact61(st.S0)) & keep) | tagS | v0;
+                    k1[2] = (mix(exact61(st.P1)) & keep) | (v0 + 1);
+                    k1[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        r1[q] = atomicAdd(&cnt[NB + (uint32_t)(k1[q] >> 56)], 1u);
+                }
+            }
+            ++kc;
+            if (kc < 2 && l < a.l_hi) continue;
+            // ---- partition round for lengths lfirst .. lfirst + kc - 1
+            __syncthreads();
+            const uint32_t t = threadIdx.x; // one bin per thread
+            const uint32_t c = cnt[t];
+            cnt[t] = 0;
+            const uint32_t seg = lfirst - a.l_lo + t / NB;
+            const uint32_t d = t % NB;
+            const uint32_t bs =
+                (c && (t / NB) < kc) ? atomicAdd(&a.fill[(uint64_t)seg * NB + d], c) : 0u;
+            const uint32_t ex = block_scan<NB2>(c, wsum);
+            lstart[t] = ex;
+            if (t == NB2 - 1) s_total = ex + c;
+            if ((uint64_t)bs + c > a.cap) {
+                gofs[t] = -1;
+                *a.overflow = 1u;
+            } else {
+                gofs[t] = (long long)(((uint64_t)seg * NB + d) * a.cap + bs) - (long long)ex;
+            }
+            __syncthreads();
+            if (valid) {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) stage[lstart[(uint32_t)(k0[q] >> 56)] + r0[q]] = k0[q];
+                if (kc == 2) {
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        stage[lstart[NB + (uint32_t)(k1[q] >> 56)] + r1[q]] = k1[q];
+                }
+            }
+            __syncthreads();
+            const uint32_t total = s_total, mid = lstart[NB];
+            for (uint32_t u = threadIdx.x; u < total; u += SC_THREADS) {
+                const uint64_t key = stage[u];
+                const long long go = gofs[(u >= mid ? NB : 0) + (uint32_t)(key >> 56)];
+                if (go >= 0) a.out[go + u] = key;
+            }
+            kc = 0;
+        }
+    }
+}
+
 lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
 {
     if (args.n == 0) return LASAGNA_OK;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
         const uint64_t blocks = ceil_div(args.n, SC_THREADS);
+        static const bool one_length = getenv("LASAGNA_SCATTER_LPR1") != nullptr;
         if (args.split)
             scatter_table_kernel<W, true><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
-        else
+        else if (one_length)
             scatter_table_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
+        else
+            scatter_table2_kernel<W><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
         LSG_LAUNCHED("scatter_table_kernel");
         return LASAGNA_OK;
     });
