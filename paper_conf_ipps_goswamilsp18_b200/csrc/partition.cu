@@ -398,14 +398,17 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 // (cp.async.bulk) stages window w+1 while window w is joined.  A half's copy is rounded up
 // to 16 bytes, so an odd fill drags one stale slot along: it is overwritten with a sentinel
 // key (~0: tag bits set, never equal to a real key of the other list) after the copy lands.
-constexpr int BJ_HALF = 2048;   // staged prefix (and suffix) entries per window
+constexpr int BJ_HALF = 3072;   // staged prefix entries per window
 constexpr int BJ_MAXB = 64;     // buckets per window
 constexpr int BJ_FILLS = 1024;  // buckets whose fills are staged at once
 constexpr int BJ_SLOTS = 4096;
+constexpr int BJ_SBATCH = 4;    // suffix entries per thread loaded before probing
 
 struct WinDesc {
-    uint32_t nb, nP, nS;             // buckets, staged prefix / suffix slots (padded)
-    uint32_t odd[2 * BJ_MAXB];       // staging offsets of the sentinel slots (or ~0)
+    uint32_t nb, nP;                 // buckets, staged prefix slots (padded)
+    uint32_t first;                  // first bucket (index within the chunk)
+    uint32_t oP[BJ_MAXB + 1];        // staging offset of each bucket's prefix half
+    uint32_t odd[BJ_MAXB];           // sentinel slot of an odd prefix fill (or ~0)
 };
 
 template <int W>
@@ -424,20 +427,26 @@ __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const ui
     }
 }
 
+// Buckets are stored split: prefix entries [b][0][0..fillP), suffix entries [b][1][0..fillS).
+// A window = consecutive whole buckets whose prefix halves fit the staging buffer; the copy
+// engine (cp.async.bulk) stages the prefix halves of window w+1 while window w is joined:
+// its prefix halves are hashed in shared memory and its suffix halves are streamed from global
+// memory (a few loads in flight per thread) and probed.  A prefix copy is rounded up to 16
+// bytes, so an odd fill drags one stale slot along: it is overwritten with a sentinel key
+// (~0, never equal to a real suffix key: the tag bits differ) after the copy lands.
 template <int W>
 __global__ void __launch_bounds__(JOIN_THREADS, 2)
 bucket_join_kernel(BucketJoinArgs b)
 {
     extern __shared__ __align__(128) unsigned char jsm[];
     uint64_t *pst = reinterpret_cast<uint64_t *>(jsm);                    // [2][BJ_HALF]
-    uint64_t *sst = pst + 2 * BJ_HALF;                                   // [2][BJ_HALF]
-    unsigned long long *buf = reinterpret_cast<unsigned long long *>(sst + 2 * BJ_HALF); // [BUF]
+    unsigned long long *buf = reinterpret_cast<unsigned long long *>(pst + 2 * BJ_HALF); // [BUF]
     uint32_t *slot = reinterpret_cast<uint32_t *>(buf + JOIN_BUF);       // [BJ_SLOTS]
     unsigned short *next = reinterpret_cast<unsigned short *>(slot + BJ_SLOTS); // [BJ_HALF]
     uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
     __shared__ WinDesc wd[2];
     __shared__ __align__(8) unsigned long long mbar[2];
-    __shared__ uint32_t bcount, vdone, s_over;
+    __shared__ uint32_t bcount, vdone, s_k[2];
     const JoinArgs &a = b.j;
     const uint64_t nbk = b.n_buckets;
     const uint64_t b0 = nbk * blockIdx.x / gridDim.x, b1 = nbk * (blockIdx.x + 1) / gridDim.x;
@@ -463,60 +472,47 @@ bucket_join_kernel(BucketJoinArgs b)
             sfill[t] = (uint32_t)min64(f, b.half_cap);
         }
         __syncthreads();
-        // plan window starting at bucket k of the chunk into descriptor slot w and start its
-        // copies (thread 0 only); returns the next bucket.  An oversized bucket (a half larger
-        // than BJ_HALF) forms a window of its own with nb = 0 and is joined in global memory.
+        // plan the window starting at chunk bucket k into descriptor w and start its copies
+        // (thread 0).  A bucket whose prefix half exceeds the staging buffer is a window of
+        // its own with nb = 0, joined in global memory.
         auto plan = [&](uint32_t k, int w) -> uint32_t {
             WinDesc &d = wd[w];
-            uint32_t nP = 0, nS = 0, nb = 0, bytes = 0;
-            if (sfill[2 * k] > (uint32_t)BJ_HALF || sfill[2 * k + 1] > (uint32_t)BJ_HALF) {
+            d.first = k;
+            if (sfill[2 * k] > (uint32_t)BJ_HALF) {
                 d.nb = 0;
-                d.nP = k; // bucket index within the chunk
                 return k + 1;
             }
-            uint32_t e = k;
+            uint32_t nP = 0, nb = 0, e = k;
             while (e < nc && nb < (uint32_t)BJ_MAXB) {
-                const uint32_t fp = sfill[2 * e], fs = sfill[2 * e + 1];
-                const uint32_t pp = (fp + 1) & ~1u, ps = (fs + 1) & ~1u;
-                if (fp > (uint32_t)BJ_HALF || fs > (uint32_t)BJ_HALF) break;
-                if (nP + pp > (uint32_t)BJ_HALF || nS + ps > (uint32_t)BJ_HALF) break;
-                d.odd[2 * nb] = (fp & 1) ? nP + fp : ~0u;
-                d.odd[2 * nb + 1] = (fs & 1) ? nS + fs : ~0u;
-                if (pp) bytes += pp * 8;
-                if (ps) bytes += ps * 8;
-                nP += pp, nS += ps, ++nb, ++e;
+                const uint32_t fp = sfill[2 * e];
+                const uint32_t pp = (fp + 1) & ~1u;
+                if (nP + pp > (uint32_t)BJ_HALF) break;
+                d.oP[nb] = nP;
+                d.odd[nb] = (fp & 1) ? nP + fp : ~0u;
+                nP += pp, ++nb, ++e;
             }
-            d.nb = nb, d.nP = nP, d.nS = nS;
-            if (bytes) {
-                // expect all bytes first, then start the copies
+            d.oP[nb] = nP;
+            d.nb = nb, d.nP = nP;
+            if (nP) {
                 asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(
                                  smem_u32(&mbar[w])),
-                             "r"(bytes)
+                             "r"(nP * 8)
                              : "memory");
-                uint32_t oP = 0, oS = 0;
-                for (uint32_t q = k; q < e; ++q) {
-                    const uint32_t pp = (sfill[2 * q] + 1) & ~1u, ps = (sfill[2 * q + 1] + 1) & ~1u;
-                    const uint64_t *gb = b.buckets + (c0 + q) * 2 * b.half_cap;
+                for (uint32_t q = 0; q < nb; ++q) {
+                    const uint32_t pp = d.oP[q + 1] - d.oP[q];
                     if (pp)
                         asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
-                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + oP)),
-                                     "l"(gb), "r"(pp * 8), "r"(smem_u32(&mbar[w]))
+                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + d.oP[q])),
+                                     "l"(b.buckets + (c0 + k + q) * 2 * b.half_cap), "r"(pp * 8),
+                                     "r"(smem_u32(&mbar[w]))
                                      : "memory");
-                    if (ps)
-                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
-                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(sst + w * BJ_HALF + oS)),
-                                     "l"(gb + b.half_cap), "r"(ps * 8), "r"(smem_u32(&mbar[w]))
-                                     : "memory");
-                    oP += pp, oS += ps;
                 }
             } else {
-                // nothing to copy: complete the phase by a plain arrive
                 asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&mbar[w]))
                              : "memory");
             }
             return e;
         };
-        __shared__ uint32_t s_k[2];
         if (threadIdx.x == 0) {
             fence_proxy_async();
             s_k[0] = plan(0, 0);
@@ -526,34 +522,29 @@ bucket_join_kernel(BucketJoinArgs b)
         uint32_t kcur = 0;
         while (kcur < nc) {
             const uint32_t knext = s_k[w];
-            // prefetch the next window into the other buffer
             if (threadIdx.x == 0 && knext < nc) {
                 fence_proxy_async();
                 s_k[w ^ 1] = plan(knext, w ^ 1);
             }
-            WinDesc &d = wd[w];
+            const WinDesc &d = wd[w];
             if (d.nb == 0) {
-                // oversized bucket: no copy was issued, join it in global memory
-                const uint64_t bk = c0 + d.nP;
+                const uint64_t bk = c0 + d.first;
                 const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
-                oversized_join_split<W>(a, gb, sfill[2 * d.nP], gb + b.half_cap,
-                                        sfill[2 * d.nP + 1], em, nfalse);
-                if (threadIdx.x == 0) s_over = 1;
+                oversized_join_split<W>(a, gb, sfill[2 * d.first], gb + b.half_cap,
+                                        sfill[2 * d.first + 1], em, nfalse);
             } else {
                 mbar_wait(&mbar[w], (phases >> w) & 1u);
                 phases ^= 1u << w;
-                uint64_t *P = pst + w * BJ_HALF, *S = sst + w * BJ_HALF;
-                for (uint32_t t = threadIdx.x; t < 2 * d.nb; t += JOIN_THREADS) {
-                    const uint32_t o = d.odd[t];
-                    if (o != ~0u) ((t & 1) ? S : P)[o] = ~0ull;
-                }
+                uint64_t *P = pst + w * BJ_HALF;
+                for (uint32_t t = threadIdx.x; t < d.nb; t += JOIN_THREADS)
+                    if (d.odd[t] != ~0u) P[d.odd[t]] = ~0ull;
                 if (++epoch == 0x10000u) {
                     for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
                     epoch = 1;
                 }
                 __syncthreads();
                 const uint32_t tag = epoch << 16;
-                const uint32_t nP = d.nP, nS = d.nS;
+                const uint32_t nP = d.nP;
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
                     const uint64_t e = P[k2];
                     if (e == ~0ull) continue;
@@ -562,15 +553,29 @@ bucket_join_kernel(BucketJoinArgs b)
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
                 __syncthreads();
-                for (uint32_t k2 = threadIdx.x; k2 < nS; k2 += JOIN_THREADS) {
-                    const uint64_t e = S[k2];
-                    if (e == ~0ull) continue;
-                    const uint32_t sv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
-                    uint32_t sl = (sv >> 16) == epoch ? (sv & 0xFFFFu) : 0xFFFFu;
-                    while (sl != 0xFFFFu) {
-                        const uint64_t p = P[sl];
-                        if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-                        sl = next[sl];
+                // probe: the suffix halves of the window's buckets, straight from global memory
+                for (uint32_t q = 0; q < d.nb; ++q) {
+                    const uint32_t fs = sfill[2 * (d.first + q) + 1];
+                    const uint64_t *gS = b.buckets + (c0 + d.first + q) * 2 * b.half_cap + b.half_cap;
+                    for (uint32_t t0 = 0; t0 < fs; t0 += JOIN_THREADS * BJ_SBATCH) {
+                        uint64_t sv[BJ_SBATCH];
+#pragma unroll
+                        for (int r = 0; r < BJ_SBATCH; ++r) {
+                            const uint32_t t = t0 + r * JOIN_THREADS + threadIdx.x;
+                            sv[r] = t < fs ? gS[t] : 0ull;
+                        }
+#pragma unroll
+                        for (int r = 0; r < BJ_SBATCH; ++r) {
+                            if (t0 + r * JOIN_THREADS + threadIdx.x >= fs) continue;
+                            const uint64_t e = sv[r];
+                            const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
+                            uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
+                            while (sl != 0xFFFFu) {
+                                const uint64_t p = P[sl];
+                                if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+                                sl = next[sl];
+                            }
+                        }
                     }
                 }
             }
@@ -583,7 +588,6 @@ bucket_join_kernel(BucketJoinArgs b)
     final_flush<W>(a, buf, &bcount, nfalse);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
-    (void)s_over;
 }
 
 // ------------------------------------------------------------------ a5, one warp per bucket
@@ -772,7 +776,7 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (args.n_buckets == 0) return LASAGNA_OK;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
+        const size_t smem = (size_t)2 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
                             (size_t)BJ_SLOTS * 4 + (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
         LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
