@@ -145,6 +145,21 @@ LASAGNA_API lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t
                                     size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
                                     lasagna_stats *stats, void *stream);
 
+/* a1-a7 from the ASCII reads: as lasagna_greedy_graph, with the 2-bit staging (a1) fused into
+ * the first table pass when the fast path runs (the packed rows are written to packed_out,
+ * device u64 [n][lasagna_words_per_read(L)], for the verification step), so the read-in of
+ * host reads over PCIe overlaps the fingerprint computation.
+ *   ascii      n*L bytes, device memory or PAGE-LOCKED host memory (read in place)
+ *   first_bad  device u64: UINT64_MAX, or the smallest index of a read holding a byte outside
+ *              ACGTacgt -> the call returns LASAGNA_EINVAL (outputs unspecified).
+ * Synchronises `stream` once at the end. */
+LASAGNA_API lasagna_status lasagna_greedy_graph_ascii(const char *ascii, uint64_t n, uint32_t L,
+                                                      uint32_t l_min, uint32_t lengths_per_pass,
+                                                      void *workspace, size_t *workspace_bytes,
+                                                      uint64_t *packed_out, uint64_t *first_bad,
+                                                      uint32_t *succ, uint8_t *olen,
+                                                      lasagna_stats *stats, void *stream);
+
 /* Planner for the semi-streaming driver (a8): the largest
  * lengths_per_pass whose workspace fits `budget_bytes`, and that workspace size.  Returns
  * LASAGNA_ENOSPC when even one length per pass does not fit (*workspace_bytes = minimum). */

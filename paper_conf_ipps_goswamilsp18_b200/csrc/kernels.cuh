@@ -72,6 +72,11 @@ struct ScatterArgs {
     uint64_t cap;
     uint32_t *overflow;
     bool split;         // final level: prefix and suffix entries in separate halves
+    // a1 fused in (optional): read ASCII (device or page-locked host memory) instead of
+    // `packed`, write the packed rows to packed_out and report bad reads in first_bad
+    const unsigned char *ascii;
+    uint64_t *packed_out;
+    unsigned long long *first_bad;
 };
 lasagna_status launch_scatter_table(const ScatterArgs &a, cudaStream_t s);
 struct RefineArgs {

@@ -193,6 +193,9 @@ struct Run {
     uint64_t *tab[2];
     uint32_t *hist;
     bool bucketed;              // partition.cu path (else exact LSD sort + contiguous join)
+    const unsigned char *ascii = nullptr; // a1 still to do: the first group's scatter packs it
+    uint64_t *packed_out = nullptr;
+    unsigned long long *first_bad = nullptr;
     uint32_t *fill1, *fill2;
     unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
@@ -284,6 +287,10 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.split = g.P == 1; // one level: the level-1 regions are the (split) buckets
     sa.cap = sa.split ? g.half1 : g.cap1;
     sa.overflow = ovf;
+    sa.ascii = r.ascii; // fused a1 (first group only)
+    sa.packed_out = r.packed_out;
+    sa.first_bad = r.first_bad;
+    r.ascii = nullptr;
     lasagna_status rc;
     if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
     if ((rc = launch_scatter_table(sa, r.s)) != LASAGNA_OK) return rc;
@@ -419,6 +426,30 @@ uint64_t lasagna_kernel_launches(void) { return launch_count(); }
 
 uint32_t lasagna_words_per_read(uint32_t L) { return stride_for(L); }
 
+// Device address of an ASCII read buffer: device memory, or page-locked host memory mapped
+// into the device address space (read in place over PCIe).  Pageable memory is rejected.
+static lasagna_status resolve_ascii(const char *ascii, const char **dev)
+{
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, ascii) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("ascii: not a CUDA-visible pointer");
+        return LASAGNA_EINVAL;
+    }
+    *dev = ascii;
+    if (at.type == cudaMemoryTypeHost) {
+        if (!at.devicePointer) {
+            set_error("ascii: page-locked host memory is not mapped into the device");
+            return LASAGNA_EINVAL;
+        }
+        *dev = (const char *)at.devicePointer;
+    } else if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+        set_error("ascii: pageable host memory; pass device or page-locked host memory");
+        return LASAGNA_EINVAL;
+    }
+    return LASAGNA_OK;
+}
+
 lasagna_status lasagna_load_reads(const char *ascii, uint64_t n, uint32_t L, uint64_t *packed,
                                   uint64_t *first_bad, void *stream)
 {
@@ -444,23 +475,9 @@ lasagna_status lasagna_load_reads(const char *ascii, uint64_t n, uint32_t L, uin
         set_error("NULL or misaligned pointer");
         return LASAGNA_EINVAL;
     }
-    cudaPointerAttributes at;
-    if (cudaPointerGetAttributes(&at, ascii) != cudaSuccess) {
-        cudaGetLastError();
-        set_error("ascii: not a CUDA-visible pointer");
-        return LASAGNA_EINVAL;
-    }
-    const char *src = ascii;
-    if (at.type == cudaMemoryTypeHost) {
-        if (!at.devicePointer) {
-            set_error("ascii: page-locked host memory is not mapped into the device");
-            return LASAGNA_EINVAL;
-        }
-        src = (const char *)at.devicePointer;
-    } else if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
-        set_error("ascii: pageable host memory; pass device or page-locked host memory");
-        return LASAGNA_EINVAL;
-    }
+    const char *src = nullptr;
+    lasagna_status rs = resolve_ascii(ascii, &src);
+    if (rs != LASAGNA_OK) return rs;
     if (!is_device_ptr(packed)) {
         set_error("packed must be device memory");
         return LASAGNA_EINVAL;
@@ -506,12 +523,15 @@ lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budge
     return LASAGNA_OK;
 }
 
-lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t L,
-                                    uint32_t l_min, uint32_t lengths_per_pass, void *workspace,
-                                    size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
-                                    lasagna_stats *stats, void *stream)
+// a1-a7.  Either `packed` (already staged) or `ascii_dev` (device address of the ASCII reads:
+// a1 is fused into the first group's table build, the packed rows land in packed_out, bad
+// reads in *first_bad).
+static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *ascii_dev,
+                                        uint64_t *packed_out, uint64_t *first_bad, uint64_t n,
+                                        uint32_t L, uint32_t l_min, uint32_t lengths_per_pass,
+                                        void *workspace, size_t *workspace_bytes, uint32_t *succ,
+                                        uint8_t *olen, lasagna_stats *stats, void *stream)
 {
-    g_err[0] = 0;
     lasagna_status rc = check_shape(n, L, l_min);
     if (rc != LASAGNA_OK) return rc;
     if (!workspace_bytes) {
@@ -531,8 +551,9 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
         if (stats) memset(stats, 0, sizeof *stats);
         return LASAGNA_OK;
     }
+    if (ascii_dev) packed = packed_out;
     if (!packed || !succ || !olen || !aligned(packed, 16) || !aligned(succ, 4) ||
-        !aligned(workspace, 256)) {
+        !aligned(workspace, 256) || (ascii_dev && (!first_bad || !aligned(first_bad, 8)))) {
         set_error("NULL or misaligned pointer");
         return LASAGNA_EINVAL;
     }
@@ -555,6 +576,19 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     r.s = s;
     r.bind(workspace);
     uint8_t *claimed = r.at<uint8_t>(r.lay.claimed);
+    if (ascii_dev) {
+        // a1: fused into the first partition pass when the fast path runs (T = 16, L <= 160),
+        // otherwise a separate pack launch
+        LSG_CUDA(cudaMemsetAsync(first_bad, 0xFF, 8, s));
+        if (use_bucketed(g) && g.P == 2 && L <= 160) {
+            r.ascii = reinterpret_cast<const unsigned char *>(ascii_dev);
+            r.packed_out = packed_out;
+            r.first_bad = reinterpret_cast<unsigned long long *>(first_bad);
+        } else {
+            if ((rc = launch_pack(ascii_dev, n, L, packed_out, first_bad, s)) != LASAGNA_OK)
+                return rc;
+        }
+    }
     GreedyBufs gb;
     gb.pool = r.pool;
     gb.pool2 = r.pool2;
@@ -610,6 +644,14 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
     unsigned long long h[CTR64_N];
     LSG_CUDA(cudaMemcpyAsync(h, r.ctr64, sizeof h, cudaMemcpyDeviceToHost, s));
     LSG_CUDA(cudaStreamSynchronize(s));
+    if (ascii_dev) {
+        unsigned long long fb = 0;
+        LSG_CUDA(cudaMemcpy(&fb, first_bad, 8, cudaMemcpyDeviceToHost));
+        if (fb != ~0ull) {
+            set_error("read %llu holds a byte outside ACGTacgt", fb);
+            return LASAGNA_EINVAL;
+        }
+    }
     if (r.bucketed && h[CTR_OVERFLOW]) continue; // a slack region overflowed: exact path
     const unsigned long long *book = h + CTR_BOOK;
     if (book[2] > cap) {
@@ -631,6 +673,38 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
   }
     set_error("internal: no path completed");
     return LASAGNA_ECUDA;
+}
+
+lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t L,
+                                    uint32_t l_min, uint32_t lengths_per_pass, void *workspace,
+                                    size_t *workspace_bytes, uint32_t *succ, uint8_t *olen,
+                                    lasagna_stats *stats, void *stream)
+{
+    g_err[0] = 0;
+    return greedy_graph_impl(packed, nullptr, nullptr, nullptr, n, L, l_min, lengths_per_pass,
+                             workspace, workspace_bytes, succ, olen, stats, stream);
+}
+
+lasagna_status lasagna_greedy_graph_ascii(const char *ascii, uint64_t n, uint32_t L,
+                                          uint32_t l_min, uint32_t lengths_per_pass,
+                                          void *workspace, size_t *workspace_bytes,
+                                          uint64_t *packed_out, uint64_t *first_bad,
+                                          uint32_t *succ, uint8_t *olen, lasagna_stats *stats,
+                                          void *stream)
+{
+    g_err[0] = 0;
+    const char *dev = nullptr;
+    if (workspace && n) {
+        if (!ascii) {
+            set_error("ascii is NULL");
+            return LASAGNA_EINVAL;
+        }
+        lasagna_status rc = resolve_ascii(ascii, &dev);
+        if (rc != LASAGNA_OK) return rc;
+    }
+    return greedy_graph_impl(nullptr, dev ? dev : ascii, packed_out, first_bad, n, L, l_min,
+                             lengths_per_pass, workspace, workspace_bytes, succ, olen, stats,
+                             stream);
 }
 
 lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,

@@ -5,7 +5,7 @@
 // so the CTA copies it into shared memory with 16-byte vector loads (from HBM, or straight
 // from page-locked host memory over PCIe: zero-copy staging), validates every byte, and
 // each thread packs one read (32 bases per u64, base 0 in the low bits).
-#include "kernels.cuh"
+#include "pack.cuh"
 
 namespace lsg {
 
@@ -20,45 +20,12 @@ pack_kernel(const unsigned char *__restrict__ ascii, uint64_t n, uint32_t L, uin
     const uint64_t r0 = (uint64_t)blockIdx.x * READS_PER_CTA;
     if (r0 >= n) return;
     const uint64_t r1 = min64(n, r0 + READS_PER_CTA);
-    const uint64_t b0 = r0 * L, b1 = r1 * L; // byte span [b0, b1)
-    // Shared-memory image of the span, laid out so that smem offset = absolute address - sbase
-    // with sbase 16-byte aligned: the aligned interior moves with 16 B vector loads/stores
-    // (from HBM, or straight from page-locked host memory), the ragged ends byte by byte.
-    const uint64_t base = (uint64_t)(uintptr_t)ascii;
-    const uint64_t sbase = (base + b0) & ~15ull;
-    const uint64_t a0 = min64((base + b0 + 15) & ~15ull, base + b1), a1 = (base + b1) & ~15ull;
-    if (a0 < a1) {
-        const uint64_t nv = (a1 - a0) / 16;
-        const uint4 *src = reinterpret_cast<const uint4 *>((uintptr_t)a0);
-        for (uint64_t t = threadIdx.x; t < nv; t += PACK_THREADS)
-            *reinterpret_cast<uint4 *>(sbuf + (a0 - sbase) + 16 * t) = src[t];
-        for (uint64_t t = base + b0 + threadIdx.x; t < a0; t += PACK_THREADS)
-            sbuf[t - sbase] = *reinterpret_cast<const unsigned char *>((uintptr_t)t);
-        for (uint64_t t = a1 + threadIdx.x; t < base + b1; t += PACK_THREADS)
-            sbuf[t - sbase] = *reinterpret_cast<const unsigned char *>((uintptr_t)t);
-    } else {
-        for (uint64_t t = base + b0 + threadIdx.x; t < base + b1; t += PACK_THREADS)
-            sbuf[t - sbase] = *reinterpret_cast<const unsigned char *>((uintptr_t)t);
-    }
+    const uint32_t off = stage_ascii(ascii, r0 * L, r1 * L, sbuf, PACK_THREADS);
     __syncthreads();
-
     const uint64_t i = r0 + threadIdx.x;
     if (i >= r1) return;
-    const unsigned char *row = sbuf + (base + b0 - sbase) + (uint64_t)threadIdx.x * L;
-    bool bad = false;
-    uint64_t *out = packed + i * stride;
-    for (uint32_t w = 0; w < stride; ++w) {
-        uint64_t word = 0;
-        uint32_t kend = min(L, 32u * (w + 1));
-        for (uint32_t k = 32u * w; k < kend; ++k) {
-            unsigned ch = row[k];
-            unsigned lc = ch | 0x20u;
-            bad |= !(lc == 'a' || lc == 'c' || lc == 'g' || lc == 't');
-            word |= (uint64_t)((ch >> 1) & 3u) << (2 * (k & 31));
-        }
-        out[w] = word;
-    }
-    if (bad && first_bad) atomicMin(first_bad, (unsigned long long)i);
+    const bool ok = pack_row(sbuf + off + (uint64_t)threadIdx.x * L, L, stride, packed + i * stride);
+    if (!ok && first_bad) atomicMin(first_bad, (unsigned long long)i);
 }
 
 __global__ void set_u64(unsigned long long *p, unsigned long long v) { *p = v; }

@@ -23,6 +23,7 @@
 #include <cstdlib>
 
 #include "fingerprint.cuh"
+#include "pack.cuh"
 #include "joinwin.cuh"
 
 namespace lsg {
@@ -155,7 +156,7 @@ scatter_table_kernel(ScatterArgs a)
 
 // Two lengths per partition round (non-split level 1): half the barriers, half the scans and
 // reservation atomics of the one-length round; bins k * 256 + digit for the round's k-th length.
-template <int W>
+template <int W, bool ASCII>
 __global__ void __launch_bounds__(SC_THREADS, 2)
 scatter_table2_kernel(ScatterArgs a)
 {
@@ -168,7 +169,27 @@ scatter_table2_kernel(ScatterArgs a)
     const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
     const bool valid = i < a.n;
     uint64_t x[W], y[W];
-    if (valid) {
+    if constexpr (ASCII) {
+        // a1 fused: stage this CTA's ASCII span (zero-copy from host memory over PCIe when
+        // the caller passed page-locked host memory), pack, validate, keep the packed rows
+        extern __shared__ __align__(16) unsigned char sascii[];
+        const uint64_t r0 = (uint64_t)blockIdx.x * SC_THREADS;
+        const uint64_t r1 = min64(a.n, r0 + SC_THREADS);
+        const uint32_t off = stage_ascii(a.ascii, r0 * a.L, r1 * a.L, sascii, SC_THREADS);
+        __syncthreads();
+        if (valid) {
+            const bool ok = pack_row_regs<W>(sascii + off + (uint64_t)threadIdx.x * a.L, a.L, x);
+            uint64_t *po = a.packed_out + i * a.stride;
+#pragma unroll
+            for (int j = 0; j < W; ++j) po[j] = x[j];
+            for (uint32_t j = W; j < a.stride; ++j) po[j] = 0;
+            if (!ok) atomicMin(a.first_bad, (unsigned long long)i);
+            rc_words<W>(x, a.L, y);
+        } else {
+#pragma unroll
+            for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
+        }
+    } else if (valid) {
         load_read<W>(a.packed, a.stride, i, x);
         rc_words<W>(x, a.L, y);
     } else {
@@ -271,8 +292,13 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
             scatter_table_kernel<W, true><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
         else if (one_length)
             scatter_table_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
-        else
-            scatter_table2_kernel<W><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
+        else if (args.ascii) {
+            const size_t smem = (size_t)SC_THREADS * args.L + 16;
+            LSG_CUDA(cudaFuncSetAttribute(scatter_table2_kernel<W, true>,
+                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            scatter_table2_kernel<W, true><<<(unsigned)blocks, SC_THREADS, smem, s>>>(args);
+        } else
+            scatter_table2_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
         LSG_LAUNCHED("scatter_table_kernel");
         return LASAGNA_OK;
     });

@@ -72,6 +72,8 @@ def lib() -> ctypes.CDLL:
         "lasagna_overlaps": [vp, u64, u32, u32, vp, psz, vp, vp, vp, u64, pu64, vp],
         "lasagna_greedy_graph": [vp, u64, u32, u32, u32, vp, psz, vp, vp,
                                  ctypes.POINTER(_Stats), vp],
+        "lasagna_greedy_graph_ascii": [vp, u64, u32, u32, u32, vp, psz, vp, vp, vp, vp,
+                                       ctypes.POINTER(_Stats), vp],
         "lasagna_plan": [u64, u32, u32, sz, pu32, psz],
         "lasagna_sort_u64": [vp, vp, u64, u32, u32, vp, psz, vp],
         "lasagna_greedy_pairs": [u64, vp, vp, vp, u64, vp, psz, vp, vp, pu32, vp],
@@ -219,14 +221,32 @@ class GreedyGraph:
         self.olen = torch.empty(2 * n, dtype=torch.uint8, device=self.device)
 
     def __call__(self, packed: torch.Tensor, stats: bool = True) -> GraphResult:
+        """a1-a7 on already packed reads (lasagna_greedy_graph)."""
+        return self._run(lambda ws, st: lib().lasagna_greedy_graph(
+            _ptr(packed), self.n, self.L, self.l_min, self.lengths_per_pass, _ptr(self.ws),
+            ctypes.byref(ws), _ptr(self.succ), _ptr(self.olen), st, _stream(self.device)), stats)
+
+    def from_ascii(self, ascii: torch.Tensor, stats: bool = True) -> GraphResult:
+        """a1-a7 from (n, L) uint8 ASCII reads on the device or in page-locked host memory
+        (lasagna_greedy_graph_ascii: staging fused into the first table pass)."""
+        if not ascii.is_cuda and not ascii.is_pinned():
+            raise ValueError("ascii must be a CUDA tensor or page-locked host memory")
+        ascii = ascii.contiguous()
+        if getattr(self, "packed", None) is None:
+            self.packed = torch.empty((self.n, words_per_read(self.L)), dtype=torch.int64,
+                                      device=self.device)
+            self.first_bad = torch.empty(1, dtype=torch.int64, device=self.device)
+        return self._run(lambda ws, st: lib().lasagna_greedy_graph_ascii(
+            _ptr(ascii), self.n, self.L, self.l_min, self.lengths_per_pass, _ptr(self.ws),
+            ctypes.byref(ws), _ptr(self.packed), _ptr(self.first_bad), _ptr(self.succ),
+            _ptr(self.olen), st, _stream(self.device)), stats)
+
+    def _run(self, call, stats: bool) -> GraphResult:
         st = _Stats()
         for _ in range(4):
             ws = ctypes.c_size_t(self.ws_bytes)
             with torch.cuda.device(self.device):
-                rc = lib().lasagna_greedy_graph(
-                    _ptr(packed), self.n, self.L, self.l_min, self.lengths_per_pass, _ptr(self.ws),
-                    ctypes.byref(ws), _ptr(self.succ), _ptr(self.olen),
-                    ctypes.byref(st) if stats else None, _stream(self.device))
+                rc = call(ws, ctypes.byref(st) if stats else None)
             if rc == ENOSPC and ws.value > self.ws_bytes:
                 self.ws_bytes = int(ws.value)
                 self.ws = None

@@ -403,3 +403,28 @@ def test_exact_path_cfg1(path):
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                          cwd=ROOT, timeout=600)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+
+
+@gpu
+@pytest.mark.parametrize("where", ["device", "pinned"])
+def test_greedy_graph_from_ascii(lz, where):
+    """lasagna_greedy_graph_ascii (a1 fused into the first table pass) == the oracle, from
+    device memory and from page-locked host memory; bad reads are reported."""
+    import torch
+    cfg = readgen.CONFIGS["cfg2"]
+    reads = readgen.config_reads(cfg, n=400_000)
+    n, L = reads.shape
+    t = torch.from_numpy(reads)
+    t = t.cuda() if where == "device" else t.pin_memory()
+    g = lz.GreedyGraph(n, L, cfg.l_min, "cuda")
+    r = g.from_ascii(t)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, cfg.l_min)
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    assert np.array_equal(_np(g.packed, np.uint64), oracle.pack(reads, lz.words_per_read(L)))
+    bad = reads.copy()
+    bad[12345, 7] = ord("N")
+    tb = torch.from_numpy(bad)
+    tb = tb.cuda() if where == "device" else tb.pin_memory()
+    with pytest.raises(lz.LasagnaError, match="read 12345"):
+        g.from_ascii(tb)
