@@ -229,6 +229,10 @@ def main() -> None:
     ap.add_argument("--lengths-per-pass", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--n", type=int, default=0, help="override read count (debug)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend of the multi-GPU path (gloo: ranks may share a GPU)")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="run the sharded multi-GPU path even with one rank")
     args = ap.parse_args()
     cfg = readgen.CONFIGS[args.config]
     if args.n:
@@ -240,7 +244,7 @@ def main() -> None:
     if args.impl == "reference":
         run_reference(args, cfg, rank)
         return
-    if world > 1:
+    if world > 1 or args.force_dist:
         from paper_conf_ipps_goswamilsp18_b200 import dist
         dist.bench_main(args, cfg, METRIC, _peaks(), ClockSampler, _bus_id, cpu_baseline)
         return

@@ -284,10 +284,13 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
     """`bench.py` under torchrun: strong scaling at fixed n (every rank holds 1/g of the reads),
     barrier + synchronize around exactly K steps, time = max over ranks."""
     import readgen
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    dist.init_process_group("nccl", device_id=dev)
+    if getattr(args, "dist_backend", "nccl") == "nccl":
+        dist.init_process_group("nccl", device_id=dev)
+    else:
+        dist.init_process_group("gloo")
     world, rank = dist.get_world_size(), dist.get_rank()
     n, L, l_min = cfg.n, cfg.L, cfg.l_min
     lo, hi, _ = shard_range(n, world, rank)
