@@ -284,6 +284,9 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
     """`bench.py` under torchrun: strong scaling at fixed n (every rank holds 1/g of the reads),
     barrier + synchronize around exactly K steps, time = max over ranks."""
     import readgen
+    for k, v in (("RANK", "0"), ("WORLD_SIZE", "1"), ("MASTER_ADDR", "127.0.0.1"),
+                 ("MASTER_PORT", "29517")):
+        os.environ.setdefault(k, v)  # --force-dist without torchrun: a one-rank group
     local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)

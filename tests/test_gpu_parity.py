@@ -428,3 +428,34 @@ def test_greedy_graph_from_ascii(lz, where):
     tb = tb.cuda() if where == "device" else tb.pin_memory()
     with pytest.raises(lz.LasagnaError, match="read 12345"):
         g.from_ascii(tb)
+
+
+@gpu
+@pytest.mark.slow
+def test_cfg3_full_size_parity_and_invariants(lz):
+    """cfg3 (BASELINE configs[2], 34.85 M reads) in the launch configuration bench.py times
+    (a1-a7 from ASCII, all 38 lengths in one pass): bit-exact against the oracle run on the
+    box's host cores (a few minutes), plus the graph invariants vectorised over all edges."""
+    import torch
+    cfg = readgen.CONFIGS["cfg3"]
+    host = torch.empty((cfg.n, cfg.L), dtype=torch.uint8).pin_memory()
+    readgen.reads_into(host.data_ptr(), cfg.seed, cfg.G, cfg.L, cfg.p_err, 0, cfg.n)
+    g = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda")
+    r = g.from_ascii(host)
+    succ = _np(r.succ, np.uint32).copy()
+    olen = _np(r.olen, np.uint8).copy()
+    st = r.stats
+    del g, r
+    torch.cuda.empty_cache()
+    esucc, eolen, m, acc = oracle.greedy_graph(host.numpy(), cfg.l_min)
+    assert st["n_pairs"] == m and st["n_greedy"] == acc
+    assert np.array_equal(succ, esucc)
+    assert np.array_equal(olen, eolen)
+    # invariants (P:L37, P:L168) on every edge: complement edge present, in-degree <= 1
+    has = succ != NONE
+    us = np.nonzero(has)[0]
+    vs = succ[us].astype(np.int64)
+    assert len(np.unique(vs)) == len(vs)
+    assert np.array_equal(succ[vs ^ 1].astype(np.int64), us ^ 1)
+    assert np.all((olen[us] >= cfg.l_min) & (olen[us] <= cfg.L - 1))
+    assert np.all((us >> 1) != (vs >> 1))
