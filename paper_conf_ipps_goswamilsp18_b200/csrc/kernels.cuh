@@ -94,7 +94,8 @@ struct RefineArgs {
 lasagna_status launch_refine(const RefineArgs &a, uint64_t n_regions, cudaStream_t s);
 struct BucketJoinArgs {
     JoinArgs j;               // packed, L, stride, l, vbits, pairs, cap, count, false_matches
-    const uint64_t *buckets;  // [n_buckets][2][half_cap]: prefix half, suffix half
+    uint64_t *buckets;        // [n_buckets][2][half_cap]: prefix half, suffix half (the join
+                              // writes sentinels after odd fills)
     const uint32_t *fills;    // [n_buckets][2]
     uint64_t half_cap, n_buckets;
     uint32_t *overflow;

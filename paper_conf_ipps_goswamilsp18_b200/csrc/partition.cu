@@ -420,21 +420,22 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 
 // ------------------------------------------------------------------ a5 over the buckets
 // Buckets are stored split: prefix entries [b][0][0..fillP), suffix entries [b][1][0..fillS).
-// A window = consecutive whole buckets whose halves fit the staging buffers; the copy engine
-// (cp.async.bulk) stages window w+1 while window w is joined.  A half's copy is rounded up
-// to 16 bytes, so an odd fill drags one stale slot along: it is overwritten with a sentinel
-// key (~0: tag bits set, never equal to a real key of the other list) after the copy lands.
-constexpr int BJ_HALF = 3072;   // staged prefix entries per window
+// A window = consecutive whole buckets whose prefix halves and suffix halves each fit a
+// staging buffer.  The copy engine (cp.async.bulk, one mbarrier per buffer pair) stages both
+// halves of window w+1 while window w is joined: its prefix entries are hashed in shared
+// memory (chained, epoch-tagged heads: never cleared) and its suffix entries probe the table.
+// A half's copy is rounded up to 16 bytes: an odd fill drags one more slot along, which the
+// CTA overwrote beforehand (in global memory) with a sentinel of the wrong tag — ~0 (tag 1)
+// in a prefix half, ~0 ^ (1 << vbits) (tag 0) in a suffix half — so the insert and probe
+// loops skip it by its tag bit alone.  Two barriers per window.
+constexpr int BJ_HALF = 2560;   // staged entries per half per window
 constexpr int BJ_MAXB = 64;     // buckets per window
-constexpr int BJ_FILLS = 1024;  // buckets whose fills are staged at once
+constexpr int BJ_FILLS = 256;   // buckets whose fills are staged at once
 constexpr int BJ_SLOTS = 4096;
-constexpr int BJ_SBATCH = 4;    // suffix entries per thread loaded before probing
 
 struct WinDesc {
-    uint32_t nb, nP;                 // buckets, staged prefix slots (padded)
+    uint32_t nb, nP, nS;             // buckets (0: one oversized bucket), staged slots
     uint32_t first;                  // first bucket (index within the chunk)
-    uint32_t oP[BJ_MAXB + 1];        // staging offset of each bucket's prefix half
-    uint32_t odd[BJ_MAXB];           // sentinel slot of an odd prefix fill (or ~0)
 };
 
 template <int W>
@@ -453,20 +454,14 @@ __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const ui
     }
 }
 
-// Buckets are stored split: prefix entries [b][0][0..fillP), suffix entries [b][1][0..fillS).
-// A window = consecutive whole buckets whose prefix halves fit the staging buffer; the copy
-// engine (cp.async.bulk) stages the prefix halves of window w+1 while window w is joined:
-// its prefix halves are hashed in shared memory and its suffix halves are streamed from global
-// memory (a few loads in flight per thread) and probed.  A prefix copy is rounded up to 16
-// bytes, so an odd fill drags one stale slot along: it is overwritten with a sentinel key
-// (~0, never equal to a real suffix key: the tag bits differ) after the copy lands.
 template <int W>
 __global__ void __launch_bounds__(JOIN_THREADS, 2)
 bucket_join_kernel(BucketJoinArgs b)
 {
     extern __shared__ __align__(128) unsigned char jsm[];
     uint64_t *pst = reinterpret_cast<uint64_t *>(jsm);                    // [2][BJ_HALF]
-    unsigned long long *buf = reinterpret_cast<unsigned long long *>(pst + 2 * BJ_HALF); // [BUF]
+    uint64_t *sst = pst + 2 * BJ_HALF;                                    // [2][BJ_HALF]
+    unsigned long long *buf = reinterpret_cast<unsigned long long *>(sst + 2 * BJ_HALF); // [BUF]
     uint32_t *slot = reinterpret_cast<uint32_t *>(buf + JOIN_BUF);       // [BJ_SLOTS]
     unsigned short *next = reinterpret_cast<unsigned short *>(slot + BJ_SLOTS); // [BJ_HALF]
     uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
@@ -478,6 +473,7 @@ bucket_join_kernel(BucketJoinArgs b)
     const uint64_t b0 = nbk * blockIdx.x / gridDim.x, b1 = nbk * (blockIdx.x + 1) / gridDim.x;
     const uint32_t kshift = a.vbits + 1;
     const uint64_t vmask = (1ull << a.vbits) - 1;
+    const uint64_t tagbit = 1ull << a.vbits;
     if (threadIdx.x == 0) {
         bcount = 0, vdone = 0;
         mbar_init(&mbar[0], 1);
@@ -495,47 +491,56 @@ bucket_join_kernel(BucketJoinArgs b)
         for (uint32_t t = threadIdx.x; t < 2 * nc; t += JOIN_THREADS) {
             const uint32_t f = b.fills[2 * c0 + t];
             if (f > b.half_cap) *b.overflow = 1u;
-            sfill[t] = (uint32_t)min64(f, b.half_cap);
+            const uint32_t fc = (uint32_t)min64(f, b.half_cap);
+            sfill[t] = fc;
+            if (fc & 1) // half_cap is even: the slot after an odd fill is inside the half
+                b.buckets[(c0 + t / 2) * 2 * b.half_cap + (t & 1) * b.half_cap + fc] =
+                    (t & 1) ? ~tagbit : ~0ull;
         }
+        // the sentinels are read by the async proxy (bulk copies)
+        asm volatile("fence.proxy.async.global;" ::: "memory");
         __syncthreads();
         // plan the window starting at chunk bucket k into descriptor w and start its copies
-        // (thread 0).  A bucket whose prefix half exceeds the staging buffer is a window of
-        // its own with nb = 0, joined in global memory.
+        // (thread 0).  A bucket with a half larger than a staging buffer is a window of its
+        // own with nb = 0, joined in global memory.
         auto plan = [&](uint32_t k, int w) -> uint32_t {
             WinDesc &d = wd[w];
             d.first = k;
-            if (sfill[2 * k] > (uint32_t)BJ_HALF) {
+            if (sfill[2 * k] > (uint32_t)BJ_HALF || sfill[2 * k + 1] > (uint32_t)BJ_HALF) {
                 d.nb = 0;
                 return k + 1;
             }
-            uint32_t nP = 0, nb = 0, e = k;
+            uint32_t nP = 0, nS = 0, nb = 0, e = k;
             while (e < nc && nb < (uint32_t)BJ_MAXB) {
-                const uint32_t fp = sfill[2 * e];
-                const uint32_t pp = (fp + 1) & ~1u;
-                if (nP + pp > (uint32_t)BJ_HALF) break;
-                d.oP[nb] = nP;
-                d.odd[nb] = (fp & 1) ? nP + fp : ~0u;
-                nP += pp, ++nb, ++e;
+                const uint32_t pp = (sfill[2 * e] + 1) & ~1u, ps = (sfill[2 * e + 1] + 1) & ~1u;
+                if (nP + pp > (uint32_t)BJ_HALF || nS + ps > (uint32_t)BJ_HALF) break;
+                nP += pp, nS += ps, ++nb, ++e;
             }
-            d.oP[nb] = nP;
-            d.nb = nb, d.nP = nP;
-            if (nP) {
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(
-                                 smem_u32(&mbar[w])),
-                             "r"(nP * 8)
+            d.nb = nb, d.nP = nP, d.nS = nS;
+            const uint32_t bar = smem_u32(&mbar[w]);
+            if (nP + nS) {
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                             "r"((nP + nS) * 8)
                              : "memory");
+                uint32_t oP = 0, oS = 0;
                 for (uint32_t q = 0; q < nb; ++q) {
-                    const uint32_t pp = d.oP[q + 1] - d.oP[q];
+                    const uint32_t pp = (sfill[2 * (k + q)] + 1) & ~1u;
+                    const uint32_t ps = (sfill[2 * (k + q) + 1] + 1) & ~1u;
+                    const uint64_t *gb = b.buckets + (c0 + k + q) * 2 * b.half_cap;
                     if (pp)
                         asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
-                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + d.oP[q])),
-                                     "l"(b.buckets + (c0 + k + q) * 2 * b.half_cap), "r"(pp * 8),
-                                     "r"(smem_u32(&mbar[w]))
+                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + oP)),
+                                     "l"(gb), "r"(pp * 8), "r"(bar)
                                      : "memory");
+                    if (ps)
+                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
+                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(sst + w * BJ_HALF + oS)),
+                                     "l"(gb + b.half_cap), "r"(ps * 8), "r"(bar)
+                                     : "memory");
+                    oP += pp, oS += ps;
                 }
             } else {
-                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&mbar[w]))
-                             : "memory");
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
             }
             return e;
         };
@@ -561,51 +566,35 @@ bucket_join_kernel(BucketJoinArgs b)
             } else {
                 mbar_wait(&mbar[w], (phases >> w) & 1u);
                 phases ^= 1u << w;
-                uint64_t *P = pst + w * BJ_HALF;
-                for (uint32_t t = threadIdx.x; t < d.nb; t += JOIN_THREADS)
-                    if (d.odd[t] != ~0u) P[d.odd[t]] = ~0ull;
-                if (++epoch == 0x10000u) {
+                if (++epoch == 0x10000u) { // block-uniform
                     for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
                     epoch = 1;
+                    __syncthreads();
                 }
-                __syncthreads();
+                const uint64_t *P = pst + w * BJ_HALF, *S = sst + w * BJ_HALF;
                 const uint32_t tag = epoch << 16;
-                const uint32_t nP = d.nP;
+                const uint32_t nP = d.nP, nS = d.nS;
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
                     const uint64_t e = P[k2];
-                    if (e == ~0ull) continue;
+                    if (e & tagbit) continue; // sentinel
                     const uint32_t h = (uint32_t)(e >> kshift) & (BJ_SLOTS - 1);
                     const uint32_t old = atomicExch(&slot[h], tag | k2);
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
                 __syncthreads();
-                // probe: the suffix halves of the window's buckets, straight from global memory
-                for (uint32_t q = 0; q < d.nb; ++q) {
-                    const uint32_t fs = sfill[2 * (d.first + q) + 1];
-                    const uint64_t *gS = b.buckets + (c0 + d.first + q) * 2 * b.half_cap + b.half_cap;
-                    for (uint32_t t0 = 0; t0 < fs; t0 += JOIN_THREADS * BJ_SBATCH) {
-                        uint64_t sv[BJ_SBATCH];
-#pragma unroll
-                        for (int r = 0; r < BJ_SBATCH; ++r) {
-                            const uint32_t t = t0 + r * JOIN_THREADS + threadIdx.x;
-                            sv[r] = t < fs ? gS[t] : 0ull;
-                        }
-#pragma unroll
-                        for (int r = 0; r < BJ_SBATCH; ++r) {
-                            if (t0 + r * JOIN_THREADS + threadIdx.x >= fs) continue;
-                            const uint64_t e = sv[r];
-                            const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
-                            uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
-                            while (sl != 0xFFFFu) {
-                                const uint64_t p = P[sl];
-                                if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-                                sl = next[sl];
-                            }
-                        }
+                for (uint32_t t = threadIdx.x; t < nS; t += JOIN_THREADS) {
+                    const uint64_t e = S[t];
+                    if (!(e & tagbit)) continue; // sentinel
+                    const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
+                    uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
+                    while (sl != 0xFFFFu) {
+                        const uint64_t p = P[sl];
+                        if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
+                        sl = next[sl];
                     }
                 }
             }
-            __syncthreads(); // window w done: its buffer may be refilled
+            __syncthreads(); // window w done: its buffers may be refilled
             window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
             kcur = knext;
             w ^= 1;
@@ -616,193 +605,13 @@ bucket_join_kernel(BucketJoinArgs b)
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
 
-// ------------------------------------------------------------------ a5, one warp per bucket
-// When a bucket half fits a warp's shared-memory slice, every warp joins whole buckets on
-// its own (no block barriers): the prefix half is hashed in the warp's slice (chained,
-// epoch-tagged heads: never cleared), the suffix half is streamed straight from global
-// memory and probed, candidates are staged per warp and verified 32 at a time.
-constexpr int WJ_WARPS = 4;
-constexpr int WJ_CAND = 64;
-constexpr int WJ_BATCH = 8; // global loads in flight per lane
-
-template <int W>
-__global__ void __launch_bounds__(WJ_WARPS * 32)
-warp_join_kernel(BucketJoinArgs b, uint32_t pcap, uint32_t nheads)
-{
-    extern __shared__ __align__(16) unsigned char wsm[];
-    const JoinArgs &a = b.j;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const size_t next_b = ((size_t)pcap * 2 + 15) & ~(size_t)15;
-    const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 + next_b + WJ_CAND * 8;
-    unsigned char *base = wsm + warp * per_warp;
-    uint64_t *P = reinterpret_cast<uint64_t *>(base);
-    uint32_t *heads = reinterpret_cast<uint32_t *>(base + (size_t)pcap * 8);
-    unsigned short *next = reinterpret_cast<unsigned short *>(base + (size_t)pcap * 8 + nheads * 4);
-    unsigned long long *cand =
-        reinterpret_cast<unsigned long long *>(base + (size_t)pcap * 8 + nheads * 4 + next_b);
-    const uint32_t kshift = a.vbits + 1;
-    const uint64_t vmask = (1ull << a.vbits) - 1;
-    const uint32_t hmask = nheads - 1;
-    const uint32_t lt = (1u << lane) - 1;
-    for (uint32_t t = lane; t < nheads; t += 32) heads[t] = 0;
-    uint32_t ncand = 0, epoch = 0;
-    unsigned long long nfalse = 0;
-
-    // verify the first 32 staged candidates (lane i takes cand[i]) and append the accepted
-    // ones to the global pool; ncand is warp-uniform
-    auto drain32 = [&](uint32_t k) {
-        __syncwarp();
-        bool ok = false;
-        unsigned long long rec = 0;
-        if ((uint32_t)lane < k) {
-            rec = cand[lane];
-            const uint32_t u = (uint32_t)(rec >> 32), bb = (uint32_t)rec;
-            ok = verify_overlap<W>(a.packed, a.stride, a.L, u, bb ^ 1u, a.l);
-            nfalse += ok ? 0 : 1;
-        }
-        const uint32_t bal = __ballot_sync(0xffffffffu, ok);
-        unsigned long long gb = 0;
-        if (lane == 0 && bal) gb = atomicAdd(a.count, (unsigned long long)__popc(bal));
-        gb = __shfl_sync(0xffffffffu, gb, 0);
-        if (ok) {
-            const unsigned long long pos = gb + __popc(bal & lt);
-            if (pos < a.cap) a.pairs[pos] = rec;
-        }
-        __syncwarp();
-        // move the remainder down
-        if ((uint32_t)lane + 32 < ncand) cand[lane] = cand[lane + 32];
-        __syncwarp();
-    };
-
-    const uint64_t total_warps = (uint64_t)gridDim.x * WJ_WARPS;
-    for (uint64_t bk = (uint64_t)blockIdx.x * WJ_WARPS + warp; bk < b.n_buckets; bk += total_warps) {
-        uint32_t fP = 0, fS = 0;
-        if (lane == 0) {
-            fP = b.fills[2 * bk];
-            fS = b.fills[2 * bk + 1];
-            if (fP > b.half_cap || fS > b.half_cap) *b.overflow = 1u;
-        }
-        fP = (uint32_t)min64(__shfl_sync(0xffffffffu, fP, 0), b.half_cap);
-        fS = (uint32_t)min64(__shfl_sync(0xffffffffu, fS, 0), b.half_cap);
-        if (fP == 0 || fS == 0) continue;
-        if (++epoch == 0x10000u) {
-            for (uint32_t t = lane; t < nheads; t += 32) heads[t] = 0;
-            epoch = 1;
-            __syncwarp();
-        }
-        const uint32_t tag = epoch << 16;
-        const uint64_t *gP = b.buckets + bk * 2 * b.half_cap;
-        const uint64_t *gS = gP + b.half_cap;
-        // stage + hash the prefix half (8 loads per lane in flight before the inserts)
-        for (uint32_t t0 = 0; t0 < fP; t0 += 32 * WJ_BATCH) {
-            uint64_t ev[WJ_BATCH];
-#pragma unroll
-            for (int q = 0; q < WJ_BATCH; ++q) {
-                const uint32_t t = t0 + q * 32 + lane;
-                ev[q] = t < fP ? gP[t] : 0;
-            }
-#pragma unroll
-            for (int q = 0; q < WJ_BATCH; ++q) {
-                const uint32_t t = t0 + q * 32 + lane;
-                if (t < fP) {
-                    P[t] = ev[q];
-                    const uint32_t old =
-                        atomicExch(&heads[(uint32_t)(ev[q] >> kshift) & hmask], tag | t);
-                    next[t] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
-                }
-            }
-        }
-        __syncwarp();
-        // probe with the suffix half, straight from global memory
-        uint64_t sv[WJ_BATCH];
-        for (uint32_t t0 = 0; t0 < fS; t0 += 32) {
-            const uint32_t qq = (t0 / 32) % WJ_BATCH;
-            if (qq == 0) {
-#pragma unroll
-                for (int q = 0; q < WJ_BATCH; ++q) {
-                    const uint32_t t = t0 + q * 32 + lane;
-                    sv[q] = t < fS ? gS[t] : 0;
-                }
-            }
-            const uint32_t t = t0 + lane;
-            uint64_t e = 0;
-#pragma unroll
-            for (int q = 0; q < WJ_BATCH; ++q)
-                if ((uint32_t)q == qq) e = sv[q];
-            uint32_t sl = 0xFFFFu;
-            if (t < fS) {
-                const uint32_t hv = heads[(uint32_t)(e >> kshift) & hmask];
-                sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
-            }
-            while (__any_sync(0xffffffffu, sl != 0xFFFFu)) {
-                bool c = false;
-                unsigned long long rec = 0;
-                if (sl != 0xFFFFu) {
-                    const uint64_t p = P[sl];
-                    if (((p ^ e) >> kshift) == 0) {
-                        const uint32_t u = (uint32_t)(e & vmask), v = (uint32_t)(p & vmask);
-                        const uint32_t bb = v ^ 1u;
-                        if ((u >> 1) != (v >> 1) && u < bb) { // R9; each pair once
-                            c = true;
-                            rec = ((unsigned long long)u << 32) | bb;
-                        }
-                    }
-                    sl = next[sl];
-                }
-                const uint32_t bal = __ballot_sync(0xffffffffu, c);
-                if (bal) {
-                    if (c) cand[ncand + __popc(bal & lt)] = rec;
-                    ncand += __popc(bal);
-                    if (ncand >= 32) {
-                        drain32(32);
-                        ncand -= 32;
-                    }
-                }
-            }
-        }
-        __syncwarp();
-    }
-    if (ncand) {
-        drain32(ncand);
-        ncand = 0;
-    }
-    for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
-    if (lane == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
-}
-
 lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
 {
     if (args.n_buckets == 0) return LASAGNA_OK;
-    // the block join (windows of whole buckets, bulk-copy staged) measured faster than the
-    // warp-per-bucket join at cfg3 (38 vs 50 ms); LASAGNA_WARP_JOIN=1 selects the latter
-    static const bool warp_join = getenv("LASAGNA_WARP_JOIN") != nullptr;
-    const uint32_t pcap = (uint32_t)((args.half_cap + 1) & ~1ull);
-    if (warp_join && pcap <= 2048) {
-        uint32_t nheads = 256; // ~1 prefix entry per chain head
-        while (nheads * 2 <= pcap) nheads <<= 1;
-        const size_t per_warp = (size_t)pcap * 8 + (size_t)nheads * 4 +
-                                (((size_t)pcap * 2 + 15) & ~(size_t)15) + WJ_CAND * 8;
-        const size_t smem = per_warp * WJ_WARPS;
-        return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
-            constexpr int W = decltype(wc)::value;
-            LSG_CUDA(cudaFuncSetAttribute(warp_join_kernel<W>,
-                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            int per_sm = 0;
-            LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, warp_join_kernel<W>,
-                                                                   WJ_WARPS * 32, smem));
-            per_sm = std::max(per_sm, 1);
-            const uint64_t blocks = std::max<uint64_t>(
-                1, std::min<uint64_t>((uint64_t)num_sms() * per_sm,
-                                      ceil_div(args.n_buckets, WJ_WARPS)));
-            warp_join_kernel<W><<<(unsigned)blocks, WJ_WARPS * 32, smem, s>>>(args, pcap, nheads);
-            LSG_LAUNCHED("warp_join_kernel");
-            return LASAGNA_OK;
-        });
-    }
-    if (args.n_buckets == 0) return LASAGNA_OK;
+    if (args.half_cap & 1) return LASAGNA_EINVAL; // sentinels need an even half capacity
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)2 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
+        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
                             (size_t)BJ_SLOTS * 4 + (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
         LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
