@@ -134,7 +134,7 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict) ->
     """Dominant phase and its achieved ALGORITHMIC GB/s (bytes per unit in DESIGN.md x units
     per launch / CUDA-event time per launch)."""
     V = 2 * n
-    N = 2 * V                     # table entries per length (prefix + suffix list)
+    N = V                         # table entries per length (one canonical entry per vertex)
     n_len = L - l_min
     G = stats["lengths_per_pass"]
     verify = 64.0 * (stats["n_pairs"] + stats["fp_false_matches"]) / max(1, n_len)
@@ -327,7 +327,7 @@ def main() -> None:
                    "G": cfg.G, "p_err": cfg.p_err, "seed": cfg.seed,
                    "lengths_per_pass": st["lengths_per_pass"], "passes": st["passes"] // args.steps,
                    "l2": "inputs larger than L2 (ASCII %.1f GB, key tables %.1f GB)"
-                         % (n * L / 1e9, 32.0 * 2 * n * st["lengths_per_pass"] / 1e9)},
+                         % (n * L / 1e9, 16.0 * 2 * n * st["lengths_per_pass"] / 1e9)},
         "overlap_edges_per_s": edges / (ms_step / 1e3),
         "read_end_pairs": st["n_pairs"], "greedy_pairs": st["n_greedy"],
         "fp_false_matches": st["fp_false_matches"], "greedy_rounds_max": st["rounds_max"],

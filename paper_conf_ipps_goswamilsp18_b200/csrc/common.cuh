@@ -50,6 +50,34 @@ __device__ __forceinline__ uint64_t addpow(uint64_t S, uint32_t c, uint64_t pw, 
 constexpr uint64_t MIX = 0x9E3779B97F4A7C15ull;
 __device__ __forceinline__ uint64_t mix(uint64_t f) { return f * MIX; }
 
+// ----------------------------------------------------------------- canonical table entries
+// ONE table entry per oriented read v and length l.  With
+// x = prefix_l(seq(v)), H = F(x) and Hr = F(RC(x)) (= the suffix fingerprint of v^1):
+//   key = mix(min(H, Hr)) top (62 - vbits) bits | flag << vbits | v
+//   flag = 0 if H < Hr ("build" side), 1 if H > Hr ("probe" side), 2 if H == Hr (both).
+// A directed overlap (u, v, l) means suffix_l(seq(u)) == prefix_l(seq(v)), i.e. the prefix
+// strings of w = u^1 and v are reverse complements: equal canonical fingerprints and
+// opposite flags (or both 2).  So the paper's two lists P_l / S_l collapse
+// into one list of V entries whose build side plays P_l and whose probe side plays S_l.
+constexpr uint32_t FLAG_BITS = 2;
+__device__ __forceinline__ uint64_t key_keep(uint32_t vbits)
+{
+    return ~((1ull << (vbits + FLAG_BITS)) - 1);
+}
+// H, Hr folded (congruent mod q); the comparison is on the exact residues
+__device__ __forceinline__ uint64_t canon_key(uint64_t H, uint64_t Hr, uint64_t keep,
+                                              uint32_t vbits, uint64_t v)
+{
+    const uint64_t h = exact61(H), hr = exact61(Hr);
+    const uint64_t c = h < hr ? h : hr;
+    const uint64_t f = h < hr ? 0ull : (h > hr ? 1ull : 2ull);
+    return (mix(c) & keep) | (f << vbits) | v;
+}
+__device__ __forceinline__ uint32_t key_flag(uint64_t key, uint32_t vbits)
+{
+    return (uint32_t)(key >> vbits) & 3u;
+}
+
 // ----------------------------------------------------------------- packed reads
 // base k of a read at bits [2(k mod 32), +2) of word k/32 (lasagna.h, a1).
 

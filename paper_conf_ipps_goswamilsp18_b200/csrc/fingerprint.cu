@@ -56,12 +56,13 @@ lasagna_status launch_fp_values(const uint64_t *packed, uint64_t n, uint32_t L, 
 
 // ---------------------------------------------------------------- key tables (a2 + a3)
 // For each length l in the group [l_lo, l_hi] (segment s = l - l_lo) and every vertex v the
-// combined table of the paper's two lists P_l and S_l:
-//   tab[s*2V + 2v]     = (mix(pfx_l(v)) & keep) | 0 << vbits | v    prefix entry
-//   tab[s*2V + 2v + 1] = (mix(sfx_l(v)) & keep) | 1 << vbits | v    suffix entry
-// (keep = the bits above tag + vid), i.e. 32 contiguous bytes per read per length, plus the
-// histogram of the first LSD digit per segment (onesweep's upfront histogram), accumulated
-// in shared memory and flushed once per CTA.
+// canonical entry (common.cuh): one list of V entries per length whose build side plays the
+// paper's prefix list P_l and whose probe side plays its suffix list S_l:
+//   tab[s*V + 2i]     = canon(pfx_l(r_i),  sfx_l(r_i'))  of vertex 2i
+//   tab[s*V + 2i + 1] = canon(pfx_l(r_i'), sfx_l(r_i))   of vertex 2i+1
+// (RC of the l-prefix of r is the l-suffix of r' and vice versa), i.e. 16 contiguous bytes per
+// read per length, plus the histogram of the first LSD digit per segment (onesweep's upfront
+// histogram), accumulated in shared memory and flushed once per CTA.
 template <int W>
 __global__ void __launch_bounds__(256)
 table_kernel(TableArgs a)
@@ -72,9 +73,8 @@ table_kernel(TableArgs a)
     if (with_hist)
         for (uint32_t t = threadIdx.x; t < G * 256; t += blockDim.x) shist[t] = 0;
     __syncthreads();
-    const uint64_t N = 4 * a.n; // 2V entries per length (of this read range)
-    const uint64_t keep = ~((2ull << a.vbits) - 1);
-    const uint64_t tagS = 1ull << a.vbits;
+    const uint64_t N = 2 * a.n; // V entries per length (of this read range)
+    const uint64_t keep = key_keep(a.vbits);
     const uint32_t dmask = (1u << a.d_bits) - 1;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
          i += (uint64_t)gridDim.x * blockDim.x) {
@@ -84,20 +84,14 @@ table_kernel(TableArgs a)
         roll_read<W>(x, y, a.l_hi, [&](uint32_t l, const FpStreams &st) {
             if (l < a.l_lo) return;
             const uint32_t s = l - a.l_lo;
-            const uint64_t v0 = 2 * (a.read_offset + i), v1 = v0 + 1; // global vertex ids
-            const uint64_t p0 = (mix(exact61(st.P0)) & keep) | v0;
-            const uint64_t s0 = (mix(exact61(st.S0)) & keep) | tagS | v0;
-            const uint64_t p1 = (mix(exact61(st.P1)) & keep) | v1;
-            const uint64_t s1 = (mix(exact61(st.S1)) & keep) | tagS | v1;
-            ulonglong2 *dst = reinterpret_cast<ulonglong2 *>(a.tab + (uint64_t)s * N + 4 * i);
-            dst[0] = make_ulonglong2(p0, s0);
-            dst[1] = make_ulonglong2(p1, s1);
+            const uint64_t v0 = 2 * (a.read_offset + i); // global vertex ids
+            const uint64_t e0 = canon_key(st.P0, st.S1, keep, a.vbits, v0);
+            const uint64_t e1 = canon_key(st.P1, st.S0, keep, a.vbits, v0 + 1);
+            *reinterpret_cast<ulonglong2 *>(a.tab + (uint64_t)s * N + 2 * i) = make_ulonglong2(e0, e1);
             if (with_hist) {
                 uint32_t *h = shist + s * 256;
-                atomicAdd(&h[(uint32_t)((p0 >> a.d_shift) & dmask)], 1u);
-                atomicAdd(&h[(uint32_t)((s0 >> a.d_shift) & dmask)], 1u);
-                atomicAdd(&h[(uint32_t)((p1 >> a.d_shift) & dmask)], 1u);
-                atomicAdd(&h[(uint32_t)((s1 >> a.d_shift) & dmask)], 1u);
+                atomicAdd(&h[(uint32_t)((e0 >> a.d_shift) & dmask)], 1u);
+                atomicAdd(&h[(uint32_t)((e1 >> a.d_shift) & dmask)], 1u);
             }
         });
     }

@@ -2,12 +2,14 @@
 // contiguous-table join (search.cu) and the bucketed join (partition.cu).
 //
 // A window holds the entries of complete T-bit buckets, so every fingerprint match of a
-// suffix entry is a prefix entry of the same window ("a fingerprint present in W_S
-// cannot be present in any window except W_P").  The prefix entries are hashed (chained
-// table in shared memory, one atomicExch per insert), every suffix entry probes it (all
-// matches of its key: the C = U - L matches of P:L164-166), and each candidate from a
-// different read with u < v^1 is staged, then verified on the 2-bit bases in a parallel
-// pass (R12) and written to the global pool as (a << 32) | b.
+// probe entry is a build entry of the same window ("a fingerprint present in W_S
+// cannot be present in any window except W_P").  Entries are canonical (common.cuh): the
+// build side (flags 0 and 2) plays the paper's prefix list, the probe side (flags 1 and 2)
+// its suffix list.  The build entries are hashed (chained table in shared memory, one
+// atomicExch per insert), every probe entry looks its key up (all matches of its key: the
+// C = U - L matches of P:L164-166), and each candidate from a different read is staged, then
+// verified on the 2-bit bases in a parallel pass (R12) and written to the global pool as the
+// read-end pair (a << 32) | b, a < b.
 #pragma once
 
 #include "kernels.cuh"
@@ -29,21 +31,28 @@ struct Stager {
     unsigned long long *pairs, cap, *count;
 };
 
+// Fingerprint match of probe entry e (vertex w, flag 1 or 2) and build entry p (vertex v,
+// flag 0 or 2): if the bases agree, the l-prefixes of w and v are reverse complements, i.e.
+// suffix_l(seq(w^1)) == prefix_l(seq(v)): the directed overlap (w^1, v, l) and its read-end
+// pair {w^1, v^1}.  Each pair has exactly one (build, probe) assignment, except when
+// both entries carry flag 2 (each probes the other): then only w < v is kept.
 template <int W>
-__device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t s_ent, uint64_t p_ent,
+__device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_t p,
                                           uint64_t vmask, Stager &sg, unsigned long long &nfalse)
 {
-    const uint32_t u = (uint32_t)(s_ent & vmask), v = (uint32_t)(p_ent & vmask);
-    const uint32_t b = v ^ 1u;
-    if ((u >> 1) == (v >> 1) || u >= b) return; // R9: no same-read edge; each pair once
-    const unsigned long long rec = ((unsigned long long)u << 32) | b;
+    const uint32_t w = (uint32_t)(e & vmask), v = (uint32_t)(p & vmask);
+    if ((w >> 1) == (v >> 1)) return; // R9: no same-read edge (also the entry itself)
+    if (w > v && key_flag(e, a.vbits) == 2 && key_flag(p, a.vbits) == 2) return;
+    const uint32_t x = w ^ 1u, y = v ^ 1u;
+    const uint32_t lo = min(x, y), hi = max(x, y);
+    const unsigned long long rec = ((unsigned long long)lo << 32) | hi;
     const uint32_t slot = atomicAdd(sg.bcount, 1u);
     if (slot < JOIN_BUF) {
         sg.buf[slot] = rec;
         return;
     }
     // staging full: verify inline and emit straight to global memory
-    if (!verify_overlap<W>(a.packed, a.stride, a.L, u, v, a.l)) {
+    if (!verify_overlap<W>(a.packed, a.stride, a.L, lo, hi ^ 1u, a.l)) {
         ++nfalse;
         return;
     }
@@ -88,19 +97,20 @@ __device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint
 }
 
 
-// hash-join the m staged entries ent[0..m) (whole buckets); slot tags = (epoch << 16) | index
+// hash-join the m staged entries ent[0..m) (whole buckets, both sides mixed); slot tags =
+// (epoch << 16) | index
 template <int W>
 __device__ __forceinline__ void hash_join_window(const JoinArgs &a, const uint64_t *ent, uint32_t m,
                                                  uint32_t *slot, unsigned short *next,
                                                  uint32_t epoch, Stager &em,
                                                  unsigned long long &nfalse)
 {
-    const uint32_t kshift = a.vbits + 1;
+    const uint32_t kshift = a.vbits + FLAG_BITS;
     const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint32_t tag = (epoch & 0xFFFFu) << 16;
     for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
         const uint64_t e = ent[k];
-        if ((e >> a.vbits) & 1) continue;
+        if ((e >> a.vbits) & 1) continue; // flag 1: probe side only
         const uint32_t h = (uint32_t)(e >> kshift) & (JOIN_SLOTS - 1);
         const uint32_t old = atomicExch(&slot[h], tag | k);
         next[k] = (old >> 16) == (tag >> 16) ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
@@ -108,36 +118,7 @@ __device__ __forceinline__ void hash_join_window(const JoinArgs &a, const uint64
     __syncthreads();
     for (uint32_t k = threadIdx.x; k < m; k += JOIN_THREADS) {
         const uint64_t e = ent[k];
-        if (!((e >> a.vbits) & 1)) continue;
-        const uint32_t sv = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
-        uint32_t sl = (sv >> 16) == (tag >> 16) ? (sv & 0xFFFFu) : 0xFFFFu;
-        while (sl != 0xFFFFu) {
-            const uint64_t p = ent[sl];
-            if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
-            sl = next[sl];
-        }
-    }
-}
-
-// split form: prefix entries ent[0..nP), suffix entries ent[s0..s0+nS) (no tag tests, no
-// divergence between the insert and probe passes)
-template <int W>
-__device__ __forceinline__ void hash_join_split(const JoinArgs &a, const uint64_t *ent, uint32_t nP,
-                                                uint32_t s0, uint32_t nS, uint32_t *slot,
-                                                unsigned short *next, uint32_t epoch, Stager &em,
-                                                unsigned long long &nfalse)
-{
-    const uint32_t kshift = a.vbits + 1;
-    const uint64_t vmask = (1ull << a.vbits) - 1;
-    const uint32_t tag = (epoch & 0xFFFFu) << 16;
-    for (uint32_t k = threadIdx.x; k < nP; k += JOIN_THREADS) {
-        const uint32_t h = (uint32_t)(ent[k] >> kshift) & (JOIN_SLOTS - 1);
-        const uint32_t old = atomicExch(&slot[h], tag | k);
-        next[k] = (old >> 16) == (tag >> 16) ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
-    }
-    __syncthreads();
-    for (uint32_t k = threadIdx.x; k < nS; k += JOIN_THREADS) {
-        const uint64_t e = ent[s0 + k];
+        if (key_flag(e, a.vbits) == 0) continue; // flag 0: build side only
         const uint32_t sv = slot[(uint32_t)(e >> kshift) & (JOIN_SLOTS - 1)];
         uint32_t sl = (sv >> 16) == (tag >> 16) ? (sv & 0xFFFFu) : 0xFFFFu;
         while (sl != 0xFFFFu) {
@@ -149,16 +130,16 @@ __device__ __forceinline__ void hash_join_split(const JoinArgs &a, const uint64_
 }
 
 // a run [lo, hi) of global entries too large for a window (massively repeated fingerprints):
-// every suffix entry scans the whole run in global memory
+// every probe entry scans the whole run in global memory
 template <int W>
 __device__ __forceinline__ void oversized_join(const JoinArgs &a, const uint64_t *A, uint64_t lo,
                                                uint64_t hi, Stager &em, unsigned long long &nfalse)
 {
-    const uint32_t kshift = a.vbits + 1;
+    const uint32_t kshift = a.vbits + FLAG_BITS;
     const uint64_t vmask = (1ull << a.vbits) - 1;
     for (uint64_t i = lo + threadIdx.x; i < hi; i += JOIN_THREADS) {
         const uint64_t e = A[i];
-        if (!((e >> a.vbits) & 1)) continue;
+        if (key_flag(e, a.vbits) == 0) continue;
         for (uint64_t j = lo; j < hi; ++j) {
             const uint64_t p = A[j];
             if (((p >> a.vbits) & 1) == 0 && ((p ^ e) >> kshift) == 0)

@@ -22,7 +22,7 @@ struct TableArgs {
     uint32_t l_lo, l_hi;      // group of lengths (segment s = l - l_lo)
     uint32_t vbits;           // b_v: vertex-id bits at the bottom of a key
     uint32_t d_shift, d_bits; // first LSD digit (histogram produced on the fly)
-    uint64_t *tab;            // [G][2V]: entry 2v = prefix key of v, 2v+1 = suffix key of v
+    uint64_t *tab;            // [G][V]: entry v = canonical key of vertex v (common.cuh)
     uint32_t *hist;           // [G][256] first-digit histogram, or null
 };
 lasagna_status launch_table(const TableArgs &a, cudaStream_t s);
@@ -47,7 +47,7 @@ lasagna_status launch_hist(const uint64_t *keys, uint64_t seg_len, uint32_t n_se
 // ---- a5 (search.cu)
 struct JoinArgs {
     const uint64_t *packed;
-    const uint64_t *keys;      // sorted combined table of this length (N = 2V entries)
+    const uint64_t *keys;      // sorted canonical table of this length (N = V entries)
     uint64_t N;
     uint32_t L, stride, l, vbits, T; // T: sorted (bucket) bits
     unsigned long long *pairs; // out pool: (a << 32) | b
@@ -68,6 +68,7 @@ struct ScatterArgs {
     uint64_t n, read_offset;
     uint32_t L, stride, l_lo, l_hi, vbits;
     uint64_t *out;      // [G][256][cap] level-1 regions (top 8 key bits); split: [G][256][2][cap]
+                        // (half 0: flags 0/2 = build side, half 1: flag 1 = probe side)
     uint32_t *fill;     // [G][256] (split: [G][256][2])
     uint64_t cap;
     uint32_t *overflow;

@@ -36,8 +36,9 @@ lasagna_status cuda_status(cudaError_t e, const char *what)
 
 // ------------------------------------------------------------------ planning
 // Geometry of the key tables:
-//   N = 2V entries per length (prefix + suffix list), V = 2n vertices
-//   key = mix(F) top (63 - vbits) bits | tag << vbits | vertex id,  vbits = ceil(log2 V)
+//   N = V entries per length (one canonical entry per vertex, common.cuh), V = 2n vertices
+//   key = mix(min(H, Hr)) top (62 - vbits) bits | flag << vbits | vertex id,
+//   vbits = ceil(log2 V)
 //   radix-sorted by the top T = 8P key bits, P = ceil((log2 N - 11.5) / 8) passes, so a
 //   T-bit bucket holds ~N / 2^T <= ~2.9K entries (one shared-memory join tile)
 struct Geometry {
@@ -72,7 +73,7 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     Geometry g;
     g.n = n;
     g.V = 2 * n;
-    g.N = 2 * g.V;
+    g.N = g.V;
     g.L = L;
     g.l_min = l_min;
     g.n_len = L - l_min; // lengths l_min .. L-1 (R5: the l = L partition is dropped)
@@ -80,7 +81,7 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     const double lg = g.N > 1 ? std::log2((double)g.N) : 0.0;
     int P = (int)std::ceil((lg - 11.5) / 8.0);
     P = std::max(1, std::min(P, 4));
-    g.T = std::min<uint32_t>(8u * (uint32_t)P, 63u - g.vbits);
+    g.T = std::min<uint32_t>(8u * (uint32_t)P, 64u - FLAG_BITS - g.vbits);
     g.P = g.T / 8;
     g.cap1 = region_cap((double)g.N / 256.0);
     g.half1 = region_cap((double)g.N / 512.0);

@@ -64,107 +64,25 @@ __device__ __forceinline__ uint32_t bin_of(uint64_t key, uint32_t dshift, uint32
 }
 
 // ------------------------------------------------------------------ level 1: fused with a2
-template <int W, bool SPLIT>
+// One thread per read, LPR lengths per partition round: the rolling streams (a2) produce the
+// two canonical keys of the read (vertex 2i and 2i+1, common.cuh) for each length; a round
+// ranks its 2 * LPR keys per thread by bin in shared memory (atomics: order inside a region is
+// irrelevant), reserves space in the regions of its lengths with one global atomic per
+// (CTA, bin), stages the keys by bin and writes them out in bin runs.  Bins are
+// q * NBL + bin_of(key) for the round's q-th length.
+template <int W, bool ASCII, bool SPLIT, int LPR>
 __global__ void __launch_bounds__(SC_THREADS, 2)
 scatter_table_kernel(ScatterArgs a)
 {
-    constexpr int NB = SPLIT ? 512 : 256;
-    __shared__ uint64_t stage[SC_THREADS * 4];
-    __shared__ uint32_t cnt[NB], lstart[NB], wsum[16];
-    __shared__ long long gofs[NB]; // per bin: element offset of stage slot 0's destination, -1 = overflow
-    __shared__ uint32_t s_total;
-
-    const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
-    const bool valid = i < a.n;
-    uint64_t x[W], y[W];
-    if (valid) {
-        load_read<W>(a.packed, a.stride, i, x);
-        rc_words<W>(x, a.L, y);
-    } else {
-#pragma unroll
-        for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
-    }
-    if (threadIdx.x < NB) cnt[threadIdx.x] = 0;
-    __syncthreads();
-    const uint64_t keep = ~((2ull << a.vbits) - 1);
-    const uint64_t tagS = 1ull << a.vbits;
-    const uint64_t v0 = 2 * (a.read_offset + i);
-    FpStreams st;
-    st.init();
-#pragma unroll
-    for (int w = 0; w < W; ++w) {
-        uint64_t xa = x[w], yb = y[w];
-        const uint32_t k0 = 32u * w;
-        if (k0 >= a.l_hi) break;
-        const uint32_t kn = min(32u, a.l_hi - k0);
-        for (uint32_t j = 0; j < kn; ++j) {
-            st.step((uint32_t)(xa & 3u), (uint32_t)(yb & 3u), k0 + j);
-            xa >>= 2;
-            yb >>= 2;
-            const uint32_t l = k0 + j + 1;
-            if (l < a.l_lo) continue; // uniform across the block
-            // ---- one partition round for length l: 4 keys per read
-            uint64_t kk[4];
-            uint32_t dd[4], rk[4];
-            if (valid) {
-                kk[0] = (mix(exact61(st.P0)) & keep) | v0;
-                kk[1] = (mix(exact61(st.S0)) & keep) | tagS | v0;
-                kk[2] = (mix(exact61(st.P1)) & keep) | (v0 + 1);
-                kk[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    dd[q] = bin_of<SPLIT>(kk[q], 56, a.vbits);
-                    rk[q] = atomicAdd(&cnt[dd[q]], 1u);
-                }
-            }
-            __syncthreads();
-            const uint32_t seg = l - a.l_lo;
-            uint32_t c = 0, bs = 0;
-            if (threadIdx.x < NB) {
-                c = cnt[threadIdx.x];
-                cnt[threadIdx.x] = 0;
-                bs = c ? atomicAdd(&a.fill[(uint64_t)seg * NB + threadIdx.x], c) : 0u;
-            }
-            const uint32_t ex = block_scan<NB>(c, wsum);
-            if (threadIdx.x < NB) {
-                lstart[threadIdx.x] = ex;
-                if (threadIdx.x == NB - 1) s_total = ex + c;
-                if ((uint64_t)bs + c > a.cap) {
-                    gofs[threadIdx.x] = -1;
-                    *a.overflow = 1u;
-                } else {
-                    gofs[threadIdx.x] = (long long)(((uint64_t)seg * NB + threadIdx.x) * a.cap + bs) -
-                                        (long long)ex;
-                }
-            }
-            __syncthreads();
-            if (valid) {
-#pragma unroll
-                for (int q = 0; q < 4; ++q) stage[lstart[dd[q]] + rk[q]] = kk[q];
-            }
-            __syncthreads();
-            const uint32_t total = s_total;
-            for (uint32_t t = threadIdx.x; t < total; t += SC_THREADS) {
-                const uint64_t key = stage[t];
-                const long long go = gofs[bin_of<SPLIT>(key, 56, a.vbits)];
-                if (go >= 0) a.out[go + t] = key;
-            }
-            // the next round's first barrier orders these reads before stage/lstart reuse
-        }
-    }
-}
-
-// Two lengths per partition round (non-split level 1): half the barriers, half the scans and
-// reservation atomics of the one-length round; bins k * 256 + digit for the round's k-th length.
-template <int W, bool ASCII>
-__global__ void __launch_bounds__(SC_THREADS, 2)
-scatter_table2_kernel(ScatterArgs a)
-{
-    constexpr int NB = 256, NB2 = 512;
-    __shared__ uint64_t stage[SC_THREADS * 8];
-    __shared__ uint32_t cnt[NB2], lstart[NB2], wsum[16];
-    __shared__ long long gofs[NB2];
-    __shared__ uint32_t s_total;
+    constexpr int NBL = SPLIT ? 512 : 256; // bins per length
+    constexpr int NBIN = LPR * NBL;
+    constexpr int BPT = NBIN / SC_THREADS; // bins per thread in the round's scan
+    constexpr int KPT = 2 * LPR;           // keys per thread per round
+    static_assert(NBIN % SC_THREADS == 0 && BPT >= 1 && BPT <= 4, "bins per thread");
+    // dynamic: stage[SC_THREADS * KPT] keys, then (ASCII) the CTA's staged read bytes
+    extern __shared__ __align__(16) uint64_t stage[];
+    __shared__ uint32_t cnt[NBIN], lstart[NBIN + 1], wsum[16];
+    __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
 
     const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
     const bool valid = i < a.n;
@@ -172,7 +90,7 @@ scatter_table2_kernel(ScatterArgs a)
     if constexpr (ASCII) {
         // a1 fused: stage this CTA's ASCII span (zero-copy from host memory over PCIe when
         // the caller passed page-locked host memory), pack, validate, keep the packed rows
-        extern __shared__ __align__(16) unsigned char sascii[];
+        unsigned char *sascii = reinterpret_cast<unsigned char *>(stage + SC_THREADS * KPT);
         const uint64_t r0 = (uint64_t)blockIdx.x * SC_THREADS;
         const uint64_t r1 = min64(a.n, r0 + SC_THREADS);
         const uint32_t off = stage_ascii(a.ascii, r0 * a.L, r1 * a.L, sascii, SC_THREADS);
@@ -196,16 +114,15 @@ scatter_table2_kernel(ScatterArgs a)
 #pragma unroll
         for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
     }
-    cnt[threadIdx.x] = 0; // NB2 == SC_THREADS
+    for (uint32_t t = threadIdx.x; t < NBIN; t += SC_THREADS) cnt[t] = 0;
     __syncthreads();
-    const uint64_t keep = ~((2ull << a.vbits) - 1);
-    const uint64_t tagS = 1ull << a.vbits;
+    const uint64_t keep = key_keep(a.vbits);
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
     st.init();
-    uint64_t k0[4], k1[4];
-    uint32_t r0[4], r1[4];
-    uint32_t kc = 0, lfirst = 0; // keys buffered this round (block-uniform)
+    uint64_t kk[KPT];
+    uint32_t rk[KPT];
+    uint32_t kc = 0, lfirst = 0; // lengths buffered this round (block-uniform)
 #pragma unroll
     for (int w = 0; w < W; ++w) {
         uint64_t xa = x[w], yb = y[w];
@@ -217,66 +134,77 @@ scatter_table2_kernel(ScatterArgs a)
             xa >>= 2;
             yb >>= 2;
             const uint32_t l = kb + j + 1;
-            if (l < a.l_lo) continue;
-            if (kc == 0) {
-                lfirst = l;
-                if (valid) {
-                    k0[0] = (mix(exact61(st.P0)) & keep) | v0;
-                    k0[1] = (mix(exact61(st.S0)) & keep) | tagS | v0;
-                    k0[2] = (mix(exact61(st.P1)) & keep) | (v0 + 1);
-                    k0[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
+            if (l < a.l_lo) continue; // uniform across the block
+            if (kc == 0) lfirst = l;
+            if (valid) {
+                const uint64_t e0 = canon_key(st.P0, st.S1, keep, a.vbits, v0);
+                const uint64_t e1 = canon_key(st.P1, st.S0, keep, a.vbits, v0 + 1);
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) r0[q] = atomicAdd(&cnt[(uint32_t)(k0[q] >> 56)], 1u);
-                }
-            } else {
-                if (valid) {
-                    k1[0] = (mix(exact61(st.P0)) & keep) | v0;
-                    k1[1] = (mix(exact61(st.S0)) & keep) | tagS | v0;
-                    k1[2] = (mix(exact61(st.P1)) & keep) | (v0 + 1);
-                    k1[3] = (mix(exact61(st.S1)) & keep) | tagS | (v0 + 1);
-#pragma unroll
-                    for (int q = 0; q < 4; ++q)
-                        r1[q] = atomicAdd(&cnt[NB + (uint32_t)(k1[q] >> 56)], 1u);
-                }
+                for (int q = 0; q < LPR; ++q)
+                    if ((uint32_t)q == kc) { // constant register indices after unrolling
+                        kk[2 * q] = e0;
+                        kk[2 * q + 1] = e1;
+                        rk[2 * q] = atomicAdd(&cnt[q * NBL + bin_of<SPLIT>(e0, 56, a.vbits)], 1u);
+                        rk[2 * q + 1] = atomicAdd(&cnt[q * NBL + bin_of<SPLIT>(e1, 56, a.vbits)], 1u);
+                    }
             }
             ++kc;
-            if (kc < 2 && l < a.l_hi) continue;
+            if (kc < (uint32_t)LPR && l < a.l_hi) continue;
             // ---- partition round for lengths lfirst .. lfirst + kc - 1
             __syncthreads();
-            const uint32_t t = threadIdx.x; // one bin per thread
-            const uint32_t c = cnt[t];
-            cnt[t] = 0;
-            const uint32_t seg = lfirst - a.l_lo + t / NB;
-            const uint32_t d = t % NB;
-            const uint32_t bs =
-                (c && (t / NB) < kc) ? atomicAdd(&a.fill[(uint64_t)seg * NB + d], c) : 0u;
-            const uint32_t ex = block_scan<NB2>(c, wsum);
-            lstart[t] = ex;
-            if (t == NB2 - 1) s_total = ex + c;
-            if ((uint64_t)bs + c > a.cap) {
-                gofs[t] = -1;
-                *a.overflow = 1u;
-            } else {
-                gofs[t] = (long long)(((uint64_t)seg * NB + d) * a.cap + bs) - (long long)ex;
+            uint32_t c[BPT], bs[BPT], sum = 0;
+#pragma unroll
+            for (int b = 0; b < BPT; ++b) {
+                const uint32_t bin = threadIdx.x * BPT + b;
+                c[b] = cnt[bin];
+                cnt[bin] = 0;
+                const uint32_t q = bin / NBL;
+                bs[b] = (c[b] && q < kc)
+                            ? atomicAdd(&a.fill[(uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL], c[b])
+                            : 0u;
+                sum += c[b];
             }
+            uint32_t run = block_scan<SC_THREADS>(sum, wsum);
+#pragma unroll
+            for (int b = 0; b < BPT; ++b) {
+                const uint32_t bin = threadIdx.x * BPT + b;
+                const uint32_t q = bin / NBL;
+                lstart[bin] = run;
+                if ((uint64_t)bs[b] + c[b] > a.cap) {
+                    gofs[bin] = -1;
+                    *a.overflow = 1u;
+                } else {
+                    gofs[bin] = (long long)(((uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL) * a.cap +
+                                            bs[b]) - (long long)run;
+                }
+                run += c[b];
+            }
+            if (threadIdx.x == SC_THREADS - 1) lstart[NBIN] = run;
             __syncthreads();
             if (valid) {
 #pragma unroll
-                for (int q = 0; q < 4; ++q) stage[lstart[(uint32_t)(k0[q] >> 56)] + r0[q]] = k0[q];
-                if (kc == 2) {
-#pragma unroll
-                    for (int q = 0; q < 4; ++q)
-                        stage[lstart[NB + (uint32_t)(k1[q] >> 56)] + r1[q]] = k1[q];
-                }
+                for (int q = 0; q < LPR; ++q)
+                    if ((uint32_t)q < kc) {
+                        stage[lstart[q * NBL + bin_of<SPLIT>(kk[2 * q], 56, a.vbits)] + rk[2 * q]] = kk[2 * q];
+                        stage[lstart[q * NBL + bin_of<SPLIT>(kk[2 * q + 1], 56, a.vbits)] + rk[2 * q + 1]] =
+                            kk[2 * q + 1];
+                    }
             }
             __syncthreads();
-            const uint32_t total = s_total, mid = lstart[NB];
+            const uint32_t total = lstart[NBIN];
+            uint32_t bnd[LPR]; // first stage slot of each length's bins
+#pragma unroll
+            for (int q = 0; q < LPR; ++q) bnd[q] = lstart[q * NBL];
             for (uint32_t u = threadIdx.x; u < total; u += SC_THREADS) {
                 const uint64_t key = stage[u];
-                const long long go = gofs[(u >= mid ? NB : 0) + (uint32_t)(key >> 56)];
+                uint32_t q = 0;
+#pragma unroll
+                for (int k = 1; k < LPR; ++k) q += u >= bnd[k];
+                const long long go = gofs[q * NBL + bin_of<SPLIT>(key, 56, a.vbits)];
                 if (go >= 0) a.out[go + u] = key;
             }
             kc = 0;
+            // the next round's first barrier orders these reads before stage/lstart reuse
         }
     }
 }
@@ -286,21 +214,21 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
     if (args.n == 0) return LASAGNA_OK;
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const uint64_t blocks = ceil_div(args.n, SC_THREADS);
-        static const bool one_length = getenv("LASAGNA_SCATTER_LPR1") != nullptr;
+        const unsigned blocks = (unsigned)ceil_div(args.n, SC_THREADS);
+        const size_t ascii_b = args.ascii ? (size_t)SC_THREADS * args.L + 16 : 0;
+        auto run = [&](auto kern, int lpr) -> lasagna_status {
+            const size_t smem = (size_t)SC_THREADS * 2 * lpr * 8 + ascii_b;
+            LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)smem));
+            kern<<<blocks, SC_THREADS, smem, s>>>(args);
+            LSG_LAUNCHED("scatter_table_kernel");
+            return LASAGNA_OK;
+        };
         if (args.split)
-            scatter_table_kernel<W, true><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
-        else if (one_length)
-            scatter_table_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
-        else if (args.ascii) {
-            const size_t smem = (size_t)SC_THREADS * args.L + 16;
-            LSG_CUDA(cudaFuncSetAttribute(scatter_table2_kernel<W, true>,
-                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            scatter_table2_kernel<W, true><<<(unsigned)blocks, SC_THREADS, smem, s>>>(args);
-        } else
-            scatter_table2_kernel<W, false><<<(unsigned)blocks, SC_THREADS, 0, s>>>(args);
-        LSG_LAUNCHED("scatter_table_kernel");
-        return LASAGNA_OK;
+            return args.ascii ? run(scatter_table_kernel<W, true, true, 1>, 1)
+                              : run(scatter_table_kernel<W, false, true, 1>, 1);
+        return args.ascii ? run(scatter_table_kernel<W, true, false, 4>, 4)
+                          : run(scatter_table_kernel<W, false, false, 4>, 4);
     });
 }
 
@@ -438,15 +366,19 @@ struct WinDesc {
     uint32_t first;                  // first bucket (index within the chunk)
 };
 
+// one bucket with a half larger than a staging buffer (massively repeated fingerprints),
+// joined in global memory: every probe entry (the probe half, plus flag-2 entries of the build
+// half) scans the build half
 template <int W>
 __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const uint64_t *P,
                                                      uint32_t nP, const uint64_t *S, uint32_t nS,
                                                      Stager &em, unsigned long long &nfalse)
 {
-    const uint32_t kshift = a.vbits + 1;
+    const uint32_t kshift = a.vbits + FLAG_BITS;
     const uint64_t vmask = (1ull << a.vbits) - 1;
-    for (uint32_t i = threadIdx.x; i < nS; i += JOIN_THREADS) {
-        const uint64_t e = S[i];
+    for (uint32_t i = threadIdx.x; i < nS + nP; i += JOIN_THREADS) {
+        const uint64_t e = i < nS ? S[i] : P[i - nS];
+        if (i >= nS && key_flag(e, a.vbits) != 2) continue;
         for (uint32_t j = 0; j < nP; ++j) {
             const uint64_t p = P[j];
             if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
@@ -467,15 +399,16 @@ bucket_join_kernel(BucketJoinArgs b)
     uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
     __shared__ WinDesc wd[2];
     __shared__ __align__(8) unsigned long long mbar[2];
-    __shared__ uint32_t bcount, vdone, s_k[2];
+    __shared__ uint32_t bcount, vdone, s_k[2], s_has2[2];
     const JoinArgs &a = b.j;
     const uint64_t nbk = b.n_buckets;
     const uint64_t b0 = nbk * blockIdx.x / gridDim.x, b1 = nbk * (blockIdx.x + 1) / gridDim.x;
-    const uint32_t kshift = a.vbits + 1;
+    const uint32_t kshift = a.vbits + FLAG_BITS;
     const uint64_t vmask = (1ull << a.vbits) - 1;
-    const uint64_t tagbit = 1ull << a.vbits;
+    const uint64_t tagbit = 1ull << a.vbits;      // half bit: 0 build side, 1 probe side
+    const uint64_t flag2bit = 2ull << a.vbits;
     if (threadIdx.x == 0) {
-        bcount = 0, vdone = 0;
+        bcount = 0, vdone = 0, s_has2[0] = 0, s_has2[1] = 0;
         mbar_init(&mbar[0], 1);
         mbar_init(&mbar[1], 1);
         fence_mbar_init();
@@ -577,20 +510,31 @@ bucket_join_kernel(BucketJoinArgs b)
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
+                    if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
                     const uint32_t h = (uint32_t)(e >> kshift) & (BJ_SLOTS - 1);
                     const uint32_t old = atomicExch(&slot[h], tag | k2);
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
                 __syncthreads();
-                for (uint32_t t = threadIdx.x; t < nS; t += JOIN_THREADS) {
-                    const uint64_t e = S[t];
-                    if (!(e & tagbit)) continue; // sentinel
+                if (threadIdx.x == 0) s_has2[w ^ 1] = 0u; // the other window's flag is stale
+                auto probe = [&](uint64_t e) {
                     const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
                     uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
                     while (sl != 0xFFFFu) {
                         const uint64_t p = P[sl];
                         if (((p ^ e) >> kshift) == 0) candidate<W>(a, e, p, vmask, em, nfalse);
                         sl = next[sl];
+                    }
+                };
+                for (uint32_t t = threadIdx.x; t < nS; t += JOIN_THREADS) {
+                    const uint64_t e = S[t];
+                    if (!(e & tagbit)) continue; // sentinel
+                    probe(e);
+                }
+                if (s_has2[w]) { // block-uniform
+                    for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
+                        const uint64_t e = P[k2];
+                        if ((e & (tagbit | flag2bit)) == flag2bit) probe(e);
                     }
                 }
             }

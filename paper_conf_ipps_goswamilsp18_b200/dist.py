@@ -61,7 +61,7 @@ class CudaBackend:
 
     def table_keys(self, packed_local, n_local, read_offset, n_total, L, l_lo, l_hi):
         G = l_hi - l_lo + 1
-        tab = torch.empty((G, 4 * n_local), dtype=torch.int64, device=self.device)
+        tab = torch.empty((G, 2 * n_local), dtype=torch.int64, device=self.device)
         f = self.L.lasagna_table_keys
         f.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
                       ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p,
@@ -207,7 +207,7 @@ def greedy_graph(ascii_local: torch.Tensor, n_total: int, L: int, l_min: int, ba
         Gc = l_hi - l_lo + 1
         # 2-3. local table, partitioned by destination hash range
         tab = be.table_keys(packed_local, n_local, lo, n_total, L, l_lo, l_hi)
-        seg = 4 * n_local
+        seg = 2 * n_local
         be.sort_segments(tab, seg, Gc, 64 - DEST_BITS, 64)
         cnt = be.digit_counts(tab, seg, Gc, 64 - DEST_BITS, DEST_BITS)          # [Gc, 256]
         send_counts = torch.zeros((Gc, world), dtype=torch.int64)

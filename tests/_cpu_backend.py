@@ -33,25 +33,28 @@ class CpuBackend:
 
     def sort_bits(self, n_total):
         vb = self.vertex_bits(n_total)
-        N = 4 * n_total
+        N = 2 * n_total  # one canonical entry per vertex and length
         P = math.ceil((math.log2(N) - 11.5) / 8) if N > 1 else 1
-        return min(8 * max(1, min(P, 4)), 63 - vb)
+        return min(8 * max(1, min(P, 4)), 62 - vb)
 
     def table_keys(self, packed_local, n_local, read_offset, n_total, L, l_lo, l_hi):
+        """Canonical entries (include/lasagna.h): per vertex v and length l, with
+        H = F(prefix_l(v)) and Hr = F(RC(prefix_l(v))) = F(suffix_l(v ^ 1)):
+        key = mix(min(H, Hr)) top bits | flag << vbits | v, flag 0 (H < Hr) / 1 (>) / 2 (=)."""
         vb = self.vertex_bits(n_total)
-        keep = np.uint64(~((2 << vb) - 1) & 0xFFFFFFFFFFFFFFFF)
+        keep = np.uint64(~((4 << vb) - 1) & 0xFFFFFFFFFFFFFFFF)
         G = l_hi - l_lo + 1
-        out = np.zeros((G, 4 * n_local), dtype=np.uint64)
+        out = np.zeros((G, 2 * n_local), dtype=np.uint64)
         if n_local:
             pfx, sfx = oracle.fingerprints(self.reads[read_offset:read_offset + n_local], l_lo)
             v = (2 * (read_offset + np.arange(n_local, dtype=np.uint64)))
             for s in range(G):
                 for o in (0, 1):
-                    vv = v + np.uint64(o)
-                    pk = (pfx[s, o::2] * MIX) & keep | vv
-                    sk = (sfx[s, o::2] * MIX) & keep | np.uint64(1 << vb) | vv
-                    out[s, 2 * o::4] = pk
-                    out[s, 2 * o + 1::4] = sk
+                    H = pfx[s, o::2]
+                    Hr = sfx[s, (o ^ 1)::2]  # RC of the prefix of r (r') is the suffix of r' (r)
+                    c = np.minimum(H, Hr)
+                    f = np.where(H < Hr, 0, np.where(H > Hr, 1, 2)).astype(np.uint64)
+                    out[s, o::2] = ((c * MIX) & keep) | (f << np.uint64(vb)) | (v + np.uint64(o))
         return torch.from_numpy(out.view(np.int64))
 
     def sort_segments(self, keys, seg_len, n_seg, lo, hi):
@@ -76,15 +79,17 @@ class CpuBackend:
         return torch.zeros(max(1, capacity), dtype=torch.int64), torch.zeros(2, dtype=torch.int64)
 
     def join(self, keys, count, packed_all, n_total, L, l, pairs, counters):
+        """Build side: flags 0/2; probe side: flags 1/2; a match (probe w, build v) is the
+        read-end pair {w^1, v^1} if suffix_l(seq(w^1)) == prefix_l(seq(v))."""
         vb = self.vertex_bits(n_total)
         k = keys.numpy().view(np.uint64)[:count]
-        kb = k >> np.uint64(vb + 1)
-        tag = (k >> np.uint64(vb)) & np.uint64(1)
-        vid = (k & np.uint64((1 << vb) - 1)).astype(np.int64)
-        byk: dict[int, list[int]] = {}
-        for key, t, v in zip(kb.tolist(), tag.tolist(), vid.tolist()):
-            if t == 0:
-                byk.setdefault(key, []).append(v)
+        kb = (k >> np.uint64(vb + 2)).tolist()
+        flag = ((k >> np.uint64(vb)) & np.uint64(3)).tolist()
+        vid = (k & np.uint64((1 << vb) - 1)).astype(np.int64).tolist()
+        byk: dict[int, list[tuple[int, int]]] = {}
+        for key, f, v in zip(kb, flag, vid):
+            if f != 1:
+                byk.setdefault(key, []).append((v, f))
         comp = bytes.maketrans(b"ACGT", b"TGCA")
 
         def seq(v):
@@ -92,18 +97,18 @@ class CpuBackend:
             return r[::-1].translate(comp) if v & 1 else r
         pos = int(counters[0])
         nf = 0
-        for key, t, u in zip(kb.tolist(), tag.tolist(), vid.tolist()):
-            if t != 1:
+        for key, fw, w in zip(kb, flag, vid):
+            if fw == 0:
                 continue
-            for v in byk.get(key, []):
-                b = v ^ 1
-                if (u >> 1) == (v >> 1) or u >= b:
+            for v, fv in byk.get(key, []):
+                if (w >> 1) == (v >> 1) or (fw == 2 and fv == 2 and w > v):
                     continue
-                if seq(u)[L - l:] != seq(v)[:l]:
+                a, b = sorted((w ^ 1, v ^ 1))
+                if seq(w ^ 1)[L - l:] != seq(v)[:l]:
                     nf += 1
                     continue
                 if pos < pairs.numel():
-                    pairs[pos] = (u << 32) | b
+                    pairs[pos] = (a << 32) | b
                 pos += 1
         counters[0] = pos
         counters[1] += nf
