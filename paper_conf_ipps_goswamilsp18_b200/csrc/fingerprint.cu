@@ -27,8 +27,7 @@ fp_values_kernel(const uint64_t *__restrict__ packed, uint64_t n, uint32_t L, ui
         uint64_t x[W], y[W];
         load_read<W>(packed, stride, i, x);
         rc_words<W>(x, L, y);
-        roll_read<W>(x, y, L, [&](uint32_t l, const FpStreams &st) {
-            if (l < l_min) return;
+        roll_read<W>(x, y, l_min, L, [&](uint32_t l, const FpStreams &st) {
             const uint64_t off = (uint64_t)(l - l_min) * V + 2 * i;
             if (pfx)
                 *reinterpret_cast<ulonglong2 *>(pfx + off) =
@@ -81,8 +80,7 @@ table_kernel(TableArgs a)
         uint64_t x[W], y[W];
         load_read<W>(a.packed, a.stride, i, x);
         rc_words<W>(x, a.L, y);
-        roll_read<W>(x, y, a.l_hi, [&](uint32_t l, const FpStreams &st) {
-            if (l < a.l_lo) return;
+        roll_read<W>(x, y, a.l_lo, a.l_hi, [&](uint32_t l, const FpStreams &st) {
             const uint32_t s = l - a.l_lo;
             const uint64_t v0 = 2 * (a.read_offset + i); // global vertex ids
             const uint64_t e0 = canon_key(st.P0, st.S1, keep, a.vbits, v0);

@@ -44,24 +44,99 @@ struct FpStreams {
     }
 };
 
-// Visit lengths l = 1..l_end; call emit(l, st) after base l-1 (values folded: use exact61).
+// ---- absorbing a read's leading bases without per-base modular steps
+// Lengths below the first one a kernel emits need no intermediate values, only the stream
+// states after them, so whole 16-base half-words are absorbed in 8-base chunks: the chunk's
+// Horner value (< 5^8 < 2^19) takes one 32-bit multiply-add per base, and the stream advances
+// by one modular multiplication per chunk: P <- P * 5^8 + V (prefix streams, bases in read
+// order) and S <- S * 5^8 + V (ascending-power streams, evaluated by Horner from the highest
+// base down: sum_{j<m} c_j 5^j = (...(c_{m-1} 5 + c_{m-2}) 5 + ...) 5 + c_0).
+
+// P * m mod q for P < 2^62 and m < 2^32, folded (< 2^61 + 8): P m = hi 2^32 + lo with
+// hi 2^32 = (hi >> 29) 2^61 + (hi mod 2^29) 2^32 == (hi >> 29) + (hi mod 2^29) 2^32.
+__device__ __forceinline__ uint64_t mulsmall61(uint64_t P, uint32_t m)
+{
+    const uint64_t lo = (uint64_t)(uint32_t)P * m;
+    const uint64_t hi = (uint64_t)(uint32_t)(P >> 32) * m;
+    return fold61(fold61(lo) + ((hi & 0x1FFFFFFFull) << 32) + (hi >> 29));
+}
+constexpr uint32_t POW5_8 = 390625u;
+// Horner value of the 8 bases in the low 16 bits of h: base 0 (lowest bits) most significant
+__device__ __forceinline__ uint32_t chunk8_fwd(uint32_t h)
+{
+    uint32_t v = 0;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) v = v * 5u + ((h >> (2 * t)) & 3u);
+    return v;
+}
+// ... base 7 (highest bits) most significant
+__device__ __forceinline__ uint32_t chunk8_bwd(uint32_t h)
+{
+    uint32_t v = 0;
+#pragma unroll
+    for (int t = 7; t >= 0; --t) v = v * 5u + ((h >> (2 * t)) & 3u);
+    return v;
+}
+
+// Stream states after the first 16 * nh bases of r (x) and r' (y), nh <= 2W (block-uniform).
+template <int W>
+__device__ __forceinline__ void fp_skip(const uint64_t (&x)[W], const uint64_t (&y)[W], uint32_t nh,
+                                        FpStreams &st)
+{
+    uint64_t P0 = 0, P1 = 0, S0 = 0, S1 = 0;
+#pragma unroll
+    for (int h = 0; h < 2 * W; ++h) {
+        if ((uint32_t)h >= nh) break;
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1)));
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1)));
+        P0 = mulsmall61(P0, POW5_8) + chunk8_fwd(hx);
+        P0 = mulsmall61(P0, POW5_8) + chunk8_fwd(hx >> 16);
+        P1 = mulsmall61(P1, POW5_8) + chunk8_fwd(hy);
+        P1 = mulsmall61(P1, POW5_8) + chunk8_fwd(hy >> 16);
+    }
+#pragma unroll
+    for (int h = 2 * W - 1; h >= 0; --h) {
+        if ((uint32_t)h >= nh) continue;
+        // ascending-power streams consume the complemented bases (c ^ 2)
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        S1 = mulsmall61(S1, POW5_8) + chunk8_bwd(hx >> 16);
+        S1 = mulsmall61(S1, POW5_8) + chunk8_bwd(hx);
+        S0 = mulsmall61(S0, POW5_8) + chunk8_bwd(hy >> 16);
+        S0 = mulsmall61(S0, POW5_8) + chunk8_bwd(hy);
+    }
+    st.P0 = fold61(P0), st.P1 = fold61(P1), st.S0 = fold61(S0), st.S1 = fold61(S1);
+}
+
+// half-words a kernel whose first emitted length is l_first can absorb (bases < l_first - 1)
+__host__ __device__ __forceinline__ uint32_t skip_halves(uint32_t l_first)
+{
+    return l_first > 1 ? (l_first - 1) / 16 : 0;
+}
+
+// Visit lengths l = l_first..l_end; call emit(l, st) after base l-1 (values folded: use
+// exact61).  The bases before the first 16-base boundary <= l_first - 1 are absorbed by fp_skip.
 template <int W, typename Emit>
 __device__ __forceinline__ void roll_read(const uint64_t (&x)[W], const uint64_t (&y)[W],
-                                          uint32_t l_end, Emit &&emit)
+                                          uint32_t l_first, uint32_t l_end, Emit &&emit)
 {
     FpStreams st;
-    st.init();
+    const uint32_t nh = min(skip_halves(l_first), 2u * W);
+    fp_skip<W>(x, y, nh, st);
+    const uint32_t kskip = 16u * nh;
 #pragma unroll
     for (int w = 0; w < W; ++w) {
-        uint64_t a = x[w], b = y[w];
         const uint32_t k0 = 32u * w;
         if (k0 >= l_end) break;
+        if (k0 + 32u <= kskip) continue;
+        const uint32_t j0 = kskip > k0 ? kskip - k0 : 0u; // 0 or 16
+        uint64_t a = x[w] >> (2 * j0), b = y[w] >> (2 * j0);
         const uint32_t kn = min(32u, l_end - k0);
-        for (uint32_t j = 0; j < kn; ++j) {
+        for (uint32_t j = j0; j < kn; ++j) {
             st.step((uint32_t)(a & 3u), (uint32_t)(b & 3u), k0 + j);
             a >>= 2;
             b >>= 2;
-            emit(k0 + j + 1, st);
+            if (k0 + j + 1 >= l_first) emit(k0 + j + 1, st);
         }
     }
 }

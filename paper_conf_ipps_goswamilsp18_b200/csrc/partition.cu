@@ -119,17 +119,21 @@ scatter_table_kernel(ScatterArgs a)
     const uint64_t keep = key_keep(a.vbits);
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
-    st.init();
+    const uint32_t nh = min(skip_halves(a.l_lo), 2u * W); // leading bases absorbed in chunks
+    fp_skip<W>(x, y, nh, st);
+    const uint32_t kskip = 16u * nh;
     uint64_t kk[KPT];
     uint32_t rk[KPT];
     uint32_t kc = 0, lfirst = 0; // lengths buffered this round (block-uniform)
 #pragma unroll
     for (int w = 0; w < W; ++w) {
-        uint64_t xa = x[w], yb = y[w];
         const uint32_t kb = 32u * w;
         if (kb >= a.l_hi) break;
+        if (kb + 32u <= kskip) continue;
+        const uint32_t j0 = kskip > kb ? kskip - kb : 0u; // 0 or 16
+        uint64_t xa = x[w] >> (2 * j0), yb = y[w] >> (2 * j0);
         const uint32_t kn = min(32u, a.l_hi - kb);
-        for (uint32_t j = 0; j < kn; ++j) {
+        for (uint32_t j = j0; j < kn; ++j) {
             st.step((uint32_t)(xa & 3u), (uint32_t)(yb & 3u), kb + j);
             xa >>= 2;
             yb >>= 2;
