@@ -24,10 +24,26 @@ __device__ __forceinline__ unsigned long long proposal(uint32_t epoch, uint32_t 
     return ((unsigned long long)epoch << 32) | (unsigned long long)(~partner);
 }
 
-__global__ void greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
-                               unsigned long long cap, const uint8_t *claimed,
-                               unsigned long long *best, uint32_t epoch,
-                               unsigned long long *out_count, unsigned long long *book)
+// Both round kernels are bound by the latency of random accesses (claimed[], best[] over
+// 2n read ends): each thread handles GK pairs per trip and issues all their loads before
+// using any, so a warp keeps 4x more random requests in flight.
+constexpr int GREEDY_THREADS = 256;
+constexpr int GK = 4;
+
+// claimed read ends: a bitmap of 2n bits (8.7 MB at cfg3: L2-resident, unlike a byte per end)
+__device__ __forceinline__ bool is_claimed(const uint32_t *cl, uint32_t x)
+{
+    return (cl[x >> 5] >> (x & 31u)) & 1u;
+}
+__device__ __forceinline__ void set_claimed(uint32_t *cl, uint32_t x)
+{
+    atomicOr(&cl[x >> 5], 1u << (x & 31u));
+}
+
+__global__ void __launch_bounds__(GREEDY_THREADS)
+greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
+               unsigned long long cap, const uint32_t *claimed, unsigned long long *best,
+               uint32_t epoch, unsigned long long *out_count, unsigned long long *book)
 {
     const unsigned long long c = *count;
     const unsigned long long m = c < cap ? c : cap;
@@ -38,47 +54,109 @@ __global__ void greedy_propose(const unsigned long long *pairs, const unsigned l
             atomicMax(&book[2], c);
         }
     }
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const unsigned long long r = pairs[i];
-        const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
-        if (claimed[a] | claimed[b]) continue;
-        atomicMax(&best[a], proposal(epoch, b));
-        atomicMax(&best[b], proposal(epoch, a));
+    const uint64_t stride = (uint64_t)gridDim.x * GREEDY_THREADS * GK;
+    for (uint64_t i0 = (uint64_t)blockIdx.x * GREEDY_THREADS * GK + threadIdx.x; i0 < m; i0 += stride) {
+        unsigned long long r[GK];
+        bool ca[GK], cb[GK];
+#pragma unroll
+        for (int k = 0; k < GK; ++k) {
+            const uint64_t i = i0 + (uint64_t)k * GREEDY_THREADS;
+            r[k] = i < m ? pairs[i] : ~0ull;
+        }
+#pragma unroll
+        for (int k = 0; k < GK; ++k)
+            if (r[k] != ~0ull)
+                ca[k] = is_claimed(claimed, (uint32_t)(r[k] >> 32)), cb[k] = is_claimed(claimed, (uint32_t)r[k]);
+#pragma unroll
+        for (int k = 0; k < GK; ++k) {
+            if (r[k] == ~0ull || (ca[k] | cb[k])) continue;
+            const uint32_t a = (uint32_t)(r[k] >> 32), b = (uint32_t)r[k];
+            atomicMax(&best[a], proposal(epoch, b));
+            atomicMax(&best[b], proposal(epoch, a));
+        }
     }
 }
 
-__device__ __forceinline__ void accept_pair(uint32_t a, uint32_t b, uint8_t *claimed, uint32_t *succ,
+__device__ __forceinline__ void accept_pair(uint32_t a, uint32_t b, uint32_t *claimed, uint32_t *succ,
                                             uint8_t *olen, uint8_t l)
 {
-    claimed[a] = 1, claimed[b] = 1;
+    set_claimed(claimed, a), set_claimed(claimed, b);
     succ[a] = b ^ 1u, succ[b] = a ^ 1u; // edges a -> b^1 and (complement) b -> a^1
     olen[a] = l, olen[b] = l;
 }
 
-__global__ void greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
-                              unsigned long long cap, uint8_t *claimed,
-                              const unsigned long long *best, uint32_t epoch, uint32_t *succ,
-                              uint8_t *olen, uint8_t l, unsigned long long *out,
-                              unsigned long long *out_count, unsigned long long *book)
+// Survivors are appended to `out` with one global atomic per block and loop trip (a
+// per-thread or per-warp atomic on the single counter serialises at L2).
+__global__ void __launch_bounds__(GREEDY_THREADS)
+greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
+              unsigned long long cap, uint32_t *claimed, const unsigned long long *best,
+              uint32_t epoch, uint32_t *succ, uint8_t *olen, uint8_t l, unsigned long long *out,
+              unsigned long long *out_count, unsigned long long *book)
 {
+    __shared__ uint32_t wsum[GREEDY_THREADS / 32];
+    __shared__ unsigned long long sbase;
     const unsigned long long c = *count;
     const unsigned long long m = c < cap ? c : cap;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     uint32_t acc = 0;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const unsigned long long r = pairs[i];
-        const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
-        if (claimed[a] | claimed[b]) continue; // dead: an end was taken in an earlier round
-        if (best[a] == proposal(epoch, b) && best[b] == proposal(epoch, a)) {
-            accept_pair(a, b, claimed, succ, olen, l);
-            ++acc;
-        } else {
-            out[atomicAdd(out_count, 1ull)] = r;
+    const uint64_t stride = (uint64_t)gridDim.x * GREEDY_THREADS * GK;
+    for (uint64_t i0 = (uint64_t)blockIdx.x * GREEDY_THREADS * GK + threadIdx.x;
+         i0 - threadIdx.x < m; i0 += stride) { // block-uniform trip count
+        unsigned long long r[GK], ba[GK], bb[GK];
+        bool ca[GK], cb[GK];
+#pragma unroll
+        for (int k = 0; k < GK; ++k) {
+            const uint64_t i = i0 + (uint64_t)k * GREEDY_THREADS;
+            r[k] = i < m ? pairs[i] : ~0ull;
         }
+#pragma unroll
+        for (int k = 0; k < GK; ++k)
+            if (r[k] != ~0ull)
+                ca[k] = is_claimed(claimed, (uint32_t)(r[k] >> 32)), cb[k] = is_claimed(claimed, (uint32_t)r[k]);
+        // best[] only for live pairs (random 32 B sectors in a 16 B/end array: the traffic that
+        // bounds the round)
+#pragma unroll
+        for (int k = 0; k < GK; ++k)
+            if (r[k] != ~0ull && !(ca[k] | cb[k])) ba[k] = best[(uint32_t)(r[k] >> 32)], bb[k] = best[(uint32_t)r[k]];
+        uint32_t keepm = 0;
+#pragma unroll
+        for (int k = 0; k < GK; ++k) {
+            if (r[k] == ~0ull || (ca[k] | cb[k])) continue; // dead: an end was taken earlier
+            const uint32_t a = (uint32_t)(r[k] >> 32), b = (uint32_t)r[k];
+            if (ba[k] == proposal(epoch, b) && bb[k] == proposal(epoch, a)) {
+                accept_pair(a, b, claimed, succ, olen, l);
+                ++acc;
+            } else {
+                keepm |= 1u << k;
+            }
+        }
+        const uint32_t nk = __popc(keepm);
+        uint32_t x = nk; // warp inclusive scan of the survivor counts
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) wsum[wid] = x;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t tot = 0;
+            for (int w = 0; w < GREEDY_THREADS / 32; ++w) {
+                const uint32_t v = wsum[w];
+                wsum[w] = tot;
+                tot += v;
+            }
+            sbase = tot ? atomicAdd(out_count, (unsigned long long)tot) : 0ull;
+        }
+        __syncthreads();
+        unsigned long long pos = sbase + wsum[wid] + x - nk;
+#pragma unroll
+        for (int k = 0; k < GK; ++k)
+            if (keepm & (1u << k)) out[pos++] = r[k];
+        __syncthreads(); // wsum / sbase reuse
     }
     for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&book[0], (unsigned long long)acc);
+    if (lane == 0 && acc) atomicAdd(&book[0], (unsigned long long)acc);
 }
 
 constexpr int TAIL_MAX = 4096;
@@ -89,7 +167,7 @@ constexpr int FINISH_THREADS = 1024;
 // (a, b) in shared memory, one thread visits the pairs in order).
 __global__ void __launch_bounds__(FINISH_THREADS)
 greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
-              unsigned long long *other, unsigned long long *other_count, uint8_t *claimed,
+              unsigned long long *other, unsigned long long *other_count, uint32_t *claimed,
               unsigned long long *best, uint32_t epoch, uint32_t fast_rounds, uint32_t *succ,
               uint8_t *olen, uint8_t l, unsigned long long *book)
 {
@@ -102,7 +180,7 @@ greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
         for (uint32_t i = threadIdx.x; i < live; i += FINISH_THREADS) {
             const unsigned long long r = cur[i];
             const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
-            if (claimed[a] | claimed[b]) continue;
+            if (is_claimed(claimed, a) || is_claimed(claimed, b)) continue;
             atomicMax(&best[a], proposal(epoch, b));
             atomicMax(&best[b], proposal(epoch, a));
         }
@@ -111,7 +189,7 @@ greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
         for (uint32_t i = threadIdx.x; i < live; i += FINISH_THREADS) {
             const unsigned long long r = cur[i];
             const uint32_t a = (uint32_t)(r >> 32), b = (uint32_t)r;
-            if (claimed[a] | claimed[b]) continue;
+            if (is_claimed(claimed, a) || is_claimed(claimed, b)) continue;
             if (best[a] == proposal(epoch, b) && best[b] == proposal(epoch, a)) {
                 accept_pair(a, b, claimed, succ, olen, l);
                 atomicAdd(&s_acc, 1u);
@@ -149,7 +227,7 @@ greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
             uint32_t acc = 0;
             for (uint32_t i = 0; i < live; ++i) {
                 const uint32_t a = (uint32_t)(s[i] >> 32), b = (uint32_t)s[i];
-                if (claimed[a] | claimed[b]) continue;
+                if (is_claimed(claimed, a) || is_claimed(claimed, b)) continue;
                 accept_pair(a, b, claimed, succ, olen, l);
                 ++acc;
             }
@@ -175,15 +253,15 @@ lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *
 {
     const int sms = num_sms();
     const unsigned blocks = (unsigned)std::max<uint64_t>(
-        1, std::min<uint64_t>(ceil_div(g.cap, 256), (uint64_t)sms * 8));
+        1, std::min<uint64_t>(ceil_div(g.cap, GREEDY_THREADS * GK), (uint64_t)sms * 8));
     unsigned long long *in = g.pool, *out = g.pool2, *cin = g.cnt, *cout = g.cnt2;
     const uint32_t e0 = g.epoch;
     g.epoch += EPOCHS_PER_LENGTH;
     for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
-        greedy_propose<<<blocks, 256, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, cout,
+        greedy_propose<<<blocks, GREEDY_THREADS, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, cout,
                                               r == 0 ? g.book : nullptr);
         LSG_LAUNCHED("greedy_propose");
-        greedy_accept<<<blocks, 256, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, succ, olen,
+        greedy_accept<<<blocks, GREEDY_THREADS, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, succ, olen,
                                              l, out, cout, g.book);
         LSG_LAUNCHED("greedy_accept");
         std::swap(in, out);

@@ -56,46 +56,76 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
         ++nfalse;
         return;
     }
+    if (a.found) atomicAdd(a.found, 1ull);
+    if (a.claimed && (((a.claimed[lo >> 5] >> (lo & 31u)) | (a.claimed[hi >> 5] >> (hi & 31u))) & 1u))
+        return;
     const unsigned long long gs = atomicAdd(sg.count, 1ull);
     if (gs < sg.cap) sg.pairs[gs] = rec;
 }
 
-// verify staged records [from, to) in parallel; rejected ones become ~0
+// verify staged records [from, to) in parallel; rejected ones become ~0.  In greedy mode a
+// verified pair with a claimed read end becomes ~1 (counted as found, not stored).
 template <int W>
 __device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long long *buf,
                                               uint32_t from, uint32_t to, unsigned long long &nfalse)
 {
+    uint32_t nfound = 0;
     for (uint32_t t = from + threadIdx.x; t < to; t += JOIN_THREADS) {
         const unsigned long long rec = buf[t];
         const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
         if (!verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
             buf[t] = ~0ull;
             ++nfalse;
+            continue;
         }
+        ++nfound;
+        if (a.claimed && (((a.claimed[u >> 5] >> (u & 31u)) | (a.claimed[b >> 5] >> (b & 31u))) & 1u))
+            buf[t] = ~1ull;
+    }
+    if (a.found) {
+        for (int o = 16; o; o >>= 1) nfound += __shfl_xor_sync(0xffffffffu, nfound, o);
+        if ((threadIdx.x & 31) == 0 && nfound) atomicAdd(a.found, (unsigned long long)nfound);
     }
 }
 
-// write the accepted staged records [0, m) to the global pool (warp-aggregated slots)
+// write the accepted staged records [0, m) to the global pool: one global atomic per block
+// reserves the block's range (a per-record or per-warp atomic on the single pool counter
+// serialises at L2 — ~86 K warp atomics per length at cfg3).  Called by all threads.
 __device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint32_t m,
                                              unsigned long long *pairs, unsigned long long cap,
                                              unsigned long long *count)
 {
-    const int lane = threadIdx.x & 31;
-    for (uint32_t t0 = 0; t0 < m; t0 += JOIN_THREADS) {
-        const uint32_t t = t0 + threadIdx.x;
-        const unsigned long long rec = t < m ? buf[t] : ~0ull;
-        const bool ok = rec != ~0ull;
-        const uint32_t bal = __ballot_sync(0xffffffffu, ok);
-        unsigned long long base = 0;
-        if (lane == 0 && bal) base = atomicAdd(count, (unsigned long long)__popc(bal));
-        base = __shfl_sync(0xffffffffu, base, 0);
-        if (ok) {
-            const unsigned long long pos = base + __popc(bal & ((1u << lane) - 1));
-            if (pos < cap) pairs[pos] = rec;
+    __shared__ uint32_t fw[JOIN_THREADS / 32];
+    __shared__ unsigned long long fbase;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    uint32_t c = 0;
+    for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS) c += buf[t] < ~1ull;
+    uint32_t x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) fw[wid] = x;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t tot = 0;
+        for (int w = 0; w < JOIN_THREADS / 32; ++w) {
+            const uint32_t v = fw[w];
+            fw[w] = tot;
+            tot += v;
         }
+        fbase = tot ? atomicAdd(count, (unsigned long long)tot) : 0ull;
+    }
+    __syncthreads();
+    unsigned long long pos = fbase + fw[wid] + x - c;
+    for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS) {
+        const unsigned long long rec = buf[t];
+        if (rec >= ~1ull) continue; // rejected (~0) or dead (~1)
+        if (pos < cap) pairs[pos] = rec;
+        ++pos;
     }
 }
-
 
 // hash-join the m staged entries ent[0..m) (whole buckets, both sides mixed); slot tags =
 // (epoch << 16) | index

@@ -54,6 +54,10 @@ struct JoinArgs {
     unsigned long long cap;
     unsigned long long *count; // pool fill (may exceed cap: overflow)
     unsigned long long *false_matches;
+    // greedy mode (may be null): pairs with a read end already claimed by a longer length
+    // (bitmap) are counted in *found but not stored — they can never be accepted
+    const uint32_t *claimed = nullptr;
+    unsigned long long *found = nullptr;
 };
 lasagna_status launch_join(const JoinArgs &a, cudaStream_t s);
 lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsigned long long *count,
@@ -109,7 +113,7 @@ struct GreedyBufs {
     unsigned long long *cnt, *cnt2;   // their fills (device)
     unsigned long long *book;         // device: [0] accepted, [1] sum |P_l|, [2] max |P_l|, [3] max rounds
     unsigned long long *best;         // u64 [V]: epoch-tagged proposals, zeroed once per call
-    uint8_t *claimed;
+    uint32_t *claimed;                // bitmap of claimed read ends (2n bits)
     unsigned long long cap;
     uint32_t epoch;                   // next free epoch (host side)
 };

@@ -100,7 +100,8 @@ struct Layout {
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
-enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR64_N = 8 };
+enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR_FOUND = 8,
+       CTR64_N = 9 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -130,7 +131,7 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     l.pool2 = take(pool_cap * 8);
     if (greedy) {
         l.best = take(g.V * 8);
-        l.claimed = take(g.V);
+        l.claimed = take(ceil_div(g.V, 32) * 4);
     } else {
         l.best = l.claimed = 0; // overlaps: pairs sorted in pool/pool2
     }
@@ -200,6 +201,7 @@ struct Run {
     uint32_t *fill1, *fill2;
     unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
+    const uint32_t *claimed = nullptr; // greedy mode: the join drops pairs with a claimed end
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
     void bind(void *workspace)
     {
@@ -354,6 +356,18 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
     return LASAGNA_OK;
 }
 
+// LASAGNA_JOIN_FILTER=1: the join drops pairs with an end claimed by a longer length (counted,
+// not stored).  Off by default: measured at cfg3 the claimed-bit reads cost the join more
+// (+2.5 ms) than the smaller pool saves the greedy (-1.2 ms); the greedy drops them instead.
+static bool join_filter()
+{
+    static const bool on = [] {
+        const char *e = getenv("LASAGNA_JOIN_FILTER");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
 // Join (search + verify) of length l into the pool; if m_out, synchronise and report the
 // pair count.
 static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, uint32_t l_lo,
@@ -375,6 +389,8 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.cap = r.lay.pool_cap;
     ja.count = r.ctr64 + CTR_POOL;
     ja.false_matches = r.ctr64 + CTR_FALSE;
+    ja.claimed = join_filter() ? r.claimed : nullptr;
+    ja.found = ja.claimed ? r.ctr64 + CTR_FOUND : nullptr;
     lasagna_status rc;
     if (r.bucketed) {
         BucketJoinArgs bj;
@@ -576,7 +592,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     r.lay = layout(g, G, cap, true);
     r.s = s;
     r.bind(workspace);
-    uint8_t *claimed = r.at<uint8_t>(r.lay.claimed);
+    uint32_t *claimed = r.at<uint32_t>(r.lay.claimed);
+    r.claimed = claimed;
     if (ascii_dev) {
         // a1: fused into the first partition pass when the fast path runs (T = 16, L <= 160),
         // otherwise a separate pack launch
@@ -618,7 +635,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     LSG_CUDA(cudaMemsetAsync(r.ctr64, 0, CTR64_N * sizeof(unsigned long long), s));
     LSG_CUDA(cudaMemsetAsync(succ, 0xFF, g.V * 4, s));
     LSG_CUDA(cudaMemsetAsync(olen, 0, g.V, s));
-    LSG_CUDA(cudaMemsetAsync(claimed, 0, g.V, s));
+    LSG_CUDA(cudaMemsetAsync(claimed, 0, ceil_div(g.V, 32) * 4, s));
     LSG_CUDA(cudaMemsetAsync(gb.best, 0, g.V * 8, s));
 
     // Everything below is stream-ordered with no host round trip: the join of length l and
@@ -631,8 +648,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         ++st.passes;
         for (int64_t l = l_hi; l >= (int64_t)l_lo; --l) {
             if ((rc = tm.start(PH_SEARCH)) != LASAGNA_OK) return rc;
-            // no pruning: the claimed bits are not consulted, so every length's full pair
-            // list is found (|P| = overlap edges / 2 is reported)
+            // every length's full pair list is found and counted (|P| = overlap edges / 2);
+            // pairs with an end claimed by a longer length are not stored for the greedy
             if ((rc = search_length(r, packed, (uint32_t)l, l_lo, which, nullptr)) != LASAGNA_OK)
                 return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
@@ -662,7 +679,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         return LASAGNA_ENOSPC;
     }
     if (stats) {
-        st.n_pairs = book[1];
+        // every verified pair, including those the join dropped as dead
+        st.n_pairs = join_filter() ? h[CTR_FOUND] : book[1];
         st.n_greedy = book[0];
         st.rounds_max = (uint32_t)book[3];
         st.fp_false_matches = h[CTR_FALSE];
@@ -852,7 +870,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     const size_t o_keys = take(c1 * 8), o_keys2 = take(c1 * 8), o_pool = take(c1 * 8),
                  o_pool2 = take(c1 * 8), o_status = take(sort_status_bytes(c1, 1)),
                  o_ctrs = take(CTR_BYTES), o_hist = take(8 * 256 * 4), o_best = take(V * 8 + 8),
-                 o_claimed = take(V + 1);
+                 o_claimed = take(ceil_div(V, 32) * 4 + 4);
     if (!workspace) {
         *workspace_bytes = off;
         return LASAGNA_OK;
@@ -884,8 +902,8 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     if (rc != LASAGNA_OK) return rc;
     unsigned long long *ctr64 = reinterpret_cast<unsigned long long *>(ws + o_ctrs + 4096 * 4);
     LSG_CUDA(cudaMemsetAsync(ctr64, 0, 8 * 8, s));
-    uint8_t *claimed = reinterpret_cast<uint8_t *>(ws + o_claimed);
-    LSG_CUDA(cudaMemsetAsync(claimed, 0, V, s));
+    uint32_t *claimed = reinterpret_cast<uint32_t *>(ws + o_claimed);
+    LSG_CUDA(cudaMemsetAsync(claimed, 0, ceil_div(V, 32) * 4, s));
     // group by length, descending: key (255 - l) << 56 | i, one 8-bit LSD pass
     uint64_t *keys[2] = {reinterpret_cast<uint64_t *>(ws + o_keys),
                          reinterpret_cast<uint64_t *>(ws + o_keys2)};

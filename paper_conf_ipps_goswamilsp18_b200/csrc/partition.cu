@@ -360,10 +360,12 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 // CTA overwrote beforehand (in global memory) with a sentinel of the wrong tag — ~0 (tag 1)
 // in a prefix half, ~0 ^ (1 << vbits) (tag 0) in a suffix half — so the insert and probe
 // loops skip it by its tag bit alone.  Two barriers per window.
-constexpr int BJ_HALF = 2560;   // staged entries per half per window
+constexpr int BJ_HALF = 2048;   // staged entries per half per window
 constexpr int BJ_MAXB = 64;     // buckets per window
 constexpr int BJ_FILLS = 256;   // buckets whose fills are staged at once
-constexpr int BJ_SLOTS = 4096;
+constexpr int BJ_SLOTS = 4096;  // chain heads (u32 epoch-tagged)
+constexpr int BJ_BLOOM = 2048;  // u32 words: a 64 Ki-bit filter of the build keys, per buffer
+constexpr int BJ_QCAP = 64;     // per-warp queue of probes that passed the filter
 
 struct WinDesc {
     uint32_t nb, nP, nS;             // buckets (0: one oversized bucket), staged slots
@@ -399,7 +401,9 @@ bucket_join_kernel(BucketJoinArgs b)
     uint64_t *sst = pst + 2 * BJ_HALF;                                    // [2][BJ_HALF]
     unsigned long long *buf = reinterpret_cast<unsigned long long *>(sst + 2 * BJ_HALF); // [BUF]
     uint32_t *slot = reinterpret_cast<uint32_t *>(buf + JOIN_BUF);       // [BJ_SLOTS]
-    unsigned short *next = reinterpret_cast<unsigned short *>(slot + BJ_SLOTS); // [BJ_HALF]
+    uint32_t *bloom = slot + BJ_SLOTS;                                    // [2][BJ_BLOOM]
+    unsigned short *queue = reinterpret_cast<unsigned short *>(bloom + 2 * BJ_BLOOM); // [16][QCAP]
+    unsigned short *next = queue + (JOIN_THREADS / 32) * BJ_QCAP;         // [BJ_HALF]
     uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
     __shared__ WinDesc wd[2];
     __shared__ __align__(8) unsigned long long mbar[2];
@@ -418,9 +422,12 @@ bucket_join_kernel(BucketJoinArgs b)
         fence_mbar_init();
     }
     for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+    for (uint32_t t = threadIdx.x; t < 2 * BJ_BLOOM; t += JOIN_THREADS) bloom[t] = 0;
     Stager em{buf, &bcount, a.pairs, a.cap, a.count};
     unsigned long long nfalse = 0;
     uint32_t epoch = 0, phases = 0; // bit w: parity of the next phase of mbar[w]
+    const int lane = threadIdx.x & 31;
+    unsigned short *wq = queue + (threadIdx.x >> 5) * BJ_QCAP; // this warp's probe queue
 
     for (uint64_t c0 = b0; c0 < b1; c0 += BJ_FILLS) {
         const uint32_t nc = (uint32_t)min64(BJ_FILLS, b1 - c0);
@@ -495,6 +502,10 @@ bucket_join_kernel(BucketJoinArgs b)
                 s_k[w ^ 1] = plan(knext, w ^ 1);
             }
             const WinDesc &d = wd[w];
+            // the other filter buffer was last read by window w-1 and is next written by
+            // window w+1 (both across an end-of-window barrier): clear it now
+            static_assert(BJ_BLOOM == 4 * JOIN_THREADS, "one 16-byte store per thread");
+            reinterpret_cast<uint4 *>(bloom + (w ^ 1) * BJ_BLOOM)[threadIdx.x] = make_uint4(0, 0, 0, 0);
             if (d.nb == 0) {
                 const uint64_t bk = c0 + d.first;
                 const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
@@ -509,19 +520,25 @@ bucket_join_kernel(BucketJoinArgs b)
                     __syncthreads();
                 }
                 const uint64_t *P = pst + w * BJ_HALF, *S = sst + w * BJ_HALF;
+                uint32_t *bl = bloom + w * BJ_BLOOM;
                 const uint32_t tag = epoch << 16;
                 const uint32_t nP = d.nP, nS = d.nS;
+                // ---- build: chained hash of the build entries + the 64 Ki-bit filter
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
                     if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
-                    const uint32_t h = (uint32_t)(e >> kshift) & (BJ_SLOTS - 1);
-                    const uint32_t old = atomicExch(&slot[h], tag | k2);
+                    const uint32_t hk = (uint32_t)(e >> kshift);
+                    atomicOr(&bl[(hk & 0xFFFFu) >> 5], 1u << (hk & 31u));
+                    const uint32_t old = atomicExch(&slot[hk & (BJ_SLOTS - 1)], tag | k2);
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
                 __syncthreads();
                 if (threadIdx.x == 0) s_has2[w ^ 1] = 0u; // the other window's flag is stale
-                auto probe = [&](uint64_t e) {
+                // ---- probe: ~95 % of the probe keys miss the filter; the rest are queued per
+                // warp and their chains walked 32 at a time (full warps, no per-lane divergence
+                // between a probe that has a chain and one that has none)
+                auto walk = [&](uint64_t e) {
                     const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
                     uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
                     while (sl != 0xFFFFu) {
@@ -530,17 +547,44 @@ bucket_join_kernel(BucketJoinArgs b)
                         sl = next[sl];
                     }
                 };
-                for (uint32_t t = threadIdx.x; t < nS; t += JOIN_THREADS) {
-                    const uint64_t e = S[t];
-                    if (!(e & tagbit)) continue; // sentinel
-                    probe(e);
+                auto drain = [&](uint32_t from, uint32_t cnt) { // lanes < cnt walk wq[from + lane]
+                    __syncwarp();
+                    const bool act = (uint32_t)lane < cnt;
+                    const uint32_t qi = act ? wq[from + lane] : 0u;
+                    __syncwarp();
+                    if (act) walk((qi & 0x8000u) ? P[qi & 0x7FFFu] : S[qi]);
+                };
+                uint32_t qn = 0; // warp-uniform
+                auto push = [&](bool pass, uint32_t qi) {
+                    const uint32_t m = __ballot_sync(0xffffffffu, pass);
+                    if (pass) wq[qn + __popc(m & ((1u << lane) - 1u))] = (unsigned short)qi;
+                    qn += __popc(m);
+                    if (qn >= 32) {
+                        drain(qn - 32, 32);
+                        qn -= 32;
+                    }
+                };
+                auto passes = [&](uint64_t e) {
+                    const uint32_t hk = (uint32_t)(e >> kshift) & 0xFFFFu;
+                    return ((bl[hk >> 5] >> (hk & 31u)) & 1u) != 0;
+                };
+                for (uint32_t t0 = 0; t0 < nS; t0 += JOIN_THREADS) { // block-uniform trip count
+                    const uint32_t t = t0 + threadIdx.x;
+                    bool pass = false;
+                    if (t < nS) {
+                        const uint64_t e = S[t];
+                        pass = (e & tagbit) && passes(e); // !tagbit: sentinel
+                    }
+                    push(pass, t);
                 }
                 if (s_has2[w]) { // block-uniform
-                    for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
-                        const uint64_t e = P[k2];
-                        if ((e & (tagbit | flag2bit)) == flag2bit) probe(e);
+                    for (uint32_t t0 = 0; t0 < nP; t0 += JOIN_THREADS) {
+                        const uint32_t k2 = t0 + threadIdx.x;
+                        const bool pass = k2 < nP && (P[k2] & (tagbit | flag2bit)) == flag2bit;
+                        push(pass, 0x8000u | k2);
                     }
                 }
+                if (qn) drain(0, qn);
             }
             __syncthreads(); // window w done: its buffers may be refilled
             window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
@@ -559,8 +603,9 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (args.half_cap & 1) return LASAGNA_EINVAL; // sentinels need an even half capacity
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 +
-                            (size_t)BJ_SLOTS * 4 + (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
+        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 + (size_t)BJ_SLOTS * 4 +
+                            (size_t)2 * BJ_BLOOM * 4 + (size_t)(JOIN_THREADS / 32) * BJ_QCAP * 2 +
+                            (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
         LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0;
