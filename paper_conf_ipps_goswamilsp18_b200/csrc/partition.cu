@@ -447,59 +447,76 @@ bucket_join_kernel(BucketJoinArgs b)
         // plan the window starting at chunk bucket k into descriptor w and start its copies
         // (thread 0).  A bucket with a half larger than a staging buffer is a window of its
         // own with nb = 0, joined in global memory.
+        // plan the window starting at chunk bucket k into descriptor w and start its copies.
+        // Run by all 32 lanes of the planning warp: lane j sizes bucket k + j, a warp scan
+        // finds how many whole buckets fit both staging halves, and each lane issues its
+        // bucket's two bulk copies (a serial plan on one thread made its warp the last to
+        // reach the next block barrier).  A bucket with a half larger than a staging buffer is
+        // a window of its own with nb = 0, joined in global memory.
         auto plan = [&](uint32_t k, int w) -> uint32_t {
+            const uint32_t j = k + lane;
+            const bool in = lane < BJ_MAXB && j < nc;
+            const uint32_t pp = in ? (sfill[2 * j] + 1) & ~1u : 0u;
+            const uint32_t ps = in ? (sfill[2 * j + 1] + 1) & ~1u : 0u;
             WinDesc &d = wd[w];
-            d.first = k;
+            const uint32_t bar = smem_u32(&mbar[w]);
             if (sfill[2 * k] > (uint32_t)BJ_HALF || sfill[2 * k + 1] > (uint32_t)BJ_HALF) {
-                d.nb = 0;
+                if (lane == 0) d.first = k, d.nb = 0;
+                __syncwarp();
                 return k + 1;
             }
-            uint32_t nP = 0, nS = 0, nb = 0, e = k;
-            while (e < nc && nb < (uint32_t)BJ_MAXB) {
-                const uint32_t pp = (sfill[2 * e] + 1) & ~1u, ps = (sfill[2 * e + 1] + 1) & ~1u;
-                if (nP + pp > (uint32_t)BJ_HALF || nS + ps > (uint32_t)BJ_HALF) break;
-                nP += pp, nS += ps, ++nb, ++e;
+            uint32_t sp = pp, ss = ps; // inclusive scans
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t yp = __shfl_up_sync(0xffffffffu, sp, o);
+                const uint32_t ys = __shfl_up_sync(0xffffffffu, ss, o);
+                if (lane >= o) sp += yp, ss += ys;
             }
-            d.nb = nb, d.nP = nP, d.nS = nS;
-            const uint32_t bar = smem_u32(&mbar[w]);
-            if (nP + nS) {
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
-                             "r"((nP + nS) * 8)
-                             : "memory");
-                uint32_t oP = 0, oS = 0;
-                for (uint32_t q = 0; q < nb; ++q) {
-                    const uint32_t pp = (sfill[2 * (k + q)] + 1) & ~1u;
-                    const uint32_t ps = (sfill[2 * (k + q) + 1] + 1) & ~1u;
-                    const uint64_t *gb = b.buckets + (c0 + k + q) * 2 * b.half_cap;
-                    if (pp)
-                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
-                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + oP)),
-                                     "l"(gb), "r"(pp * 8), "r"(bar)
-                                     : "memory");
-                    if (ps)
-                        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
-                                     "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(sst + w * BJ_HALF + oS)),
-                                     "l"(gb + b.half_cap), "r"(ps * 8), "r"(bar)
-                                     : "memory");
-                    oP += pp, oS += ps;
-                }
-            } else {
-                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+            const bool fits = in && sp <= (uint32_t)BJ_HALF && ss <= (uint32_t)BJ_HALF;
+            const uint32_t nb = __popc(__ballot_sync(0xffffffffu, fits)); // fits is a lane prefix
+            const uint32_t nP = __shfl_sync(0xffffffffu, sp, nb - 1);
+            const uint32_t nS = __shfl_sync(0xffffffffu, ss, nb - 1);
+            if (lane == 0) {
+                d.first = k, d.nb = nb, d.nP = nP, d.nS = nS;
+                if (nP + nS)
+                    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                                 "r"((nP + nS) * 8)
+                                 : "memory");
+                else
+                    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
             }
-            return e;
+            __syncwarp();
+            if ((uint32_t)lane < nb) {
+                const uint64_t *gb = b.buckets + (c0 + j) * 2 * b.half_cap;
+                if (pp)
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
+                                 "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(pst + w * BJ_HALF + sp - pp)),
+                                 "l"(gb), "r"(pp * 8), "r"(bar)
+                                 : "memory");
+                if (ps)
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"
+                                 "bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(sst + w * BJ_HALF + ss - ps)),
+                                 "l"(gb + b.half_cap), "r"(ps * 8), "r"(bar)
+                                 : "memory");
+            }
+            return k + nb;
         };
-        if (threadIdx.x == 0) {
+        constexpr int PLAN_WARP = JOIN_THREADS / 32 - 1;
+        const bool planner = (threadIdx.x >> 5) == PLAN_WARP;
+        if (planner) {
             fence_proxy_async();
-            s_k[0] = plan(0, 0);
+            const uint32_t kn = plan(0, 0);
+            if (lane == 0) s_k[0] = kn;
         }
         __syncthreads();
         int w = 0;
         uint32_t kcur = 0;
         while (kcur < nc) {
             const uint32_t knext = s_k[w];
-            if (threadIdx.x == 0 && knext < nc) {
+            if (planner && knext < nc) {
                 fence_proxy_async();
-                s_k[w ^ 1] = plan(knext, w ^ 1);
+                const uint32_t kn = plan(knext, w ^ 1);
+                if (lane == 0) s_k[w ^ 1] = kn;
             }
             const WinDesc &d = wd[w];
             // the other filter buffer was last read by window w-1 and is next written by
