@@ -189,18 +189,26 @@ LASAGNA_API lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, c
 /* ---------------------------------------------------------------------------------------
  * Sharded phases: the building blocks of the multi-GPU driver (one process per GPU, tables
  * partitioned by hash range; paper_conf_ipps_goswamilsp18_b200/dist.py).  The key layout is
- * the one lasagna_greedy_graph uses internally for a read set of n_total reads:
- *   key = mix(F) top (63 - vbits) bits | tag << vbits | global vertex id
- *   (tag 0 = prefix entry, 1 = suffix entry; vbits = lasagna_vertex_bits(n_total)),
- * and the join needs the keys of one length sorted by their top lasagna_key_sort_bits(n_total)
- * bits.  A hash-range shard is any set of keys sharing their top bits.
+ * the one lasagna_greedy_graph uses internally for a read set of n_total reads: ONE canonical
+ * entry per oriented read v and length l.  With
+ * x = prefix_l(seq(v)), H = F(x) and Hr = F(RC(x)) (= F(suffix_l(seq(v^1)))):
+ *   key  = mix(min(H, Hr)) top (62 - vbits) bits | flag << vbits | global vertex id
+ *   flag = 0 if H < Hr, 1 if H > Hr, 2 if H == Hr;  mix(f) = f * 0x9E3779B97F4A7C15 mod 2^64;
+ *   vbits = lasagna_vertex_bits(n_total).
+ * The paper's prefix list P_l is the build side (flags 0 and 2), its suffix list S_l
+ * the probe side (flags 1 and 2): suffix_l(seq(u)) == prefix_l(seq(v)) iff the prefixes of
+ * u^1 and v are reverse complements, i.e. equal canonical fingerprints with opposite flags
+ * (or both 2).  The join needs the keys of one length sorted by their top
+ * lasagna_key_sort_bits(n_total) bits.  A hash-range shard is any set of keys sharing their
+ * top bits.
  */
 LASAGNA_API uint32_t lasagna_vertex_bits(uint64_t n_total);
 LASAGNA_API uint32_t lasagna_key_sort_bits(uint64_t n_total);
 
 /* a2/a3 for the reads [read_offset, read_offset + n_local) of an n_total-read set whose packed
- * rows start at `packed`: tab[(l - l_lo) * 4 n_local + 4i + 2o + tag] for l in [l_lo, l_hi]
- * (at most 64 lengths), i local read, o orientation.  Asynchronous. */
+ * rows start at `packed`: tab[(l - l_lo) * 2 n_local + 2i + o] = the canonical key of vertex
+ * 2(read_offset + i) + o at length l, for l in [l_lo, l_hi] (at most 64 lengths), i local read,
+ * o orientation.  Asynchronous. */
 LASAGNA_API lasagna_status lasagna_table_keys(const uint64_t *packed, uint64_t n_local,
                                               uint64_t read_offset, uint64_t n_total, uint32_t L,
                                               uint32_t l_lo, uint32_t l_hi, uint64_t *tab,

@@ -267,6 +267,48 @@ def test_cfg2_parity(lz, seed):
     assert np.array_equal(_np(r.olen, np.uint8), eolen)
 
 
+def _palindrome_rich_reads(seed: int, G: int, n: int, L: int, every: int, plen: int) -> np.ndarray:
+    """Error-free reads (half reverse-complemented) of a random genome in which a reverse-
+    complement palindrome of length plen starts every `every` bases: reads starting at one
+    have palindromic prefixes (H == Hr, flag 2 in the canonical table), so build/probe
+    assignments of flag-2 entries, their double discovery and same-read palindromes are all
+    exercised at a size that runs the two-level (T = 16) bucketed path."""
+    rng = np.random.default_rng(seed)
+    comp = np.zeros(256, dtype=np.uint8)
+    for a, b in zip(b"ACGT", b"TGCA"):
+        comp[a] = b
+    alpha = np.frombuffer(b"ACGT", dtype=np.uint8)
+    g = alpha[rng.integers(0, 4, G)]
+    for s0 in range(0, G - plen, every):
+        half = g[s0:s0 + plen // 2].copy()
+        g[s0 + plen // 2:s0 + plen] = comp[half[::-1]]
+    starts = rng.integers(0, G - L + 1, n)
+    # a third of the reads start exactly on a palindrome
+    k = n // 3
+    starts[:k] = (rng.integers(0, (G - L) // every, k) * every)
+    reads = g[starts[:, None] + np.arange(L)[None, :]]
+    flip = rng.random(n) < 0.5
+    reads[flip] = comp[reads[flip][:, ::-1]]
+    return np.ascontiguousarray(reads)
+
+
+@gpu
+def test_palindrome_rich_parity_two_level(lz):
+    """~1.7 M table entries per length (T = 16: level-1 + level-2 partition, split buckets):
+    overlaps and greedy graph bit-exact vs the oracle on palindrome-rich reads."""
+    import torch
+    reads = _palindrome_rich_reads(7, 4_000_000, 420_000, 40, 37, 20)
+    n, L = reads.shape
+    l_min = 16
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, n, L, l_min)
+    assert r.stats["key_sort_bits"] == 16 and r.stats["bucketed"] == 1
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+
+
 def _random_candidates(n, k, rng, lens):
     V = 2 * n
     k = min(k, len(lens) * V * (V - 1) // 4)  # at most half of all distinct (l, a, b)
@@ -378,6 +420,29 @@ def test_region_overflow_falls_back_to_exact_path(tmp_path):
         "assert pl.numel() == m\n"
         "print('ok')\n")
     env = dict(os.environ, LASAGNA_TEST_TIGHT_REGIONS="1", PYTHONPATH=ROOT)
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                         cwd=ROOT, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+
+
+@gpu
+def test_join_side_dead_pair_filter_option():
+    """LASAGNA_JOIN_FILTER=1 (the join drops pairs with an already claimed end, counting them):
+    same graph and the same |P| as the default path."""
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, torch, readgen, oracle\n"
+        "import paper_conf_ipps_goswamilsp18_b200 as lz\n"
+        "reads = readgen.config_reads('cfg2', n=300000)\n"
+        "packed = lz.load_reads(torch.from_numpy(reads).cuda())\n"
+        "r = lz.greedy_graph(packed, 300000, 100, 63)\n"
+        "es, eo, m, acc = oracle.greedy_graph(reads, 63)\n"
+        "assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), es)\n"
+        "assert np.array_equal(r.olen.cpu().numpy(), eo)\n"
+        "assert r.stats['n_pairs'] == m and r.stats['n_greedy'] == acc\n"
+        "print('ok')\n")
+    env = dict(os.environ, LASAGNA_JOIN_FILTER="1", PYTHONPATH=ROOT)
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                          cwd=ROOT, timeout=600)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
