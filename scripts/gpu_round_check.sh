@@ -5,4 +5,4 @@ python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke
 timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest=$? >> gpurun_out/status.txt
 timeout 900 python bench.py > gpurun_out/bench.log 2>&1; echo bench=$? >> gpurun_out/status.txt
 export BENCH_ALLOW_SHORT_WARMUP=1
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/launches_r01b_cfg3.csv python bench.py --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/launches.log 2>&1; echo ncu=$? >> gpurun_out/status.txt
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/launches_${TAG:-r01e}_cfg3.csv python bench.py --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/launches.log 2>&1; echo ncu=$? >> gpurun_out/status.txt
