@@ -72,4 +72,42 @@ __device__ __forceinline__ bool pack_row_regs(const unsigned char *row, uint32_t
     return !bad;
 }
 
+// The same, four bases per step (SWAR), for a row in shared memory staged by stage_ascii with
+// at least 8 readable bytes after the row end: each step funnel-shifts 4 bytes out of two
+// aligned words; the codes are (byte >> 1) & 3 in every byte lane, and a byte is valid iff
+// (byte | 0x20) equals the lowercase letter its own code names ("a", "c", "t", "g" for codes
+// 0..3), looked up for all four lanes at once with one byte permute.
+template <int W>
+__device__ __forceinline__ bool pack_row_regs_swar(const unsigned char *row, uint32_t L,
+                                                   uint64_t (&x)[W])
+{
+    const uint32_t *p = reinterpret_cast<const uint32_t *>((uintptr_t)row & ~(uintptr_t)3);
+    const uint32_t sh = ((uint32_t)(uintptr_t)row & 3u) * 8u;
+    uint32_t bad = 0, lo = p[0];
+#pragma unroll
+    for (int w = 0; w < W; ++w) x[w] = 0;
+#pragma unroll
+    for (int g = 0; g < 8 * W; ++g) {
+        if (4u * g >= L) break;
+        const uint32_t hi = p[g + 1];
+        const uint32_t c4 = __funnelshift_r(lo, hi, sh); // bytes row[4g .. 4g+3]
+        lo = hi;
+        const uint32_t rem = L - 4u * g;                 // >= 1
+        const uint32_t cx = (c4 >> 1) & 0x03030303u;     // codes, one per byte lane
+        const uint32_t nib = cx | (cx >> 4);             // codes in nibbles 0, 1, 4, 5
+        const uint32_t sel = (nib & 0xFFu) | ((nib >> 8) & 0xFF00u);
+        const uint32_t expect = __byte_perm(0x67746361u, 0u, sel); // 'a' 'c' 't' 'g' by code
+        const uint32_t t = cx | (cx >> 6);               // codes at bits 0-3 and 16-19
+        uint32_t b8 = (t & 0xFu) | ((t >> 12) & 0xF0u);
+        uint32_t diff = (c4 | 0x20202020u) ^ expect;
+        if (rem < 4) {
+            diff &= 0xFFFFFFFFu >> (8u * (4u - rem));
+            b8 &= (1u << (2u * rem)) - 1u;
+        }
+        bad |= diff;
+        x[g >> 3] |= (uint64_t)b8 << (8 * (g & 7));
+    }
+    return bad == 0;
+}
+
 } // namespace lsg

@@ -96,7 +96,7 @@ scatter_table_kernel(ScatterArgs a)
         const uint32_t off = stage_ascii(a.ascii, r0 * a.L, r1 * a.L, sascii, SC_THREADS);
         __syncthreads();
         if (valid) {
-            const bool ok = pack_row_regs<W>(sascii + off + (uint64_t)threadIdx.x * a.L, a.L, x);
+            const bool ok = pack_row_regs_swar<W>(sascii + off + (uint64_t)threadIdx.x * a.L, a.L, x);
             uint64_t *po = a.packed_out + i * a.stride;
 #pragma unroll
             for (int j = 0; j < W; ++j) po[j] = x[j];
@@ -219,7 +219,7 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
     return dispatch_W(args.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
         const unsigned blocks = (unsigned)ceil_div(args.n, SC_THREADS);
-        const size_t ascii_b = args.ascii ? (size_t)SC_THREADS * args.L + 16 : 0;
+        const size_t ascii_b = args.ascii ? (size_t)SC_THREADS * args.L + 32 : 0; // + SWAR overread
         auto run = [&](auto kern, int lpr) -> lasagna_status {
             const size_t smem = (size_t)SC_THREADS * 2 * lpr * 8 + ascii_b;
             LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -496,6 +496,30 @@ def test_greedy_graph_from_ascii(lz, where):
 
 
 @gpu
+@pytest.mark.parametrize("L", [101, 127])
+def test_greedy_graph_from_ascii_unaligned_rows(lz, L):
+    """The fused a1 packs four bases per step from rows that start at any byte offset (L not
+    a multiple of 4): parity with the oracle on mixed-case input, and a bad byte in the last
+    base of a row (the partial final step) or in its first base is reported (R13)."""
+    import torch
+    n, l_min = 400_000, L - 38
+    reads = readgen.reads(7, 2_000_000, n, L, 0.01)
+    mixed = reads.copy()
+    mixed[::3] = np.char.lower(mixed[::3].view(f"S{L}")).view(np.uint8).reshape(-1, L)
+    g = lz.GreedyGraph(n, L, l_min, "cuda")
+    r = g.from_ascii(torch.from_numpy(mixed).pin_memory())
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    assert np.array_equal(_np(g.packed, np.uint64), oracle.pack(reads, lz.words_per_read(L)))
+    for row, col, ch in [(2**17 + 3, L - 1, "N"), (54_321, 0, "x"), (n - 1, L - 1, "@")]:
+        bad = reads.copy()
+        bad[row, col] = ord(ch)
+        with pytest.raises(lz.LasagnaError, match=f"read {row}"):
+            g.from_ascii(torch.from_numpy(bad).cuda())
+
+
+@gpu
 @pytest.mark.slow
 def test_cfg3_full_size_parity_and_invariants(lz):
     """cfg3 (BASELINE configs[2], 34.85 M reads) in the launch configuration bench.py times
