@@ -363,11 +363,9 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 constexpr int BJ_HALF = 2048;   // staged entries per half per window
 constexpr int BJ_MAXB = 64;     // buckets per window
 constexpr int BJ_FILLS = 256;   // buckets whose fills are staged at once
-constexpr int BJ_SLOTS = 1024;  // chain heads (u32 epoch-tagged); only filter survivors enter
-constexpr int BJ_BLOOM = 2048;  // u32 words: a 64 Ki-bit filter (one for build, one for probe keys)
-// per-warp queue of probes that passed the build filter: a warp pushes at most 32 per pass
-// over the probe half plus 32 per pass over the build half (flag-2 entries), so it never fills
-constexpr int BJ_QCAP = 64 * ((BJ_HALF + 511) / 512);
+constexpr int BJ_SLOTS = 4096;  // chain heads (u32 epoch-tagged)
+constexpr int BJ_BLOOM = 2048;  // u32 words: a 64 Ki-bit filter of the build keys, per buffer
+constexpr int BJ_QCAP = 64;     // per-warp queue of probes that passed the filter
 
 struct WinDesc {
     uint32_t nb, nP, nS;             // buckets (0: one oversized bucket), staged slots
@@ -521,6 +519,10 @@ bucket_join_kernel(BucketJoinArgs b)
                 if (lane == 0) s_k[w ^ 1] = kn;
             }
             const WinDesc &d = wd[w];
+            // the other filter buffer was last read by window w-1 and is next written by
+            // window w+1 (both across an end-of-window barrier): clear it now
+            static_assert(BJ_BLOOM == 4 * JOIN_THREADS, "one 16-byte store per thread");
+            reinterpret_cast<uint4 *>(bloom + (w ^ 1) * BJ_BLOOM)[threadIdx.x] = make_uint4(0, 0, 0, 0);
             if (d.nb == 0) {
                 const uint64_t bk = c0 + d.first;
                 const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
@@ -535,68 +537,24 @@ bucket_join_kernel(BucketJoinArgs b)
                     __syncthreads();
                 }
                 const uint64_t *P = pst + w * BJ_HALF, *S = sst + w * BJ_HALF;
-                uint32_t *blB = bloom, *blS = bloom + BJ_BLOOM; // build-key / probe-key filters
+                uint32_t *bl = bloom + w * BJ_BLOOM;
                 const uint32_t tag = epoch << 16;
                 const uint32_t nP = d.nP, nS = d.nS;
-                auto fbit = [&](uint64_t e) { return (uint32_t)(e >> kshift) & 0xFFFFu; };
-                auto test = [&](const uint32_t *bl, uint32_t h) { return ((bl[h >> 5] >> (h & 31u)) & 1u) != 0; };
-                // Four phases, each a flat pass (most entries take the cheap path):
-                //  A  build keys -> filter B
-                //  B  probe keys tested against B (~8 % true matches + ~3 % filter noise pass):
-                //     queued per warp, and their keys -> filter S
-                //  C  build keys tested against S: only those (~9 %) enter the chained hash
-                //  D  queued probes walk the chains (32 at a time, full warps)
-                // ---- A
+                // ---- build: chained hash of the build entries + the 64 Ki-bit filter
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
                     if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
-                    const uint32_t h = fbit(e);
-                    atomicOr(&blB[h >> 5], 1u << (h & 31u));
-                }
-                __syncthreads();
-                if (threadIdx.x == 0) s_has2[w ^ 1] = 0u; // the other window's flag is stale
-                // ---- B
-                uint32_t qn = 0; // warp-uniform queue fill
-                auto push = [&](bool pass, uint32_t qi, uint64_t e) {
-                    const uint32_t m = __ballot_sync(0xffffffffu, pass);
-                    if (pass) {
-                        wq[qn + __popc(m & ((1u << lane) - 1u))] = (unsigned short)qi;
-                        const uint32_t h = fbit(e);
-                        atomicOr(&blS[h >> 5], 1u << (h & 31u));
-                    }
-                    qn += __popc(m);
-                };
-                for (uint32_t t0 = 0; t0 < nS; t0 += JOIN_THREADS) { // block-uniform trip count
-                    const uint32_t t = t0 + threadIdx.x;
-                    uint64_t e = 0;
-                    bool pass = false;
-                    if (t < nS) {
-                        e = S[t];
-                        pass = (e & tagbit) && test(blB, fbit(e)); // !tagbit: sentinel
-                    }
-                    push(pass, t, e);
-                }
-                if (s_has2[w]) { // block-uniform
-                    for (uint32_t t0 = 0; t0 < nP; t0 += JOIN_THREADS) {
-                        const uint32_t k2 = t0 + threadIdx.x;
-                        const uint64_t e = k2 < nP ? P[k2] : 0ull;
-                        push(k2 < nP && (e & (tagbit | flag2bit)) == flag2bit, 0x8000u | k2, e);
-                    }
-                }
-                __syncthreads();
-                // ---- C (filter B is free again: clear it for the next window)
-                reinterpret_cast<uint4 *>(blB)[threadIdx.x] = make_uint4(0, 0, 0, 0);
-                for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
-                    const uint64_t e = P[k2];
-                    if (e & tagbit) continue; // sentinel
-                    if (!test(blS, fbit(e))) continue; // no probe key can match it
-                    const uint32_t old = atomicExch(&slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)], tag | k2);
+                    const uint32_t hk = (uint32_t)(e >> kshift);
+                    atomicOr(&bl[(hk & 0xFFFFu) >> 5], 1u << (hk & 31u));
+                    const uint32_t old = atomicExch(&slot[hk & (BJ_SLOTS - 1)], tag | k2);
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
                 __syncthreads();
-                // ---- D (filter S is free again)
-                reinterpret_cast<uint4 *>(blS)[threadIdx.x] = make_uint4(0, 0, 0, 0);
+                if (threadIdx.x == 0) s_has2[w ^ 1] = 0u; // the other window's flag is stale
+                // ---- probe: ~95 % of the probe keys miss the filter; the rest are queued per
+                // warp and their chains walked 32 at a time (full warps, no per-lane divergence
+                // between a probe that has a chain and one that has none)
                 auto walk = [&](uint64_t e) {
                     const uint32_t hv = slot[(uint32_t)(e >> kshift) & (BJ_SLOTS - 1)];
                     uint32_t sl = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
@@ -613,9 +571,35 @@ bucket_join_kernel(BucketJoinArgs b)
                     __syncwarp();
                     if (act) walk((qi & 0x8000u) ? P[qi & 0x7FFFu] : S[qi]);
                 };
-                while (qn >= 32) {
-                    drain(qn - 32, 32);
-                    qn -= 32;
+                uint32_t qn = 0; // warp-uniform
+                auto push = [&](bool pass, uint32_t qi) {
+                    const uint32_t m = __ballot_sync(0xffffffffu, pass);
+                    if (pass) wq[qn + __popc(m & ((1u << lane) - 1u))] = (unsigned short)qi;
+                    qn += __popc(m);
+                    if (qn >= 32) {
+                        drain(qn - 32, 32);
+                        qn -= 32;
+                    }
+                };
+                auto passes = [&](uint64_t e) {
+                    const uint32_t hk = (uint32_t)(e >> kshift) & 0xFFFFu;
+                    return ((bl[hk >> 5] >> (hk & 31u)) & 1u) != 0;
+                };
+                for (uint32_t t0 = 0; t0 < nS; t0 += JOIN_THREADS) { // block-uniform trip count
+                    const uint32_t t = t0 + threadIdx.x;
+                    bool pass = false;
+                    if (t < nS) {
+                        const uint64_t e = S[t];
+                        pass = (e & tagbit) && passes(e); // !tagbit: sentinel
+                    }
+                    push(pass, t);
+                }
+                if (s_has2[w]) { // block-uniform
+                    for (uint32_t t0 = 0; t0 < nP; t0 += JOIN_THREADS) {
+                        const uint32_t k2 = t0 + threadIdx.x;
+                        const bool pass = k2 < nP && (P[k2] & (tagbit | flag2bit)) == flag2bit;
+                        push(pass, 0x8000u | k2);
+                    }
                 }
                 if (qn) drain(0, qn);
             }
