@@ -316,6 +316,7 @@ refine_kernel(RefineArgs a)
             }
         }
         __syncthreads();
+#pragma unroll 4
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
             const long long go = gofs[bin_of<SPLIT>(k, a.dshift, a.vbits)];
