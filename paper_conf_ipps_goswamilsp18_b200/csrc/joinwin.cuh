@@ -20,7 +20,7 @@ constexpr int JOIN_THREADS = 512;
 constexpr int JOIN_CHUNK = 2048;   // nominal entries per CTA
 constexpr int JOIN_CAP = 6144;     // staged entries per CTA (chunk + the bucket straddling its end)
 constexpr int JOIN_SLOTS = 8192;   // hash chain heads (u32); chains through next[] (u16)
-constexpr int JOIN_BUF = 1024;     // staged output pairs
+constexpr int JOIN_BUF = 1024;     // staged output pairs (2 per thread of a JOIN_THREADS block)
 
 // Candidates are staged in shared memory and verified in a separate, fully parallel pass
 // (a fingerprint match is rare: verifying it inline would run the long verify path with one
@@ -29,6 +29,7 @@ struct Stager {
     unsigned long long *buf; // shared: staged (u << 32 | b) records, ~0 = rejected
     uint32_t *bcount;        // shared
     unsigned long long *pairs, cap, *count;
+    uint32_t bufcap = JOIN_BUF; // records `buf` holds (2 per thread of the block)
 };
 
 // Fingerprint match of probe entry e (vertex w, flag 1 or 2) and build entry p (vertex v,
@@ -47,7 +48,7 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
     const uint32_t lo = min(x, y), hi = max(x, y);
     const unsigned long long rec = ((unsigned long long)lo << 32) | hi;
     const uint32_t slot = atomicAdd(sg.bcount, 1u);
-    if (slot < JOIN_BUF) {
+    if (slot < sg.bufcap) {
         sg.buf[slot] = rec;
         return;
     }
@@ -65,12 +66,12 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
 
 // verify staged records [from, to) in parallel; rejected ones become ~0.  In greedy mode a
 // verified pair with a claimed read end becomes ~1 (counted as found, not stored).
-template <int W>
+template <int W, int NT = JOIN_THREADS>
 __device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long long *buf,
                                               uint32_t from, uint32_t to, unsigned long long &nfalse)
 {
     uint32_t nfound = 0;
-    for (uint32_t t = from + threadIdx.x; t < to; t += JOIN_THREADS) {
+    for (uint32_t t = from + threadIdx.x; t < to; t += NT) {
         const unsigned long long rec = buf[t];
         const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
         if (!verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
@@ -91,15 +92,16 @@ __device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long l
 // write the accepted staged records [0, m) to the global pool: one global atomic per block
 // reserves the block's range (a per-record or per-warp atomic on the single pool counter
 // serialises at L2 — ~86 K warp atomics per length at cfg3).  Called by all threads.
+template <int NT = JOIN_THREADS>
 __device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint32_t m,
                                              unsigned long long *pairs, unsigned long long cap,
                                              unsigned long long *count)
 {
-    __shared__ uint32_t fw[JOIN_THREADS / 32];
+    __shared__ uint32_t fw[NT / 32];
     __shared__ unsigned long long fbase;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     uint32_t c = 0;
-    for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS) c += buf[t] < ~1ull;
+    for (uint32_t t = threadIdx.x; t < m; t += NT) c += buf[t] < ~1ull;
     uint32_t x = c;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -110,7 +112,7 @@ __device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint
     __syncthreads();
     if (threadIdx.x == 0) {
         uint32_t tot = 0;
-        for (int w = 0; w < JOIN_THREADS / 32; ++w) {
+        for (int w = 0; w < NT / 32; ++w) {
             const uint32_t v = fw[w];
             fw[w] = tot;
             tot += v;
@@ -119,7 +121,7 @@ __device__ __forceinline__ void flush_staged(const unsigned long long *buf, uint
     }
     __syncthreads();
     unsigned long long pos = fbase + fw[wid] + x - c;
-    for (uint32_t t = threadIdx.x; t < m; t += JOIN_THREADS) {
+    for (uint32_t t = threadIdx.x; t < m; t += NT) {
         const unsigned long long rec = buf[t];
         if (rec >= ~1ull) continue; // rejected (~0) or dead (~1)
         if (pos < cap) pairs[pos] = rec;
@@ -181,16 +183,16 @@ __device__ __forceinline__ void oversized_join(const JoinArgs &a, const uint64_t
 // after a window (called by all threads after a __syncthreads()): once at least one candidate
 // per thread is staged, verify them all in parallel (the long verify path runs with full
 // warps) and flush the accepted ones.  Cheaper windows just leave the buffer as it is.
-template <int W>
+template <int W, int NT = JOIN_THREADS>
 __device__ __forceinline__ void window_epilogue(const JoinArgs &a, unsigned long long *buf,
                                                 uint32_t *bcount, uint32_t *vdone,
                                                 unsigned long long &nfalse)
 {
-    const uint32_t to = min(*bcount, (uint32_t)JOIN_BUF);
-    if (to >= (uint32_t)JOIN_THREADS) {
-        verify_staged<W>(a, buf, 0, to, nfalse);
+    const uint32_t to = min(*bcount, 2u * NT);
+    if (to >= (uint32_t)NT) {
+        verify_staged<W, NT>(a, buf, 0, to, nfalse);
         __syncthreads();
-        flush_staged(buf, to, a.pairs, a.cap, a.count);
+        flush_staged<NT>(buf, to, a.pairs, a.cap, a.count);
         __syncthreads();
         if (threadIdx.x == 0) *bcount = 0;
         __syncthreads();
@@ -199,15 +201,15 @@ __device__ __forceinline__ void window_epilogue(const JoinArgs &a, unsigned long
 }
 
 // end of a join kernel: verify and flush whatever is still staged
-template <int W>
+template <int W, int NT = JOIN_THREADS>
 __device__ __forceinline__ void final_flush(const JoinArgs &a, unsigned long long *buf,
                                             uint32_t *bcount, unsigned long long &nfalse)
 {
     __syncthreads();
-    const uint32_t to = min(*bcount, (uint32_t)JOIN_BUF);
-    verify_staged<W>(a, buf, 0, to, nfalse);
+    const uint32_t to = min(*bcount, 2u * NT);
+    verify_staged<W, NT>(a, buf, 0, to, nfalse);
     __syncthreads();
-    flush_staged(buf, to, a.pairs, a.cap, a.count);
+    flush_staged<NT>(buf, to, a.pairs, a.cap, a.count);
 }
 
 } // namespace lsg

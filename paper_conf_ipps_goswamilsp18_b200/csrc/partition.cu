@@ -361,7 +361,9 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 // CTA overwrote beforehand (in global memory) with a sentinel of the wrong tag — ~0 (tag 1)
 // in a prefix half, ~0 ^ (1 << vbits) (tag 0) in a suffix half — so the insert and probe
 // loops skip it by its tag bit alone.  Two barriers per window.
-constexpr int BJ_HALF = 2048;   // staged entries per half per window
+constexpr int BJ_THREADS = 1024; // threads per CTA (one CTA per SM)
+constexpr int BJ_HALF = 4096;   // staged entries per half per window
+constexpr int BJ_BUF = 2 * BJ_THREADS; // staged candidate pairs
 constexpr int BJ_MAXB = 64;     // buckets per window
 constexpr int BJ_FILLS = 256;   // buckets whose fills are staged at once
 constexpr int BJ_SLOTS = 4096;  // chain heads (u32 epoch-tagged)
@@ -383,7 +385,7 @@ __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const ui
 {
     const uint32_t kshift = a.vbits + FLAG_BITS;
     const uint64_t vmask = (1ull << a.vbits) - 1;
-    for (uint32_t i = threadIdx.x; i < nS + nP; i += JOIN_THREADS) {
+    for (uint32_t i = threadIdx.x; i < nS + nP; i += BJ_THREADS) {
         const uint64_t e = i < nS ? S[i] : P[i - nS];
         if (i >= nS && key_flag(e, a.vbits) != 2) continue;
         for (uint32_t j = 0; j < nP; ++j) {
@@ -394,17 +396,17 @@ __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const ui
 }
 
 template <int W>
-__global__ void __launch_bounds__(JOIN_THREADS, 2)
+__global__ void __launch_bounds__(BJ_THREADS, BJ_THREADS >= 1024 ? 1 : 2)
 bucket_join_kernel(BucketJoinArgs b)
 {
     extern __shared__ __align__(128) unsigned char jsm[];
     uint64_t *pst = reinterpret_cast<uint64_t *>(jsm);                    // [2][BJ_HALF]
     uint64_t *sst = pst + 2 * BJ_HALF;                                    // [2][BJ_HALF]
     unsigned long long *buf = reinterpret_cast<unsigned long long *>(sst + 2 * BJ_HALF); // [BUF]
-    uint32_t *slot = reinterpret_cast<uint32_t *>(buf + JOIN_BUF);       // [BJ_SLOTS]
+    uint32_t *slot = reinterpret_cast<uint32_t *>(buf + BJ_BUF);       // [BJ_SLOTS]
     uint32_t *bloom = slot + BJ_SLOTS;                                    // [2][BJ_BLOOM]
     unsigned short *queue = reinterpret_cast<unsigned short *>(bloom + 2 * BJ_BLOOM); // [16][QCAP]
-    unsigned short *next = queue + (JOIN_THREADS / 32) * BJ_QCAP;         // [BJ_HALF]
+    unsigned short *next = queue + (BJ_THREADS / 32) * BJ_QCAP;         // [BJ_HALF]
     uint32_t *sfill = reinterpret_cast<uint32_t *>(next + BJ_HALF);       // [2 * BJ_FILLS]
     __shared__ WinDesc wd[2];
     __shared__ __align__(8) unsigned long long mbar[2];
@@ -422,9 +424,9 @@ bucket_join_kernel(BucketJoinArgs b)
         mbar_init(&mbar[1], 1);
         fence_mbar_init();
     }
-    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
-    for (uint32_t t = threadIdx.x; t < 2 * BJ_BLOOM; t += JOIN_THREADS) bloom[t] = 0;
-    Stager em{buf, &bcount, a.pairs, a.cap, a.count};
+    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += BJ_THREADS) slot[t] = 0;
+    for (uint32_t t = threadIdx.x; t < 2 * BJ_BLOOM; t += BJ_THREADS) bloom[t] = 0;
+    Stager em{buf, &bcount, a.pairs, a.cap, a.count, BJ_BUF};
     unsigned long long nfalse = 0;
     uint32_t epoch = 0, phases = 0; // bit w: parity of the next phase of mbar[w]
     const int lane = threadIdx.x & 31;
@@ -433,7 +435,7 @@ bucket_join_kernel(BucketJoinArgs b)
     for (uint64_t c0 = b0; c0 < b1; c0 += BJ_FILLS) {
         const uint32_t nc = (uint32_t)min64(BJ_FILLS, b1 - c0);
         __syncthreads();
-        for (uint32_t t = threadIdx.x; t < 2 * nc; t += JOIN_THREADS) {
+        for (uint32_t t = threadIdx.x; t < 2 * nc; t += BJ_THREADS) {
             const uint32_t f = b.fills[2 * c0 + t];
             if (f > b.half_cap) *b.overflow = 1u;
             const uint32_t fc = (uint32_t)min64(f, b.half_cap);
@@ -502,7 +504,7 @@ bucket_join_kernel(BucketJoinArgs b)
             }
             return k + nb;
         };
-        constexpr int PLAN_WARP = JOIN_THREADS / 32 - 1;
+        constexpr int PLAN_WARP = BJ_THREADS / 32 - 1;
         const bool planner = (threadIdx.x >> 5) == PLAN_WARP;
         if (planner) {
             fence_proxy_async();
@@ -522,8 +524,8 @@ bucket_join_kernel(BucketJoinArgs b)
             const WinDesc &d = wd[w];
             // the other filter buffer was last read by window w-1 and is next written by
             // window w+1 (both across an end-of-window barrier): clear it now
-            static_assert(BJ_BLOOM == 4 * JOIN_THREADS, "one 16-byte store per thread");
-            reinterpret_cast<uint4 *>(bloom + (w ^ 1) * BJ_BLOOM)[threadIdx.x] = make_uint4(0, 0, 0, 0);
+            for (uint32_t t = threadIdx.x; t < BJ_BLOOM / 4; t += BJ_THREADS)
+                reinterpret_cast<uint4 *>(bloom + (w ^ 1) * BJ_BLOOM)[t] = make_uint4(0, 0, 0, 0);
             if (d.nb == 0) {
                 const uint64_t bk = c0 + d.first;
                 const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
@@ -533,7 +535,7 @@ bucket_join_kernel(BucketJoinArgs b)
                 mbar_wait(&mbar[w], (phases >> w) & 1u);
                 phases ^= 1u << w;
                 if (++epoch == 0x10000u) { // block-uniform
-                    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += JOIN_THREADS) slot[t] = 0;
+                    for (uint32_t t = threadIdx.x; t < BJ_SLOTS; t += BJ_THREADS) slot[t] = 0;
                     epoch = 1;
                     __syncthreads();
                 }
@@ -542,7 +544,7 @@ bucket_join_kernel(BucketJoinArgs b)
                 const uint32_t tag = epoch << 16;
                 const uint32_t nP = d.nP, nS = d.nS;
                 // ---- build: chained hash of the build entries + the 64 Ki-bit filter
-                for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += JOIN_THREADS) {
+                for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += BJ_THREADS) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
                     if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
@@ -586,7 +588,7 @@ bucket_join_kernel(BucketJoinArgs b)
                     const uint32_t hk = (uint32_t)(e >> kshift) & 0xFFFFu;
                     return ((bl[hk >> 5] >> (hk & 31u)) & 1u) != 0;
                 };
-                for (uint32_t t0 = 0; t0 < nS; t0 += JOIN_THREADS) { // block-uniform trip count
+                for (uint32_t t0 = 0; t0 < nS; t0 += BJ_THREADS) { // block-uniform trip count
                     const uint32_t t = t0 + threadIdx.x;
                     bool pass = false;
                     if (t < nS) {
@@ -596,7 +598,7 @@ bucket_join_kernel(BucketJoinArgs b)
                     push(pass, t);
                 }
                 if (s_has2[w]) { // block-uniform
-                    for (uint32_t t0 = 0; t0 < nP; t0 += JOIN_THREADS) {
+                    for (uint32_t t0 = 0; t0 < nP; t0 += BJ_THREADS) {
                         const uint32_t k2 = t0 + threadIdx.x;
                         const bool pass = k2 < nP && (P[k2] & (tagbit | flag2bit)) == flag2bit;
                         push(pass, 0x8000u | k2);
@@ -605,12 +607,12 @@ bucket_join_kernel(BucketJoinArgs b)
                 if (qn) drain(0, qn);
             }
             __syncthreads(); // window w done: its buffers may be refilled
-            window_epilogue<W>(a, buf, &bcount, &vdone, nfalse);
+            window_epilogue<W, BJ_THREADS>(a, buf, &bcount, &vdone, nfalse);
             kcur = knext;
             w ^= 1;
         }
     }
-    final_flush<W>(a, buf, &bcount, nfalse);
+    final_flush<W, BJ_THREADS>(a, buf, &bcount, nfalse);
     for (int o = 16; o; o >>= 1) nfalse += __shfl_xor_sync(0xffffffffu, nfalse, o);
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
@@ -621,18 +623,18 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (args.half_cap & 1) return LASAGNA_EINVAL; // sentinels need an even half capacity
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)JOIN_BUF * 8 + (size_t)BJ_SLOTS * 4 +
-                            (size_t)2 * BJ_BLOOM * 4 + (size_t)(JOIN_THREADS / 32) * BJ_QCAP * 2 +
+        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)BJ_BUF * 8 + (size_t)BJ_SLOTS * 4 +
+                            (size_t)2 * BJ_BLOOM * 4 + (size_t)(BJ_THREADS / 32) * BJ_QCAP * 2 +
                             (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
         LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0;
         LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bucket_join_kernel<W>,
-                                                               JOIN_THREADS, smem));
+                                                               BJ_THREADS, smem));
         per_sm = std::max(per_sm, 1);
         const uint64_t blocks =
             std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)num_sms() * per_sm, args.n_buckets));
-        bucket_join_kernel<W><<<(unsigned)blocks, JOIN_THREADS, smem, s>>>(args);
+        bucket_join_kernel<W><<<(unsigned)blocks, BJ_THREADS, smem, s>>>(args);
         LSG_LAUNCHED("bucket_join_kernel");
         return LASAGNA_OK;
     });
