@@ -40,22 +40,62 @@ __device__ __forceinline__ void set_claimed(uint32_t *cl, uint32_t x)
     atomicOr(&cl[x >> 5], 1u << (x & 31u));
 }
 
+// Append the pairs r[k] with bit k of keepm set to out[]: one global atomic per block and
+// loop trip (a per-thread or per-warp atomic on the single counter serialises at L2).  Called
+// by every thread of the block (block-uniform trip counts).
+__device__ __forceinline__ void block_append(const unsigned long long (&r)[GK], uint32_t keepm,
+                                             unsigned long long *out, unsigned long long *out_count)
+{
+    __shared__ uint32_t wsum[GREEDY_THREADS / 32];
+    __shared__ unsigned long long sbase;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const uint32_t nk = __popc(keepm);
+    uint32_t x = nk; // warp inclusive scan of the counts
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t tot = 0;
+        for (int w = 0; w < GREEDY_THREADS / 32; ++w) {
+            const uint32_t v = wsum[w];
+            wsum[w] = tot;
+            tot += v;
+        }
+        sbase = tot ? atomicAdd(out_count, (unsigned long long)tot) : 0ull;
+    }
+    __syncthreads();
+    unsigned long long pos = sbase + wsum[wid] + x - nk;
+#pragma unroll
+    for (int k = 0; k < GK; ++k)
+        if (keepm & (1u << k)) out[pos++] = r[k];
+    __syncthreads(); // wsum / sbase reuse
+}
+
+// Round part 1: every pair with both ends free proposes its partner to both ends and is
+// appended to the round's live list (dead pairs — an end claimed by a longer length or an
+// earlier round — are dropped here, once).  *reset is the counter two kernels ahead.
 __global__ void __launch_bounds__(GREEDY_THREADS)
 greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
                unsigned long long cap, const uint32_t *claimed, unsigned long long *best,
-               uint32_t epoch, unsigned long long *out_count, unsigned long long *book)
+               uint32_t epoch, unsigned long long *live, unsigned long long *live_count,
+               unsigned long long *reset, unsigned long long *book)
 {
     const unsigned long long c = *count;
     const unsigned long long m = c < cap ? c : cap;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-        *out_count = 0;
+        *reset = 0;
         if (book) { // first round of a length: |P_l| bookkeeping
             atomicAdd(&book[1], c);
             atomicMax(&book[2], c);
         }
     }
     const uint64_t stride = (uint64_t)gridDim.x * GREEDY_THREADS * GK;
-    for (uint64_t i0 = (uint64_t)blockIdx.x * GREEDY_THREADS * GK + threadIdx.x; i0 < m; i0 += stride) {
+    for (uint64_t i0 = (uint64_t)blockIdx.x * GREEDY_THREADS * GK + threadIdx.x;
+         i0 - threadIdx.x < m; i0 += stride) { // block-uniform trip count
         unsigned long long r[GK];
         bool ca[GK], cb[GK];
 #pragma unroll
@@ -67,13 +107,16 @@ greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
         for (int k = 0; k < GK; ++k)
             if (r[k] != ~0ull)
                 ca[k] = is_claimed(claimed, (uint32_t)(r[k] >> 32)), cb[k] = is_claimed(claimed, (uint32_t)r[k]);
+        uint32_t keepm = 0;
 #pragma unroll
         for (int k = 0; k < GK; ++k) {
             if (r[k] == ~0ull || (ca[k] | cb[k])) continue;
             const uint32_t a = (uint32_t)(r[k] >> 32), b = (uint32_t)r[k];
             atomicMax(&best[a], proposal(epoch, b));
             atomicMax(&best[b], proposal(epoch, a));
+            keepm |= 1u << k;
         }
+        block_append(r, keepm, live, live_count);
     }
 }
 
@@ -85,43 +128,39 @@ __device__ __forceinline__ void accept_pair(uint32_t a, uint32_t b, uint32_t *cl
     olen[a] = l, olen[b] = l;
 }
 
-// Survivors are appended to `out` with one global atomic per block and loop trip (a
-// per-thread or per-warp atomic on the single counter serialises at L2).
+// Round part 2 over the live list: a pair whose two ends both chose each other is accepted;
+// the others survive to the next round (some of them now have an end claimed by a pair
+// accepted in this round: the next propose drops them).  No claimed-bit reads: every listed
+// pair was live when the proposals were made, and acceptance is decided by best[] alone.
 __global__ void __launch_bounds__(GREEDY_THREADS)
 greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
               unsigned long long cap, uint32_t *claimed, const unsigned long long *best,
               uint32_t epoch, uint32_t *succ, uint8_t *olen, uint8_t l, unsigned long long *out,
-              unsigned long long *out_count, unsigned long long *book)
+              unsigned long long *out_count, unsigned long long *reset, unsigned long long *book)
 {
-    __shared__ uint32_t wsum[GREEDY_THREADS / 32];
-    __shared__ unsigned long long sbase;
     const unsigned long long c = *count;
     const unsigned long long m = c < cap ? c : cap;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *reset = 0;
+    const int lane = threadIdx.x & 31;
     uint32_t acc = 0;
     const uint64_t stride = (uint64_t)gridDim.x * GREEDY_THREADS * GK;
     for (uint64_t i0 = (uint64_t)blockIdx.x * GREEDY_THREADS * GK + threadIdx.x;
          i0 - threadIdx.x < m; i0 += stride) { // block-uniform trip count
         unsigned long long r[GK], ba[GK], bb[GK];
-        bool ca[GK], cb[GK];
 #pragma unroll
         for (int k = 0; k < GK; ++k) {
             const uint64_t i = i0 + (uint64_t)k * GREEDY_THREADS;
             r[k] = i < m ? pairs[i] : ~0ull;
         }
+        // best[] of both ends (random 32 B sectors in an 8 B/end array: the traffic that bounds
+        // the round)
 #pragma unroll
         for (int k = 0; k < GK; ++k)
-            if (r[k] != ~0ull)
-                ca[k] = is_claimed(claimed, (uint32_t)(r[k] >> 32)), cb[k] = is_claimed(claimed, (uint32_t)r[k]);
-        // best[] only for live pairs (random 32 B sectors in a 16 B/end array: the traffic that
-        // bounds the round)
-#pragma unroll
-        for (int k = 0; k < GK; ++k)
-            if (r[k] != ~0ull && !(ca[k] | cb[k])) ba[k] = best[(uint32_t)(r[k] >> 32)], bb[k] = best[(uint32_t)r[k]];
+            if (r[k] != ~0ull) ba[k] = best[(uint32_t)(r[k] >> 32)], bb[k] = best[(uint32_t)r[k]];
         uint32_t keepm = 0;
 #pragma unroll
         for (int k = 0; k < GK; ++k) {
-            if (r[k] == ~0ull || (ca[k] | cb[k])) continue; // dead: an end was taken earlier
+            if (r[k] == ~0ull) continue;
             const uint32_t a = (uint32_t)(r[k] >> 32), b = (uint32_t)r[k];
             if (ba[k] == proposal(epoch, b) && bb[k] == proposal(epoch, a)) {
                 accept_pair(a, b, claimed, succ, olen, l);
@@ -130,30 +169,7 @@ greedy_accept(const unsigned long long *pairs, const unsigned long long *count,
                 keepm |= 1u << k;
             }
         }
-        const uint32_t nk = __popc(keepm);
-        uint32_t x = nk; // warp inclusive scan of the survivor counts
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        if (lane == 31) wsum[wid] = x;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            uint32_t tot = 0;
-            for (int w = 0; w < GREEDY_THREADS / 32; ++w) {
-                const uint32_t v = wsum[w];
-                wsum[w] = tot;
-                tot += v;
-            }
-            sbase = tot ? atomicAdd(out_count, (unsigned long long)tot) : 0ull;
-        }
-        __syncthreads();
-        unsigned long long pos = sbase + wsum[wid] + x - nk;
-#pragma unroll
-        for (int k = 0; k < GK; ++k)
-            if (keepm & (1u << k)) out[pos++] = r[k];
-        __syncthreads(); // wsum / sbase reuse
+        block_append(r, keepm, out, out_count);
     }
     for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
     if (lane == 0 && acc) atomicAdd(&book[0], (unsigned long long)acc);
@@ -254,20 +270,27 @@ lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *
     const int sms = num_sms();
     const unsigned blocks = (unsigned)std::max<uint64_t>(
         1, std::min<uint64_t>(ceil_div(g.cap, GREEDY_THREADS * GK), (uint64_t)sms * 8));
-    unsigned long long *in = g.pool, *out = g.pool2, *cin = g.cnt, *cout = g.cnt2;
+    // Round r: propose reads X (count ctr[2r % 3]) and lists the live pairs in Y
+    // (ctr[(2r+1) % 3]); accept reads Y and writes the survivors back to X (ctr[(2r+2) % 3]).
+    // A kernel never resets a counter another block of the same launch may still read: each
+    // one zeroes the counter two launches ahead.  With three rounds the survivors end in
+    // ctr[0], and the last reset (ctr[1]) is the first append target of the next length.
+    static_assert(FAST_ROUNDS == 3, "counter rotation");
+    unsigned long long *X = g.pool, *Y = g.pool2;
+    unsigned long long *ctr[3] = {g.cnt, g.cnt2, g.cnt3};
     const uint32_t e0 = g.epoch;
     g.epoch += EPOCHS_PER_LENGTH;
     for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
-        greedy_propose<<<blocks, GREEDY_THREADS, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, cout,
-                                              r == 0 ? g.book : nullptr);
+        greedy_propose<<<blocks, GREEDY_THREADS, 0, s>>>(X, ctr[(2 * r) % 3], g.cap, g.claimed, g.best,
+                                                         e0 + r, Y, ctr[(2 * r + 1) % 3],
+                                                         ctr[(2 * r + 2) % 3], r == 0 ? g.book : nullptr);
         LSG_LAUNCHED("greedy_propose");
-        greedy_accept<<<blocks, GREEDY_THREADS, 0, s>>>(in, cin, g.cap, g.claimed, g.best, e0 + r, succ, olen,
-                                             l, out, cout, g.book);
+        greedy_accept<<<blocks, GREEDY_THREADS, 0, s>>>(Y, ctr[(2 * r + 1) % 3], g.cap, g.claimed, g.best,
+                                                        e0 + r, succ, olen, l, X, ctr[(2 * r + 2) % 3],
+                                                        ctr[(2 * r) % 3], g.book);
         LSG_LAUNCHED("greedy_accept");
-        std::swap(in, out);
-        std::swap(cin, cout);
     }
-    greedy_finish<<<1, FINISH_THREADS, 0, s>>>(in, cin, out, cout, g.claimed, g.best,
+    greedy_finish<<<1, FINISH_THREADS, 0, s>>>(X, ctr[0], Y, ctr[1], g.claimed, g.best,
                                                e0 + FAST_ROUNDS, FAST_ROUNDS, succ, olen, l, g.book);
     LSG_LAUNCHED("greedy_finish");
     return LASAGNA_OK;

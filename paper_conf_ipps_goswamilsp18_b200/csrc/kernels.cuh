@@ -110,7 +110,8 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s);
 // ---- a6/a7 (greedy.cu)
 struct GreedyBufs {
     unsigned long long *pool, *pool2; // pair lists (ping-pong)
-    unsigned long long *cnt, *cnt2;   // their fills (device)
+    unsigned long long *cnt, *cnt2;   // their fills (device); cnt: the input count
+    unsigned long long *cnt3;         // third round counter (zero, like cnt2, on the first call)
     unsigned long long *book;         // device: [0] accepted, [1] sum |P_l|, [2] max |P_l|, [3] max rounds
     unsigned long long *best;         // u64 [V]: epoch-tagged proposals, zeroed once per call
     uint32_t *claimed;                // bitmap of claimed read ends (2n bits)

@@ -101,7 +101,7 @@ struct Layout {
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
 enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR_FOUND = 8,
-       CTR64_N = 9 };
+       CTR_POOL3 = 9, CTR64_N = 10 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -612,6 +612,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     gb.pool2 = r.pool2;
     gb.cnt = r.ctr64 + CTR_POOL;
     gb.cnt2 = r.ctr64 + CTR_POOL2;
+    gb.cnt3 = r.ctr64 + CTR_POOL3;
     gb.book = r.ctr64 + CTR_BOOK;
     gb.best = r.at<unsigned long long>(r.lay.best);
     gb.claimed = claimed;
@@ -901,7 +902,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     lasagna_status rc = sort_ctx_reset(c, s);
     if (rc != LASAGNA_OK) return rc;
     unsigned long long *ctr64 = reinterpret_cast<unsigned long long *>(ws + o_ctrs + 4096 * 4);
-    LSG_CUDA(cudaMemsetAsync(ctr64, 0, 8 * 8, s));
+    LSG_CUDA(cudaMemsetAsync(ctr64, 0, CTR64_N * 8, s));
     uint32_t *claimed = reinterpret_cast<uint32_t *>(ws + o_claimed);
     LSG_CUDA(cudaMemsetAsync(claimed, 0, ceil_div(V, 32) * 4, s));
     // group by length, descending: key (255 - l) << 56 | i, one 8-bit LSD pass
@@ -920,6 +921,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     gb.pool2 = reinterpret_cast<unsigned long long *>(ws + o_pool2);
     gb.cnt = ctr64 + CTR_POOL;
     gb.cnt2 = ctr64 + CTR_POOL2;
+    gb.cnt3 = ctr64 + CTR_POOL3;
     gb.book = ctr64 + CTR_BOOK;
     gb.best = reinterpret_cast<unsigned long long *>(ws + o_best);
     gb.claimed = claimed;
