@@ -130,7 +130,8 @@ def cpu_baseline(reads: np.ndarray, l_min: int, target_s: float = 12.0) -> dict:
 
 
 # ------------------------------------------------------------------ algorithmic bytes
-def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict) -> dict:
+def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict,
+             sm_mhz: float | None = None) -> dict:
     """Dominant phase and its achieved ALGORITHMIC GB/s (bytes per unit in DESIGN.md x units
     per launch / CUDA-event time per launch)."""
     V = 2 * n
@@ -172,10 +173,28 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict) ->
                   "gbs": (v[2] / (v[0] / 1e3 / max(1, v[1])) / 1e9) if v[0] > 0 else None}
               for k, v in per.items()}
     phases["greedy"] = {"ms_per_step": stats["ms_greedy"] / steps}
+    # Issue view of the same kernel (integer-ALU-bound kernels): warp instructions per launch
+    # from the committed ncu capture (profiles/ncu_inst.json) over the live launch time, against
+    # the SM issue peak = SMs x 4 schedulers x 1 warp instruction per cycle x the SM clock.
+    issue = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_inst.json")) as f:
+            inst = json.load(f).get(name)
+        if inst and avg_s > 0:
+            import torch
+            sms = torch.cuda.get_device_properties(0).multi_processor_count
+            ghz = (sm_mhz or 1965.0) / 1e3
+            pk = sms * 4 * ghz
+            ach = inst / avg_s / 1e9
+            issue = {"unit": "G warp-inst/s", "achieved": round(ach, 1), "peak": round(pk, 1),
+                     "frac": round(ach / pk, 4), "inst_per_launch": inst,
+                     "peak_basis": f"{sms} SMs x 4 issue/clk x {ghz:.3f} GHz (measured SM clock)"}
+    except Exception:
+        pass
     return {"bound": "hbm", "kernel": name, "achieved": round(achieved, 1),
             "peak": peak["hbm_gbs"], "peak_source": peak["source"], "unit": "GB/s",
             "frac": round(achieved / peak["hbm_gbs"], 4), "traffic": traffic,
-            "bytes_per_launch": bytes_per_launch, "phases": phases}
+            "bytes_per_launch": bytes_per_launch, "issue": issue, "phases": phases}
 
 
 # ------------------------------------------------------------------ reference arm (the oracle)
@@ -318,7 +337,7 @@ def main() -> None:
     e2e_ms = f0.elapsed_time(f1) / args.steps
 
     peak = _peaks()
-    roof = roofline(st, n, L, l_min, args.steps, peak)
+    roof = roofline(st, n, L, l_min, args.steps, peak, clocks.get("sm_mhz"))
     out = {
         "metric": METRIC, "value": value, "unit": "reads/s", "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,

@@ -5,8 +5,9 @@
 Produces profiles/<TAG>_launches.md (per-kernel share of one bench step, from the
 `--metrics gpu__time_duration.sum --clock-control none` launch list — cold-cache and
 serialised: compare shares, not absolutes), profiles/<TAG>_ncu.md (selected raw metrics
-of one `--set full` launch per kernel) and profiles/ncu_traffic.json (DRAM bytes per launch,
-read by bench.py's roofline.traffic).
+of one `--set full` launch per kernel), profiles/ncu_traffic.json (DRAM bytes per launch,
+read by bench.py's roofline.traffic) and profiles/ncu_inst.json (warp instructions per launch,
+read by bench.py's roofline.issue).
 """
 from __future__ import annotations
 
@@ -85,6 +86,8 @@ def main() -> None:
         f.write(launch_table(launches) + "\n")
     traffic_path = os.path.join(prof, "ncu_traffic.json")
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+    inst_path = os.path.join(prof, "ncu_inst.json")
+    inst = json.load(open(inst_path)) if os.path.exists(inst_path) else {}
     lines = [f"# {tag}: one `ncu --set full --clock-control none` launch per kernel (cfg3)\n"]
     for rp in reps:
         d = raw(rp)
@@ -99,10 +102,14 @@ def main() -> None:
         lines.append(f"| DRAM bytes per launch | {rb + wb:.4g} |\n")
         if name in NAMES:
             traffic[NAMES[name]] = rb + wb
+            if "smsp__inst_executed.sum" in d: # warp instructions per launch (issue view)
+                inst[NAMES[name]] = float(d["smsp__inst_executed.sum"][0].replace(",", ""))
     with open(os.path.join(prof, f"{tag}_ncu.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     with open(traffic_path, "w") as f:
         json.dump(traffic, f, indent=1)
+    with open(inst_path, "w") as f:
+        json.dump(inst, f, indent=1)
     print("wrote", tag)
 
 
