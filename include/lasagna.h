@@ -149,7 +149,12 @@ LASAGNA_API lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t
  * the first table pass when the fast path runs (the packed rows are written to packed_out,
  * device u64 [n][lasagna_words_per_read(L)], for the verification step), so the read-in of
  * host reads over PCIe overlaps the fingerprint computation.
- *   ascii      n*L bytes, device memory or PAGE-LOCKED host memory (read in place)
+ *   ascii      n*L bytes, device memory or PAGE-LOCKED host memory.  Host input is streamed in
+ *              by the DMA engine (a8 level 2): chunks of 512 Ki reads on an internal
+ *              copy stream into a three-buffer ring inside the workspace, each chunk's table
+ *              pass launched on `stream` as soon as it lands (event-ordered); off the fast
+ *              path, or when the workspace has no room for the ring, it is read in place
+ *              (zero-copy).  The host buffer must stay valid until the call returns.
  *   first_bad  device u64: UINT64_MAX, or the smallest index of a read holding a byte outside
  *              ACGTacgt -> the call returns LASAGNA_EINVAL (outputs unspecified).
  * Synchronises `stream` once at the end. */

@@ -96,6 +96,7 @@ struct Layout {
     uint64_t pool_cap;   // pair pool capacity (pairs)
     size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, fill1,
         fill2, total;
+    size_t tabB_bytes;   // tabB's size (the level-2 regions; the a1 staging ring before them)
 };
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
@@ -120,7 +121,8 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half1 : 256 * g.cap1) * 8;
     const size_t lvl2_b = g.P >= 2 ? (size_t)G * 131072 * g.half2 * 8 : 0;
     l.tabA = take(std::max(exact_b, lvl1_b));
-    l.tabB = take(std::max(exact_b, lvl2_b));
+    l.tabB_bytes = std::max(exact_b, lvl2_b);
+    l.tabB = take(l.tabB_bytes);
     l.fill1 = take((size_t)G * 512 * 4);
     l.fill2 = take(g.P >= 2 ? (size_t)G * 131072 * 4 : 4);
     l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
@@ -196,6 +198,7 @@ struct Run {
     uint32_t *hist;
     bool bucketed;              // partition.cu path (else exact LSD sort + contiguous join)
     const unsigned char *ascii = nullptr; // a1 still to do: the first group's scatter packs it
+    const char *ascii_host = nullptr;     // ... from this page-locked host copy (chunked DMA)
     uint64_t *packed_out = nullptr;
     unsigned long long *first_bad = nullptr;
     uint32_t *fill1, *fill2;
@@ -268,6 +271,66 @@ struct PhaseTimer {
     }
 };
 
+// a8 level 2: the host -> device leg of the semi-streaming driver.  The ASCII
+// reads (page-locked host memory) are copied by the DMA engine in chunks into a ring of three
+// device buffers on a copy stream, and each chunk's fused a1 + a2 + level-1 partition launch
+// runs on the call's stream as soon as its copy has landed, while the next chunks are in
+// flight (events order copy k before scatter k, and scatter k before the copy that reuses its
+// slot).  The ring lives in the level-2 region buffer, which nothing touches before the refine
+// pass that follows.  Chunks are whole scatter CTAs (multiples of 512 reads); per-(CTA, bin)
+// reservations accumulate across the launches exactly as within one.
+static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const char *host)
+{
+    constexpr int NSLOT = 3;
+    const uint64_t n = base.n, L = base.L;
+    // 512 Ki reads per chunk (~53 MB at L = 101); LASAGNA_TEST_A1_CHUNK (tests only) overrides
+    static const uint64_t want = [] {
+        const char *e = getenv("LASAGNA_TEST_A1_CHUNK");
+        const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
+        return v ? v : (uint64_t)512 * 1024;
+    }();
+    uint64_t chunk = std::max<uint64_t>(512, want / 512 * 512);
+    const uint64_t fit = r.lay.tabB_bytes / (NSLOT * L);
+    chunk = std::min(chunk, fit / 512 * 512);
+    if (chunk == 0) return launch_scatter_table(base, r.s); // no room: zero-copy reads
+    unsigned char *ring = reinterpret_cast<unsigned char *>(r.tab[1]);
+    const size_t slot_bytes = (size_t)chunk * L;
+    struct Res {
+        cudaStream_t cs = nullptr;
+        cudaEvent_t ev[2 * NSLOT + 1] = {};
+        ~Res()
+        {
+            for (auto e : ev)
+                if (e) cudaEventDestroy(e);
+            if (cs) cudaStreamDestroy(cs);
+        }
+    } res;
+    LSG_CUDA(cudaStreamCreateWithFlags(&res.cs, cudaStreamNonBlocking));
+    for (auto &e : res.ev) LSG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    cudaEvent_t *copied = res.ev, *consumed = res.ev + NSLOT, start = res.ev[2 * NSLOT];
+    LSG_CUDA(cudaEventRecord(start, r.s)); // the ring's previous users (an earlier call) are done
+    LSG_CUDA(cudaStreamWaitEvent(res.cs, start, 0));
+    uint32_t k = 0;
+    for (uint64_t r0 = 0; r0 < n; r0 += chunk, ++k) {
+        const int slot = (int)(k % NSLOT);
+        const uint64_t m = std::min(chunk, n - r0);
+        if (k >= (uint32_t)NSLOT) LSG_CUDA(cudaStreamWaitEvent(res.cs, consumed[slot], 0));
+        LSG_CUDA(cudaMemcpyAsync(ring + slot * slot_bytes, host + r0 * L, m * L,
+                                 cudaMemcpyHostToDevice, res.cs));
+        LSG_CUDA(cudaEventRecord(copied[slot], res.cs));
+        LSG_CUDA(cudaStreamWaitEvent(r.s, copied[slot], 0));
+        ScatterArgs sa = base;
+        sa.ascii = ring + slot * slot_bytes;
+        sa.n = m;
+        sa.read_offset = base.read_offset + r0;
+        sa.packed_out = base.packed_out + r0 * base.stride;
+        lasagna_status rc = launch_scatter_table(sa, r.s);
+        if (rc != LASAGNA_OK) return rc;
+        LSG_CUDA(cudaEventRecord(consumed[slot], r.s));
+    }
+    return LASAGNA_OK;
+}
+
 // Build + sort the key tables of lengths [l_lo, l_hi]; returns which tab buffer is sorted.
 static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint32_t l_lo,
                                            uint32_t l_hi, PhaseTimer &tm, lasagna_stats *st)
@@ -293,10 +356,16 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.ascii = r.ascii; // fused a1 (first group only)
     sa.packed_out = r.packed_out;
     sa.first_bad = r.first_bad;
+    const char *host = r.ascii_host;
     r.ascii = nullptr;
+    r.ascii_host = nullptr;
     lasagna_status rc;
     if ((rc = tm.start(PH_TABLE)) != LASAGNA_OK) return rc;
-    if ((rc = launch_scatter_table(sa, r.s)) != LASAGNA_OK) return rc;
+    if (sa.ascii && host && g.P >= 2) {
+        if ((rc = scatter_from_host(r, sa, host)) != LASAGNA_OK) return rc;
+    } else if ((rc = launch_scatter_table(sa, r.s)) != LASAGNA_OK) {
+        return rc;
+    }
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     if (g.P >= 2) {
         RefineArgs ra;
@@ -445,7 +514,7 @@ uint32_t lasagna_words_per_read(uint32_t L) { return stride_for(L); }
 
 // Device address of an ASCII read buffer: device memory, or page-locked host memory mapped
 // into the device address space (read in place over PCIe).  Pageable memory is rejected.
-static lasagna_status resolve_ascii(const char *ascii, const char **dev)
+static lasagna_status resolve_ascii(const char *ascii, const char **dev, bool *is_host = nullptr)
 {
     cudaPointerAttributes at;
     if (cudaPointerGetAttributes(&at, ascii) != cudaSuccess) {
@@ -454,6 +523,7 @@ static lasagna_status resolve_ascii(const char *ascii, const char **dev)
         return LASAGNA_EINVAL;
     }
     *dev = ascii;
+    if (is_host) *is_host = at.type == cudaMemoryTypeHost;
     if (at.type == cudaMemoryTypeHost) {
         if (!at.devicePointer) {
             set_error("ascii: page-locked host memory is not mapped into the device");
@@ -544,6 +614,7 @@ lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budge
 // a1 is fused into the first group's table build, the packed rows land in packed_out, bad
 // reads in *first_bad).
 static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *ascii_dev,
+                                        const char *ascii_host,
                                         uint64_t *packed_out, uint64_t *first_bad, uint64_t n,
                                         uint32_t L, uint32_t l_min, uint32_t lengths_per_pass,
                                         void *workspace, size_t *workspace_bytes, uint32_t *succ,
@@ -600,6 +671,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         LSG_CUDA(cudaMemsetAsync(first_bad, 0xFF, 8, s));
         if (use_bucketed(g) && g.P == 2 && L <= 160) {
             r.ascii = reinterpret_cast<const unsigned char *>(ascii_dev);
+            r.ascii_host = ascii_host;
             r.packed_out = packed_out;
             r.first_bad = reinterpret_cast<unsigned long long *>(first_bad);
         } else {
@@ -701,7 +773,7 @@ lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t n, uint32_t
                                     lasagna_stats *stats, void *stream)
 {
     g_err[0] = 0;
-    return greedy_graph_impl(packed, nullptr, nullptr, nullptr, n, L, l_min, lengths_per_pass,
+    return greedy_graph_impl(packed, nullptr, nullptr, nullptr, nullptr, n, L, l_min, lengths_per_pass,
                              workspace, workspace_bytes, succ, olen, stats, stream);
 }
 
@@ -714,15 +786,18 @@ lasagna_status lasagna_greedy_graph_ascii(const char *ascii, uint64_t n, uint32_
 {
     g_err[0] = 0;
     const char *dev = nullptr;
+    bool is_host = false;
     if (workspace && n) {
         if (!ascii) {
             set_error("ascii is NULL");
             return LASAGNA_EINVAL;
         }
-        lasagna_status rc = resolve_ascii(ascii, &dev);
+        lasagna_status rc = resolve_ascii(ascii, &dev, &is_host);
         if (rc != LASAGNA_OK) return rc;
     }
-    return greedy_graph_impl(nullptr, dev ? dev : ascii, packed_out, first_bad, n, L, l_min,
+    // page-locked host input: the fast path streams it in by DMA (scatter_from_host)
+    const char *host = is_host ? ascii : nullptr;
+    return greedy_graph_impl(nullptr, dev ? dev : ascii, host, packed_out, first_bad, n, L, l_min,
                              lengths_per_pass, workspace, workspace_bytes, succ, olen, stats,
                              stream);
 }

@@ -101,7 +101,7 @@ scatter_table_kernel(ScatterArgs a)
 #pragma unroll
             for (int j = 0; j < W; ++j) po[j] = x[j];
             for (uint32_t j = W; j < a.stride; ++j) po[j] = 0;
-            if (!ok) atomicMin(a.first_bad, (unsigned long long)i);
+            if (!ok) atomicMin(a.first_bad, (unsigned long long)(a.read_offset + i));
             rc_words<W>(x, a.L, y);
         } else {
 #pragma unroll

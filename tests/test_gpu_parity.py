@@ -309,6 +309,37 @@ def test_palindrome_rich_parity_two_level(lz):
     assert np.array_equal(_np(r.olen, np.uint8), eolen)
 
 
+@gpu
+def test_oversized_fingerprint_class(lz):
+    """A fingerprint class far larger than a bucket's slack: 4200 copies of one read X plus a
+    read Y whose 80-base prefix is X's 80-base suffix, among 400 K genome reads (T = 16).  X's
+    entries of every length overflow their level-2 bucket (capacity ~750), the overflow is
+    detected and the call is redone on the exact LSD path (stats.bucketed = 0); the 4200
+    (X, Y) pairs at l = 80 and the greedy result match the oracle bit for bit."""
+    import torch
+    L, l_min = 101, 63
+    reads = readgen.reads(11, 4_000_000, 400_000, L, 0.01)
+    rng = np.random.default_rng(5)
+    acgt = np.frombuffer(b"ACGT", dtype=np.uint8)
+    x = acgt[rng.integers(0, 4, L)]
+    y = np.concatenate([x[L - 80:], acgt[rng.integers(0, 4, L - 80)]])
+    reads[1000:5200] = x
+    reads[7] = y
+    n = reads.shape[0]
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, n, L, l_min)
+    assert r.stats["key_sort_bits"] == 16 and r.stats["bucketed"] == 0
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc
+    assert np.array_equal(_np(r.succ, np.uint32), esucc)
+    assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    pl, pa, pb = lz.overlaps(packed, n, L, l_min)
+    epl, epa, epb = oracle.overlaps(reads, l_min)
+    assert np.array_equal(_np(pl, np.uint8), epl) and int((epl == 80).sum()) >= 4200
+    assert np.array_equal(_np(pa, np.uint32), epa)
+    assert np.array_equal(_np(pb, np.uint32), epb)
+
+
 def _random_candidates(n, k, rng, lens):
     V = 2 * n
     k = min(k, len(lens) * V * (V - 1) // 4)  # at most half of all distinct (l, a, b)
@@ -422,6 +453,38 @@ def test_region_overflow_falls_back_to_exact_path(tmp_path):
     env = dict(os.environ, LASAGNA_TEST_TIGHT_REGIONS="1", PYTHONPATH=ROOT)
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                          cwd=ROOT, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+
+
+@gpu
+def test_host_ascii_streamed_in_chunks():
+    """Page-locked host ASCII streamed by DMA in many chunks (LASAGNA_TEST_A1_CHUNK = 37 x 512
+    reads, a ragged last chunk): greedy graph and packed rows equal the oracle; a bad byte in a
+    late chunk is reported with its global read index."""
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, torch, readgen, oracle\n"
+        "import paper_conf_ipps_goswamilsp18_b200 as lz\n"
+        "reads = readgen.config_reads('cfg2', n=400_001)\n"
+        "n, L = reads.shape\n"
+        "g = lz.GreedyGraph(n, L, 63, 'cuda')\n"
+        "r = g.from_ascii(torch.from_numpy(reads).pin_memory())\n"
+        "es, eo, m, acc = oracle.greedy_graph(reads, 63)\n"
+        "assert r.stats['bucketed'] == 1 and r.stats['key_sort_bits'] == 16\n"
+        "assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), es)\n"
+        "assert np.array_equal(r.olen.cpu().numpy(), eo)\n"
+        "assert np.array_equal(g.packed.cpu().numpy().view(np.uint64), oracle.pack(reads, lz.words_per_read(L)))\n"
+        "bad = reads.copy(); bad[399_990, 5] = ord('N'); bad[399_999, 0] = ord('-')\n"
+        "try:\n"
+        "    g.from_ascii(torch.from_numpy(bad).pin_memory())\n"
+        "    raise SystemExit('bad read not reported')\n"
+        "except lz.LasagnaError as e:\n"
+        "    assert 'read 399990' in str(e), str(e)\n"
+        "print('ok')\n")
+    env = dict(os.environ, LASAGNA_TEST_A1_CHUNK=str(37 * 512), PYTHONPATH=ROOT)
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                         cwd=ROOT, timeout=900)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
 
 
