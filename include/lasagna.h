@@ -151,7 +151,7 @@ LASAGNA_API lasagna_status lasagna_greedy_graph(const uint64_t *packed, uint64_t
  * host reads over PCIe overlaps the fingerprint computation.
  *   ascii      n*L bytes, device memory or PAGE-LOCKED host memory.  Host input is streamed in
  *              by the DMA engine (a8 level 2): chunks of 512 Ki reads on an internal
- *              copy stream into a three-buffer ring inside the workspace, each chunk's table
+ *              copy stream into a ring of up to 64 chunk buffers inside the workspace, each chunk's table
  *              pass launched on `stream` as soon as it lands (event-ordered); off the fast
  *              path, or when the workspace has no room for the ring, it is read in place
  *              (zero-copy).  The host buffer must stay valid until the call returns.

@@ -272,16 +272,14 @@ struct PhaseTimer {
 };
 
 // a8 level 2: the host -> device leg of the semi-streaming driver.  The ASCII
-// reads (page-locked host memory) are copied by the DMA engine in chunks into a ring of three
-// device buffers on a copy stream, and each chunk's fused a1 + a2 + level-1 partition launch
-// runs on the call's stream as soon as its copy has landed, while the next chunks are in
-// flight (events order copy k before scatter k, and scatter k before the copy that reuses its
-// slot).  The ring lives in the level-2 region buffer, which nothing touches before the refine
+// reads (page-locked host memory) are copied by the DMA engine in chunks into a ring of device
+// buffers on a copy stream, and each chunk's fused a1 + a2 + level-1 partition launch runs on
+// the call's stream as soon as its copy has landed, while the next chunks are in flight
+// (events order copy k before scatter k, and scatter k before a copy that reuses its slot).  The ring lives in the level-2 region buffer, which nothing touches before the refine
 // pass that follows.  Chunks are whole scatter CTAs (multiples of 512 reads); per-(CTA, bin)
 // reservations accumulate across the launches exactly as within one.
 static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const char *host)
 {
-    constexpr int NSLOT = 3;
     const uint64_t n = base.n, L = base.L;
     // 512 Ki reads per chunk (~53 MB at L = 101); LASAGNA_TEST_A1_CHUNK (tests only) overrides
     static const uint64_t want = [] {
@@ -289,15 +287,22 @@ static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const c
         const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
         return v ? v : (uint64_t)512 * 1024;
     }();
-    uint64_t chunk = std::max<uint64_t>(512, want / 512 * 512);
-    const uint64_t fit = r.lay.tabB_bytes / (NSLOT * L);
-    chunk = std::min(chunk, fit / 512 * 512);
-    if (chunk == 0) return launch_scatter_table(base, r.s); // no room: zero-copy reads
-    unsigned char *ring = reinterpret_cast<unsigned char *>(r.tab[1]);
+    const uint64_t chunk = std::max<uint64_t>(512, want / 512 * 512);
     const size_t slot_bytes = (size_t)chunk * L;
+    const uint64_t nchunk = ceil_div(n, chunk);
+    // as many ring slots as the region buffer holds, up to one per chunk (then the copy engine
+    // never waits for a table pass, e.g. while another call's kernels hold the SMs), at most 64
+    static const uint64_t max_slots = [] { // LASAGNA_TEST_A1_SLOTS (tests only) lowers it
+        const char *e = getenv("LASAGNA_TEST_A1_SLOTS");
+        const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
+        return v >= 3 && v < 64 ? v : (uint64_t)64;
+    }();
+    const uint64_t nslot = std::min<uint64_t>({nchunk, max_slots, r.lay.tabB_bytes / slot_bytes});
+    if (nslot < std::min<uint64_t>(nchunk, 3)) return launch_scatter_table(base, r.s); // zero-copy
+    unsigned char *ring = reinterpret_cast<unsigned char *>(r.tab[1]);
     struct Res {
         cudaStream_t cs = nullptr;
-        cudaEvent_t ev[2 * NSLOT + 1] = {};
+        std::vector<cudaEvent_t> ev;
         ~Res()
         {
             for (auto e : ev)
@@ -306,19 +311,21 @@ static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const c
         }
     } res;
     LSG_CUDA(cudaStreamCreateWithFlags(&res.cs, cudaStreamNonBlocking));
+    // copied: two alternating events (a wait snapshots the event's latest record); consumed:
+    // one per ring slot, recorded after the table pass that read it
+    const uint64_t nreuse = nchunk > nslot ? nslot : 0;
+    res.ev.assign(3 + nreuse, nullptr);
     for (auto &e : res.ev) LSG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    cudaEvent_t *copied = res.ev, *consumed = res.ev + NSLOT, start = res.ev[2 * NSLOT];
+    cudaEvent_t start = res.ev[0], *copied = &res.ev[1], *consumed = res.ev.data() + 3;
     LSG_CUDA(cudaEventRecord(start, r.s)); // the ring's previous users (an earlier call) are done
     LSG_CUDA(cudaStreamWaitEvent(res.cs, start, 0));
-    uint32_t k = 0;
-    for (uint64_t r0 = 0; r0 < n; r0 += chunk, ++k) {
-        const int slot = (int)(k % NSLOT);
-        const uint64_t m = std::min(chunk, n - r0);
-        if (k >= (uint32_t)NSLOT) LSG_CUDA(cudaStreamWaitEvent(res.cs, consumed[slot], 0));
+    for (uint64_t k = 0; k < nchunk; ++k) {
+        const uint64_t slot = k % nslot, r0 = k * chunk, m = std::min(chunk, n - r0);
+        if (k >= nslot) LSG_CUDA(cudaStreamWaitEvent(res.cs, consumed[slot], 0));
         LSG_CUDA(cudaMemcpyAsync(ring + slot * slot_bytes, host + r0 * L, m * L,
                                  cudaMemcpyHostToDevice, res.cs));
-        LSG_CUDA(cudaEventRecord(copied[slot], res.cs));
-        LSG_CUDA(cudaStreamWaitEvent(r.s, copied[slot], 0));
+        LSG_CUDA(cudaEventRecord(copied[k & 1], res.cs));
+        LSG_CUDA(cudaStreamWaitEvent(r.s, copied[k & 1], 0));
         ScatterArgs sa = base;
         sa.ascii = ring + slot * slot_bytes;
         sa.n = m;
@@ -326,7 +333,7 @@ static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const c
         sa.packed_out = base.packed_out + r0 * base.stride;
         lasagna_status rc = launch_scatter_table(sa, r.s);
         if (rc != LASAGNA_OK) return rc;
-        LSG_CUDA(cudaEventRecord(consumed[slot], r.s));
+        if (nreuse) LSG_CUDA(cudaEventRecord(consumed[slot], r.s));
     }
     return LASAGNA_OK;
 }
@@ -525,6 +532,10 @@ static lasagna_status resolve_ascii(const char *ascii, const char **dev, bool *i
     *dev = ascii;
     if (is_host) *is_host = at.type == cudaMemoryTypeHost;
     if (at.type == cudaMemoryTypeHost) {
+        void *mapped = nullptr;
+        if (!at.devicePointer && cudaHostGetDevicePointer(&mapped, (void *)ascii, 0) == cudaSuccess)
+            at.devicePointer = mapped;
+        cudaGetLastError();
         if (!at.devicePointer) {
             set_error("ascii: page-locked host memory is not mapped into the device");
             return LASAGNA_EINVAL;
@@ -737,7 +748,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     LSG_CUDA(cudaStreamSynchronize(s));
     if (ascii_dev) {
         unsigned long long fb = 0;
-        LSG_CUDA(cudaMemcpy(&fb, first_bad, 8, cudaMemcpyDeviceToHost));
+        LSG_CUDA(cudaMemcpyAsync(&fb, first_bad, 8, cudaMemcpyDeviceToHost, s));
+        LSG_CUDA(cudaStreamSynchronize(s));
         if (fb != ~0ull) {
             set_error("read %llu holds a byte outside ACGTacgt", fb);
             return LASAGNA_EINVAL;

@@ -257,6 +257,77 @@ class GreedyGraph:
         raise LasagnaError(ENOSPC, "greedy_graph: could not size the workspace")
 
 
+class GraphPipeline:
+    """Greedy graphs of a stream of read batches with two batches in flight (a8 level 2 across
+    batches): batch k+1's host -> device copy (one copy stream, so the copies run back to back
+    at the link's rate) overlaps batch k's device work and its result read-back.  Two
+    GreedyGraph runners with their own workspaces and device input buffers, one compute stream
+    and one host thread each (a call blocks its thread until its stream is done); batch k goes
+    to runner k % 2, whose buffer is refilled only after its previous call returned.
+    Plumbing only: every step of the path runs in liblasagna.so (lasagna_greedy_graph_ascii on
+    the device copy of the batch)."""
+
+    def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0):
+        self.n, self.L, self.device = n, L, torch.device(device)
+        self.runners = [GreedyGraph(n, L, l_min, self.device, lengths_per_pass) for _ in range(2)]
+        self.bufs = [torch.empty((n, L), dtype=torch.uint8, device=self.device) for _ in range(2)]
+        self.copy = torch.cuda.Stream(self.device)
+        self.lanes = [torch.cuda.Stream(self.device) for _ in range(2)]
+
+    def run(self, batches, outs) -> None:
+        """batches[k]: (n, L) uint8 page-locked host tensor; outs[k]: (succ, olen) page-locked
+        host tensors receiving batch k's result.  Returns when every result is on the host."""
+        import queue
+        import threading
+        q = [queue.Queue(), queue.Queue()]
+        free = [threading.Semaphore(1), threading.Semaphore(1)]
+        errors = []
+
+        def lane(j: int) -> None:
+            try:
+                torch.cuda.set_device(self.device)
+                with torch.cuda.stream(self.lanes[j]):
+                    while True:
+                        item = q[j].get()
+                        if item is None:
+                            return
+                        ev, k = item
+                        # wait on the host, not in-stream: a stream parked on an event wait can
+                        # hold a hardware queue that the other lane's kernels share
+                        ev.synchronize()
+                        r = self.runners[j].from_ascii(self.bufs[j], stats=False)
+                        outs[k][0].copy_(r.succ, non_blocking=True)
+                        outs[k][1].copy_(r.olen, non_blocking=True)
+                        self.lanes[j].synchronize()
+                        free[j].release()
+            except BaseException as e:  # re-raised by the caller's thread
+                errors.append(e)
+                free[j].release()
+
+        th = [threading.Thread(target=lane, args=(j,)) for j in range(2)]
+        for t in th:
+            t.start()
+        try:
+            for k, b in enumerate(batches):
+                j = k % 2
+                free[j].acquire()  # runner j's previous batch has returned
+                if errors:
+                    break
+                self.copy.wait_stream(self.lanes[j])
+                with torch.cuda.stream(self.copy):
+                    self.bufs[j].copy_(b, non_blocking=True)
+                    ev = torch.cuda.Event()
+                    ev.record(self.copy)
+                q[j].put((ev, k))
+        finally:
+            for j in range(2):
+                q[j].put(None)
+            for t in th:
+                t.join()
+        if errors:
+            raise errors[0]
+
+
 def greedy_graph(packed: torch.Tensor, n: int, L: int, l_min: int, lengths_per_pass: int = 0,
                  stats: bool = True) -> GraphResult:
     g = GreedyGraph(n, L, l_min, packed.device, lengths_per_pass)

@@ -457,10 +457,12 @@ def test_region_overflow_falls_back_to_exact_path(tmp_path):
 
 
 @gpu
-def test_host_ascii_streamed_in_chunks():
+@pytest.mark.parametrize("slots", ["64", "3"])
+def test_host_ascii_streamed_in_chunks(slots):
     """Page-locked host ASCII streamed by DMA in many chunks (LASAGNA_TEST_A1_CHUNK = 37 x 512
-    reads, a ragged last chunk): greedy graph and packed rows equal the oracle; a bad byte in a
-    late chunk is reported with its global read index."""
+    reads, a ragged last chunk), one ring slot per chunk or three reused slots: greedy graph
+    and packed rows equal the oracle; a bad byte in a late chunk is reported with its global
+    read index."""
     import subprocess
     import sys
     code = (
@@ -482,7 +484,8 @@ def test_host_ascii_streamed_in_chunks():
         "except lz.LasagnaError as e:\n"
         "    assert 'read 399990' in str(e), str(e)\n"
         "print('ok')\n")
-    env = dict(os.environ, LASAGNA_TEST_A1_CHUNK=str(37 * 512), PYTHONPATH=ROOT)
+    env = dict(os.environ, LASAGNA_TEST_A1_CHUNK=str(37 * 512), LASAGNA_TEST_A1_SLOTS=slots,
+               PYTHONPATH=ROOT)
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                          cwd=ROOT, timeout=900)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
