@@ -457,6 +457,25 @@ def test_region_overflow_falls_back_to_exact_path(tmp_path):
 
 
 @gpu
+def test_graph_pipeline_batches():
+    """GraphPipeline (two batches in flight, host -> device copy of batch k+1 overlapping batch
+    k): five different read batches, each result equal to the oracle's for that batch."""
+    import torch
+    import paper_conf_ipps_goswamilsp18_b200 as lz
+    n, L, l_min = 60_000, 100, 63
+    batches = [readgen.reads(100 + k, 300_000, n, L, 0.01) for k in range(5)]
+    pipe = lz.GraphPipeline(n, L, l_min, "cuda")
+    hb = [torch.from_numpy(b).pin_memory() for b in batches]
+    outs = [(torch.empty(2 * n, dtype=torch.int32).pin_memory(),
+             torch.empty(2 * n, dtype=torch.uint8).pin_memory()) for _ in batches]
+    pipe.run(hb, outs)
+    for b, (succ, olen) in zip(batches, outs):
+        esucc, eolen, m, acc = oracle.greedy_graph(b, l_min)
+        assert np.array_equal(succ.numpy().view(np.uint32), esucc)
+        assert np.array_equal(olen.numpy(), eolen)
+
+
+@gpu
 @pytest.mark.parametrize("slots", ["64", "3"])
 def test_host_ascii_streamed_in_chunks(slots):
     """Page-locked host ASCII streamed by DMA in many chunks (LASAGNA_TEST_A1_CHUNK = 37 x 512
