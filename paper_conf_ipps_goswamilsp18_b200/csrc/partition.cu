@@ -544,6 +544,7 @@ bucket_join_kernel(BucketJoinArgs b)
                 const uint32_t tag = epoch << 16;
                 const uint32_t nP = d.nP, nS = d.nS;
                 // ---- build: chained hash of the build entries + the 64 Ki-bit filter
+#pragma unroll 2
                 for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += BJ_THREADS) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
@@ -588,6 +589,7 @@ bucket_join_kernel(BucketJoinArgs b)
                     const uint32_t hk = (uint32_t)(e >> kshift) & 0xFFFFu;
                     return ((bl[hk >> 5] >> (hk & 31u)) & 1u) != 0;
                 };
+#pragma unroll 2
                 for (uint32_t t0 = 0; t0 < nS; t0 += BJ_THREADS) { // block-uniform trip count
                     const uint32_t t = t0 + threadIdx.x;
                     bool pass = false;

@@ -80,8 +80,8 @@ def main() -> None:
     with open(os.path.join(prof, f"{tag}_launches.md"), "w") as f:
         f.write(f"# {tag}: kernel launch list of one bench step\n\n")
         f.write("`ncu --metrics gpu__time_duration.sum --clock-control none` over "
-                "`bench.py --steps 1 --warmup 1` (4 steps executed: warm-up, timed, e2e warm-up, "
-                "e2e; pack_kernel's e2e launches read host memory over PCIe). Cold-cache, "
+                "`bench.py --steps 1 --warmup 1` (every step the bench runs: warm-up, timed, "
+                "the serial and pipelined e2e legs). Cold-cache, "
                 "serialised: compare shares, not absolute times.\n\n")
         f.write(launch_table(launches) + "\n")
     traffic_path = os.path.join(prof, "ncu_traffic.json")
