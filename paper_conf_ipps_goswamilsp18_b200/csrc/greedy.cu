@@ -269,7 +269,7 @@ lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *
 {
     const int sms = num_sms();
     const unsigned blocks = (unsigned)std::max<uint64_t>(
-        1, std::min<uint64_t>(ceil_div(g.cap, GREEDY_THREADS * GK), (uint64_t)sms * 8));
+        1, std::min<uint64_t>(ceil_div(g.cap, GREEDY_THREADS * GK), (uint64_t)sms * 16));
     // Round r: propose reads X (count ctr[2r % 3]) and lists the live pairs in Y
     // (ctr[(2r+1) % 3]); accept reads Y and writes the survivors back to X (ctr[(2r+2) % 3]).
     // A kernel never resets a counter another block of the same launch may still read: each
