@@ -268,7 +268,10 @@ class GraphPipeline:
     the device copy of the batch)."""
 
     def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0):
-        self.n, self.L, self.device = n, L, torch.device(device)
+        dev = torch.device(device)
+        if dev.index is None:  # the worker threads select the device by index
+            dev = torch.device(dev.type, torch.cuda.current_device())
+        self.n, self.L, self.device = n, L, dev
         self.runners = [GreedyGraph(n, L, l_min, self.device, lengths_per_pass) for _ in range(2)]
         self.bufs = [torch.empty((n, L), dtype=torch.uint8, device=self.device) for _ in range(2)]
         self.copy = torch.cuda.Stream(self.device)
