@@ -267,6 +267,36 @@ def test_cfg2_parity(lz, seed):
     assert np.array_equal(_np(r.olen, np.uint8), eolen)
 
 
+def _expected_false_matches(n: int, L: int, l_min: int, vbits: int) -> float:
+    """R12 closed form for the fingerprint hits the bases reject: per length, V/2 probe-side
+    and V/2 build-side canonical entries (V = 2n) whose stored keys carry the top 62 - vbits
+    bits of mix(min(H, Hr)); two unrelated entries agree on them with probability
+    2^-(62 - vbits), so E[false] = (L - l_min) (V/2)^2 / 2^(62 - vbits)."""
+    V = 2 * n
+    return (L - l_min) * (V / 2) ** 2 / 2.0 ** (62 - vbits)
+
+
+def _assert_poisson(observed: int, expected: float):
+    assert abs(observed - expected) <= 5 * expected ** 0.5 + 0.02 * expected, (observed, expected)
+
+
+@gpu
+def test_false_match_rate_closed_form(lz):
+    """Hash-collision rate (north star: "checked on hash-collision rates"): the fingerprint
+    hits the exact verification rejects at cfg2 match the R12 closed form (Poisson, 5 sigma).
+    A key layout that stored fewer fingerprint bits, or a mix that clustered keys, would show
+    here as a multiple of the expected count."""
+    import torch
+    cfg = readgen.CONFIGS["cfg2"]
+    reads = readgen.config_reads(cfg)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min)
+    vbits = max(1, (2 * cfg.n - 1).bit_length())  # ceil(log2 V), lasagna.h key layout
+    exp = _expected_false_matches(cfg.n, cfg.L, cfg.l_min, vbits)
+    assert exp > 100
+    _assert_poisson(r.stats["fp_false_matches"], exp)
+
+
 def _palindrome_rich_reads(seed: int, G: int, n: int, L: int, every: int, plen: int) -> np.ndarray:
     """Error-free reads (half reverse-complemented) of a random genome in which a reverse-
     complement palindrome of length plen starts every `every` bases: reads starting at one
@@ -621,6 +651,9 @@ def test_cfg3_full_size_parity_and_invariants(lz):
     st = r.stats
     del g, r
     torch.cuda.empty_cache()
+    # R12 collision rate at full size (~1.34 M rejected hits expected)
+    vbits = max(1, (2 * cfg.n - 1).bit_length())  # ceil(log2 V), lasagna.h key layout
+    _assert_poisson(st["fp_false_matches"], _expected_false_matches(cfg.n, cfg.L, cfg.l_min, vbits))
     esucc, eolen, m, acc = oracle.greedy_graph(host.numpy(), cfg.l_min)
     assert st["n_pairs"] == m and st["n_greedy"] == acc
     assert np.array_equal(succ, esucc)
