@@ -254,15 +254,16 @@ def test_error_reads_expected_count():
 
 def test_fingerprint_collision_rate_small_modulus():
     """Hash-collision rate of the oracle's Rabin-Karp F with a small prime
-    modulus: N distinct 40-mers that share their last 32 bases and differ only in the first 8
+    modulus: N distinct 40-mers that share their last 24 bases and differ only in the first 16
     collide in pairs as a uniform hash would (Poisson, mean C(N, 2) / q), i.e. the leading
     bases reach the fingerprint through their place values.  Negative control: radix 4 modulo
     2^13, whose place values vanish beyond 7 bases, maps every one of them to one value."""
     rng = np.random.default_rng(11)
     q, N = 8191, 20_000
-    tail = "".join("ACGT"[i] for i in rng.integers(0, 4, 32))
-    heads = rng.choice(4 ** 8, N, replace=False)
-    strs = ["".join("ACGT"[(h >> (2 * k)) & 3] for k in range(8)) + tail for h in heads]
+    tail = "".join("ACGT"[i] for i in rng.integers(0, 4, 24))
+    heads = np.unique(rng.integers(0, 4 ** 16, N + 100, dtype=np.int64))[:N]
+    assert len(heads) == N
+    strs = ["".join("ACGT"[(int(h) >> (2 * k)) & 3] for k in range(16)) + tail for h in heads]
     vals = np.array([oracle.F(x, 5, q) for x in strs], dtype=np.int64)
     assert vals.min() >= 0 and vals.max() < q
     c = np.bincount(vals, minlength=q)
