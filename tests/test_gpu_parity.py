@@ -666,3 +666,24 @@ def test_cfg3_full_size_parity_and_invariants(lz):
     assert np.array_equal(succ[vs ^ 1].astype(np.int64), us ^ 1)
     assert np.all((olen[us] >= cfg.l_min) & (olen[us] <= cfg.L - 1))
     assert np.all((us >> 1) != (vs >> 1))
+
+
+def test_product_path_fails_loudly_without_the_library(monkeypatch, tmp_path):
+    """No CPU fallback: with liblasagna.so absent (and no nvcc to rebuild it) the binding
+    raises instead of computing anything; the package never imports the oracle."""
+    from paper_conf_ipps_goswamilsp18_b200 import lasagna as lz
+
+    def no_nvcc():
+        raise RuntimeError("nvcc not found")
+
+    monkeypatch.setattr(lz, "_lib", None)
+    monkeypatch.setattr(lz._build, "SO", str(tmp_path / "liblasagna.so"))
+    monkeypatch.setattr(lz._build, "stale", no_nvcc)
+    with pytest.raises((lz.LasagnaError, RuntimeError)):
+        lz.lib()
+    pkg = os.path.join(ROOT, "paper_conf_ipps_goswamilsp18_b200")
+    for name in os.listdir(pkg):
+        if name.endswith(".py"):
+            with open(os.path.join(pkg, name)) as f:
+                src = f.read()
+            assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), name
