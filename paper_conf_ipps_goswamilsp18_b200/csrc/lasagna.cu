@@ -665,8 +665,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     // spare bytes beyond the chosen layout enlarge the pair pool
     {
         size_t spare = *workspace_bytes - layout(g, G, cap, true).total;
-        cap += spare / 16 / 2;
-        while (cap > default_pool_cap(g) && layout(g, G, cap, true).total > *workspace_bytes) cap -= cap / 16 + 1;
+        cap += spare / 16; // pool + pool2: 16 B per pair (the status words shrink it below)
+        while (cap > default_pool_cap(g) && layout(g, G, cap, true).total > *workspace_bytes) cap -= cap / 256 + 1;
     }
     cudaStream_t s = (cudaStream_t)stream;
     Run r;
@@ -848,8 +848,8 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
     }
     {
         size_t spare = *workspace_bytes - layout(g, G, cap, false).total;
-        cap += spare / 16 / 2;
-        while (cap > default_pool_cap(g) && layout(g, G, cap, false).total > *workspace_bytes) cap -= cap / 16 + 1;
+        cap += spare / 16; // pool + pool2: 16 B per pair (the status words shrink it below)
+        while (cap > default_pool_cap(g) && layout(g, G, cap, false).total > *workspace_bytes) cap -= cap / 256 + 1;
     }
     cudaStream_t s = (cudaStream_t)stream;
     Run r;

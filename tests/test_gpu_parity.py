@@ -687,3 +687,26 @@ def test_product_path_fails_loudly_without_the_library(monkeypatch, tmp_path):
             with open(os.path.join(pkg, name)) as f:
                 src = f.read()
             assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), name
+
+
+@gpu
+@pytest.mark.parametrize("L,l_min,n,G,p_err", [(256, 200, 4000, 40_000, 0.0), (256, 255, 4000, 40_000, 0.0),
+                                             (64, 1, 3000, 20_000, 0.01), (255, 128, 3000, 30_000, 0.002)])
+def test_greedy_graph_extreme_lengths(lz, L, l_min, n, G, p_err):
+    """Edge shapes: the maximum read length (L = 256, four packed words), a single matched
+    length (l_min = L - 1), every length from 1 (millions of pairs: one length overflows the
+    default pair pool, so the call returns ENOSPC with a larger workspace and is retried), an
+    odd L near the maximum."""
+    import torch
+    reads = readgen.reads(7, G, n, L, p_err)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    for src in (torch.from_numpy(reads).cuda(), torch.from_numpy(reads).pin_memory()):
+        r = lz.greedy_graph(lz.load_reads(src), n, L, l_min)
+        assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc, (r.stats, m, acc)
+        assert np.array_equal(_np(r.succ, np.uint32), esucc)
+        assert np.array_equal(_np(r.olen, np.uint8), eolen)
+    pl, pa, pb = lz.overlaps(lz.load_reads(torch.from_numpy(reads).cuda()), n, L, l_min)
+    epl, epa, epb = oracle.overlaps(reads, l_min)
+    assert len(epl) == m
+    assert np.array_equal(_np(pa, np.uint32), epa) and np.array_equal(_np(pb, np.uint32), epb)
+    assert np.array_equal(_np(pl, np.uint8), epl)
