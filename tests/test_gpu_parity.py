@@ -710,3 +710,24 @@ def test_greedy_graph_extreme_lengths(lz, L, l_min, n, G, p_err):
     assert len(epl) == m
     assert np.array_equal(_np(pa, np.uint32), epa) and np.array_equal(_np(pb, np.uint32), epb)
     assert np.array_equal(_np(pl, np.uint8), epl)
+
+
+def test_planner_host_logic_without_gpu():
+    """a8 planner (host only, no CUDA call): the largest length group that fits the budget,
+    monotone in the budget, ENOSPC below the one-length workspace, and the greedy call's size
+    query agrees with the plan for that group."""
+    from paper_conf_ipps_goswamilsp18_b200 import lasagna as lz
+    n, L, l_min = 34_851_485, 101, 63  # cfg3
+    lp, ws = lz.plan(n, L, l_min, 170 << 30)
+    assert lp == L - l_min and 0 < ws <= 170 << 30
+    prev = (lp, ws)
+    for budget in (60 << 30, 30 << 30, 12 << 30, 6 << 30):
+        g, w = lz.plan(n, L, l_min, budget)
+        assert 1 <= g <= prev[0] and w <= budget and w <= prev[1], (budget, g, w)
+        q = ctypes.c_size_t(0)
+        assert lz.lib().lasagna_greedy_graph(None, n, L, l_min, g, None, ctypes.byref(q), None, None,
+                                             None, None) == lz.OK
+        assert q.value == w
+        prev = (g, w)
+    g, w = lz.plan(n, L, l_min, 1 << 20)
+    assert g == 0 and w > 1 << 20
