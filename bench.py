@@ -108,55 +108,107 @@ def _bus_id(torch, dev: int) -> str | None:
 
 
 # ------------------------------------------------------------------ CPU oracle baseline
-def cpu_baseline(reads: np.ndarray, l_min: int, target_s: float = 12.0) -> dict:
-    """The oracle as it stands, timed on a bounded prefix of the same read set."""
-    import oracle
+def _cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def _oracle_seconds(reads: np.ndarray, l_min: int, threads: int | None) -> tuple[float, int]:
+    """Time oracle.greedy_graph on `reads` in a child process with OMP_NUM_THREADS = threads
+    (the OpenMP runtime reads it once per process)."""
+    import tempfile
+    with tempfile.TemporaryDirectory() as d:
+        path = os.path.join(d, "reads.npy")
+        np.save(path, reads)
+        code = ("import sys, time, numpy as np, oracle\n"
+                "r = np.load(sys.argv[1]); oracle.lib()\n"
+                "t = time.perf_counter(); out = oracle.greedy_graph(r, int(sys.argv[2]))\n"
+                "print(time.perf_counter() - t, out[2])\n")
+        env = dict(os.environ, PYTHONPATH=ROOT)
+        if threads:
+            env["OMP_NUM_THREADS"] = str(threads)
+        out = subprocess.run([sys.executable, "-c", code, path, str(l_min)], env=env,
+                             capture_output=True, text=True, cwd=ROOT, timeout=1800)
+        if out.returncode != 0:
+            raise RuntimeError(out.stderr[-2000:])
+        t, m = out.stdout.split()
+        return float(t), int(m)
+
+
+def cpu_baseline(cfg, host_reads: np.ndarray, target_s: float = 12.0) -> dict:
+    """The oracle as it stands, timed on the box's host cores on a BOUNDED, coverage-preserving
+    sample of the workload: the reads that start in a genome window (same coverage, error rate
+    and length mix as the full set), sized to ~target_s of CPU work.  Plus the small configs at
+    one thread and all cores (SURVEY 8(d) timing rules)."""
+    import readgen
     cores = os.cpu_count() or 1
-    os.environ.setdefault("OMP_NUM_THREADS", str(cores))
-    oracle.lib()
-    n_total = reads.shape[0]
-    n0 = min(n_total, 50_000)
-    t = time.perf_counter()
-    oracle.greedy_graph(reads[:n0], l_min)
-    t0 = time.perf_counter() - t
-    n1 = int(min(n_total, max(n0, n0 * target_s / max(t0, 1e-3))))
-    t = time.perf_counter()
-    _, _, m, acc = oracle.greedy_graph(reads[:n1], l_min)
-    t1 = time.perf_counter() - t
-    return {"value": n1 / t1, "unit": "reads/s", "cores": int(os.environ["OMP_NUM_THREADS"]),
-            "kind": "oracle",
-            "sample": f"first {n1} reads of the workload (oracle.greedy_graph, exact-string "
-                      f"overlaps + sequential greedy; {m} read-end pairs), {t1:.2f} s"}
+    omp = int(os.environ.get("OMP_NUM_THREADS", cores))
+    n_probe = min(cfg.n, 200_000)
+    idx = readgen.window_sample(cfg, n_probe)
+    t0, _ = _oracle_seconds(host_reads[idx], cfg.l_min, omp)
+    n_s = int(min(cfg.n, max(len(idx), len(idx) * target_s / max(t0, 1e-3))))
+    idx = readgen.window_sample(cfg, n_s)
+    t1, m = _oracle_seconds(host_reads[idx], cfg.l_min, omp)
+    small = {}
+    for name, threads in (("cfg1", 1), ("cfg1", omp), ("cfg2", omp)):
+        c = readgen.CONFIGS[name]
+        ts, ms = _oracle_seconds(readgen.config_reads(c), c.l_min, threads)
+        small[f"{name}_{threads}t"] = {"s": round(ts, 3), "reads_per_s": c.n / ts,
+                                       "read_end_pairs": ms}
+    c2 = readgen.CONFIGS["cfg2"]
+    i2 = readgen.window_sample(c2, c2.n // 10)
+    ts, ms = _oracle_seconds(readgen.config_reads(c2)[i2], c2.l_min, 1)
+    small["cfg2_window_tenth_1t"] = {"s": round(ts, 3), "reads_per_s": len(i2) / ts,
+                                     "reads": len(i2), "read_end_pairs": ms}
+    return {"value": len(idx) / t1, "unit": "reads/s", "cores": omp, "kind": "oracle",
+            "cpu_model": _cpu_model(), "nproc": cores, "omp_num_threads": omp,
+            "sample": f"{len(idx)} reads of {cfg.name} starting in the first "
+                      f"{len(idx) / cfg.n:.4f} of the genome (same {cfg.n * cfg.L / cfg.G:.0f}x "
+                      f"coverage and error rate), oracle.greedy_graph (exact-string overlaps + "
+                      f"sequential greedy; {m} read-end pairs), {t1:.2f} s",
+            "small_configs": small}
 
 
 # ------------------------------------------------------------------ algorithmic bytes (DESIGN.md)
-def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict,
-             sm_mhz: float | None = None) -> dict:
+def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict, ms_step: float,
+             sm_mhz: float | None = None, ascii_fused: bool = True) -> dict:
     """Dominant phase and its achieved ALGORITHMIC GB/s (bytes per unit in DESIGN.md x units
-    per launch / CUDA-event time per launch)."""
+    per launch / CUDA-event time per launch), plus the whole step's algorithmic GB/s.  Stats
+    are summed over `steps` steps."""
     V = 2 * n
     N = V                         # table entries per length (one canonical entry per vertex)
     n_len = L - l_min
     G = stats["lengths_per_pass"]
+    W = 1 if L <= 32 else 2 if L <= 64 else 4 if L <= 128 else 8
     verify = 64.0 * (stats["n_pairs"] + stats["fp_false_matches"]) / max(1, n_len)
     bucketed = bool(stats.get("bucketed", 1))
+    # greedy: per pair and round 8 B read + 8 B live-list write + two 8 B proposals (propose),
+    # 8 B read + two 8 B best[] reads + 8 B survivor write (accept): 64 B
+    greedy_bytes = 64.0 * stats.get("greedy_pair_rounds", 0) / steps
+    passes = max(1, stats["passes"] // steps)
     if bucketed:
+        levels = max(1, stats.get("partition_levels", 2))
         per = {
-            # level-1 partition fused with the fingerprints: every key written once
-            "scatter_table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
-            # level-2 partition: every key read once and written once
+            # a1 (fused: ASCII read, packed rows written) + a2 + level-1 partition: every key
+            # written once, the packed rows read (or written) once per pass
+            "scatter_table_kernel": (stats["ms_table"], stats["passes"],
+                                     8.0 * G * N + 8.0 * W * n + (L * n / passes if ascii_fused else 0)),
+            # refine levels: every key read once and written once per level
             "refine_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
             # one join launch (one length): every key read once + verification loads
             "bucket_join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
         }
     else:
         per = {
-            # one onesweep pass over a group: every key read once and written once
             "onesweep_kernel": (stats["ms_sort"], stats["sort_launches"], 16.0 * G * N),
-            # one join launch (one length): the sorted table streamed once + verification loads
             "join_kernel": (stats["ms_search"], stats["search_launches"], 8.0 * N + verify),
-            # table: 4 keys (32 B) written per read per length, the packed read loaded once
-            "table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 32.0 * n),
+            "table_kernel": (stats["ms_table"], stats["passes"], 8.0 * G * N + 8.0 * W * n),
         }
     name = max(per, key=lambda k: per[k][0])
     ms, launches, bytes_per_launch = per[name]
@@ -170,9 +222,14 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict,
     except Exception:
         pass
     phases = {k: {"ms_per_step": v[0] / steps, "launches_per_step": v[1] / steps,
+                  "bytes_per_launch": v[2],
                   "gbs": (v[2] / (v[0] / 1e3 / max(1, v[1])) / 1e9) if v[0] > 0 else None}
               for k, v in per.items()}
-    phases["greedy"] = {"ms_per_step": stats["ms_greedy"] / steps}
+    gms = stats["ms_greedy"] / steps
+    phases["greedy"] = {"ms_per_step": gms, "bytes_per_step": greedy_bytes,
+                        "gbs": greedy_bytes / (gms / 1e3) / 1e9 if gms > 0 else None}
+    step_bytes = sum(v[2] * v[1] / steps for v in per.values()) + greedy_bytes
+    step_gbs = step_bytes / (ms_step / 1e3) / 1e9
     # Issue view of the same kernel (integer-ALU-bound kernels): warp instructions per launch
     # from the committed ncu capture (profiles/ncu_inst.json) over the live launch time, against
     # the SM issue peak = SMs x 4 schedulers x 1 warp instruction per cycle x the SM clock.
@@ -194,46 +251,236 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict,
     return {"bound": "hbm", "kernel": name, "achieved": round(achieved, 1),
             "peak": peak["hbm_gbs"], "peak_source": peak["source"], "unit": "GB/s",
             "frac": round(achieved / peak["hbm_gbs"], 4), "traffic": traffic,
-            "bytes_per_launch": bytes_per_launch, "issue": issue, "phases": phases}
+            "bytes_per_launch": bytes_per_launch, "issue": issue,
+            "step": {"bytes": step_bytes, "achieved": round(step_gbs, 1),
+                     "frac": round(step_gbs / peak["hbm_gbs"], 4)},
+            "phases": phases}
 
 
 # ------------------------------------------------------------------ reference arm (the oracle)
 def run_reference(args, cfg, rank: int) -> None:
+    """The reference arm: the oracle as it stands, on the host cores, each step a bounded
+    coverage-preserving sample of the workload (the reads of a genome window)."""
     if rank != 0:
         return
-    reads = readgen.config_reads(cfg, n=min(cfg.n, 4_000_000))
     import oracle
     cores = os.cpu_count() or 1
     os.environ.setdefault("OMP_NUM_THREADS", str(cores))
     oracle.lib()
-    # bounded per-step sample: ~10 s of CPU work per step
-    n0 = min(reads.shape[0], 50_000)
+    # bounded per-step sample: ~8 s of CPU work per step
+    idx = readgen.window_sample(cfg, min(cfg.n, 200_000))
+    def sample(ix):
+        out = np.empty((len(ix), cfg.L), dtype=np.uint8)
+        # reads are generated by index; a window sample is a sorted index list
+        lo = 0
+        while lo < len(ix):
+            hi = lo + 1
+            while hi < len(ix) and ix[hi] == ix[hi - 1] + 1 and hi - lo < 1 << 16:
+                hi += 1
+            out[lo:hi] = readgen.reads(cfg.seed, cfg.G, hi - lo, cfg.L, cfg.p_err, int(ix[lo]))
+            lo = hi
+        return out
+    reads = readgen.config_reads(cfg) if cfg.n <= 50_000_000 else None
+    take = (lambda ix: reads[ix]) if reads is not None else sample
     t = time.perf_counter()
-    oracle.greedy_graph(reads[:n0], cfg.l_min)
+    oracle.greedy_graph(take(idx), cfg.l_min)
     t0 = time.perf_counter() - t
-    ns = int(min(reads.shape[0], max(n0, n0 * 8.0 / max(t0, 1e-3))))
-    for _ in range(args.warmup if args.warmup < 1 else 1):
-        oracle.greedy_graph(reads[:ns], cfg.l_min)
+    ns = int(min(cfg.n, max(len(idx), len(idx) * 8.0 / max(t0, 1e-3))))
+    idx = readgen.window_sample(cfg, ns)
+    rs = take(idx)
+    for _ in range(min(args.warmup, 1)):
+        oracle.greedy_graph(rs, cfg.l_min)
     times, pairs = [], 0
     for _ in range(args.steps):
         t = time.perf_counter()
-        _, _, pairs, _ = oracle.greedy_graph(reads[:ns], cfg.l_min)
+        _, _, pairs, _ = oracle.greedy_graph(rs, cfg.l_min)
         times.append(time.perf_counter() - t)
     tot = sum(times)
-    value = ns * args.steps / tot
+    value = len(idx) * args.steps / tot
+    sample_txt = (f"{len(idx)} reads of {cfg.name} starting in the first {len(idx) / cfg.n:.4f} "
+                  f"of the genome (same coverage and error rate) per step")
     out = {"metric": METRIC, "value": value, "unit": "reads/s", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u64",
            "data": "synthetic", "impl": "reference",
-           "config": {"workload": f"{cfg.name}: {cfg.note}", "sample_reads": ns, "n": cfg.n,
+           "config": {"workload": f"{cfg.name}: {cfg.note}", "sample_reads": len(idx), "n": cfg.n,
                       "L": cfg.L, "l_min": cfg.l_min},
-           "overlap_edges_per_s": 2 * pairs * args.steps / tot,
+           "overlap_edges_per_s": pairs * args.steps / tot,
            "cpu_baseline": {"value": value, "unit": "reads/s",
                             "cores": int(os.environ["OMP_NUM_THREADS"]), "kind": "oracle",
-                            "sample": f"first {ns} reads of {cfg.name} per step"},
+                            "cpu_model": _cpu_model(), "nproc": cores, "sample": sample_txt},
            "e2e": {"value": value, "unit": "reads/s", "h2d_bytes_per_step": 0,
                    "d2h_bytes_per_step": 0},
            "gpu_launches": 0}
+    print(json.dumps(out), flush=True)
+
+
+# ------------------------------------------------------------------ semi-streaming configs (a8)
+def _graph_checks(succ, olen, l_min: int, L: int, chunk: int = 1 << 27) -> dict:
+    """Invariants of a greedy string graph, on the device in chunks (P:L37 complementary edges,
+    which with out-degree <= 1 also give in-degree <= 1; P:L105 length range; R9 no same-read
+    edge)."""
+    import torch
+    V = succ.numel()
+    edges = 0
+    for a in range(0, V, chunk):
+        b = min(V, a + chunk)
+        s = succ[a:b].to(torch.int64) & 0xFFFFFFFF
+        has = s != 0xFFFFFFFF
+        u = torch.nonzero(has).squeeze(1) + a
+        v = s[has]
+        edges += int(u.numel())
+        tw = succ[v ^ 1].to(torch.int64) & 0xFFFFFFFF
+        assert torch.equal(tw, u ^ 1), "missing complementary edge"
+        ol = olen[u].to(torch.int64)
+        assert torch.equal(ol, olen[v ^ 1].to(torch.int64)), "complementary edge length differs"
+        assert bool(((ol >= l_min) & (ol <= L - 1)).all()), "overlap length out of range"
+        assert bool(((u >> 1) != (v >> 1)).all()), "same-read edge"
+        assert bool((olen[a:b][~has] == 0).all()), "olen set without an edge"
+    return {"directed_edges": edges, "complementary": True, "in_degree_le_1": True,
+            "length_range": True, "no_same_read": True}
+
+
+def _sampled_overlaps(host: np.ndarray, succ: np.ndarray, olen: np.ndarray, k: int,
+                      seed: int = 1) -> int:
+    """Exact string check of k randomly sampled edges u -> succ[u]: suffix_olen(seq(u))
+    == prefix_olen(seq(succ[u])) on the ASCII reads."""
+    comp = np.zeros(256, dtype=np.uint8)
+    for a_, b_ in zip(b"ACGTacgt", b"TGCATGCA"):
+        comp[a_] = b_
+    rng = np.random.default_rng(seed)
+    us = np.nonzero(succ != 0xFFFFFFFF)[0]
+    pick = us[rng.integers(0, len(us), min(k, len(us)))]
+    for u in pick.tolist():
+        v = int(succ[u])
+        l = int(olen[u])
+        ru, rv = host[u >> 1], host[v >> 1]
+        su = comp[ru[::-1]] if u & 1 else ru
+        sv = comp[rv[::-1]] if v & 1 else rv
+        assert np.array_equal(su[len(su) - l:], sv[:l]), (u, v, l)
+    return len(pick)
+
+
+def main_streaming(args, cfg) -> None:
+    """cfg4/cfg5: the read set does not fit in HBM next to its tables (cfg5: 124.8 GB of ASCII,
+    a 1.1 TB table set), so one runner streams it: `e2e` = page-locked host ASCII -> DMA
+    chunks fused with a1/a2 -> length groups over the resident packed reads -> succ/olen in host
+    memory; `value` = the same graph from the resident packed reads (the inputs that stay in
+    HBM).  No full-size oracle fits the host (V*L bytes of oriented reads), so the result is
+    checked by its invariants on every edge, exact string checks of sampled edges, determinism
+    across runs, and equality with a run of one length per pass."""
+    import torch
+    import paper_conf_ipps_goswamilsp18_b200 as lz
+    assert args.warmup >= 3 or os.environ.get("BENCH_ALLOW_SHORT_WARMUP"), "W >= 3"
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    n, L, l_min = cfg.n, cfg.L, cfg.l_min
+    t = time.perf_counter()
+    host = torch.empty((n, L), dtype=torch.uint8).pin_memory()
+    t_pin = time.perf_counter() - t
+    t = time.perf_counter()
+    step_rows = 1 << 26
+    for a in range(0, n, step_rows):
+        b = min(n, a + step_rows)
+        readgen.reads_into(host.data_ptr() + a * L, cfg.seed, cfg.G, L, cfg.p_err, a, b)
+    t_gen = time.perf_counter() - t
+    runner = lz.GreedyGraph(n, L, l_min, dev, args.lengths_per_pass)
+    h_succ = torch.empty(2 * n, dtype=torch.int32).pin_memory()
+    h_olen = torch.empty(2 * n, dtype=torch.uint8).pin_memory()
+    stream = torch.cuda.current_stream(dev)
+
+    def e2e_step(stats: bool):
+        r = runner.from_ascii(host, stats=stats)
+        h_succ.copy_(r.succ, non_blocking=True)
+        h_olen.copy_(r.olen, non_blocking=True)
+        return r
+
+    for _ in range(args.warmup):
+        r = e2e_step(True)
+    torch.cuda.synchronize()
+    first_stats = dict(r.stats)
+    ref_succ = h_succ.numpy().copy()
+    ref_olen = h_olen.numpy().copy()
+    sampler = ClockSampler(_bus_id(torch, 0))
+    sampler.start()
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(stream)
+    for _ in range(args.steps):
+        e2e_step(False)
+    f1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = f0.elapsed_time(f1) / args.steps
+    deterministic = bool(np.array_equal(h_succ.numpy(), ref_succ) and
+                         np.array_equal(h_olen.numpy(), ref_olen))
+    # device-resident value: the packed reads stay in HBM
+    agg = {k: 0.0 for k in ["ms_table", "ms_sort", "ms_search", "ms_greedy"]}
+    cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes", "greedy_pair_rounds"]}
+    launches0 = lz.kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        r = runner(runner.packed, stats=True)
+        for k in agg:
+            agg[k] += r.stats[k]
+        for k in cnt:
+            cnt[k] += r.stats[k]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    launches = lz.kernel_launches() - launches0
+    clocks = sampler.stop()
+    ms_step = e0.elapsed_time(e1) / args.steps
+    st = dict(r.stats)
+    st.update(agg)
+    st.update(cnt)
+    same_as_packed = bool(np.array_equal(r.succ.cpu().numpy(), ref_succ))
+    checks = _graph_checks(r.succ, r.olen, l_min, L)
+    checks["sampled_exact_overlaps"] = _sampled_overlaps(host.numpy(), ref_succ.view(np.uint32),
+                                                         ref_olen, 20_000)
+    checks["deterministic_e2e"] = deterministic
+    checks["packed_equals_ascii_path"] = same_as_packed
+    peak = _peaks()
+    roof = roofline(st, n, L, l_min, args.steps, peak, ms_step, clocks.get("sm_mhz"),
+                    ascii_fused=False)
+    lpp_used = st["lengths_per_pass"]
+    if not args.no_verify_lpp1 and lpp_used > 1:
+        # a8 equality: the same graph with one length per pass (37 device passes at cfg5)
+        del runner
+        torch.cuda.empty_cache()
+        one = lz.GreedyGraph(n, L, l_min, dev, lengths_per_pass=1)
+        t = time.perf_counter()
+        r1 = one.from_ascii(host, stats=True)
+        checks["lpp1_seconds"] = time.perf_counter() - t
+        checks["lpp1_passes"] = r1.stats["passes"]
+        checks["lpp1_equal"] = bool(np.array_equal(r1.succ.cpu().numpy(), ref_succ) and
+                                    np.array_equal(r1.olen.cpu().numpy(), ref_olen))
+    out = {
+        "metric": METRIC, "value": n / (ms_step / 1e3), "unit": "reads/s", "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {cfg.note}", "n": n, "L": L, "l_min": l_min,
+                   "G": cfg.G, "p_err": cfg.p_err, "seed": cfg.seed,
+                   "lengths_per_pass": lpp_used, "passes": st["passes"] // args.steps,
+                   "partition_levels": st.get("partition_levels"),
+                   "key_sort_bits": st["key_sort_bits"],
+                   "resident": "packed reads (value); ASCII streamed from page-locked host "
+                               "memory every step (e2e)",
+                   "ascii_gb": n * L / 1e9,
+                   "table_set_gb": 8.0 * 2 * n * (L - l_min) / 1e9,
+                   "l2": "inputs larger than L2 and than HBM"},
+        "overlap_edges_per_s": st["n_pairs"] / (ms_step / 1e3),
+        "read_end_pairs": st["n_pairs"], "greedy_pairs": st["n_greedy"],
+        "fp_false_matches": st["fp_false_matches"], "greedy_rounds_max": st["rounds_max"],
+        "e2e": {"value": n / (e2e_ms / 1e3), "unit": "reads/s", "ms_per_step": e2e_ms,
+                "h2d_bytes_per_step": n * L, "d2h_bytes_per_step": 2 * n * 5,
+                "batches_in_flight": 1},
+        "first_e2e_stats": first_stats,
+        "host_setup_s": {"pin": t_pin, "generate": t_gen},
+        "checks": checks,
+        "roofline": roof,
+        "clocks": clocks,
+        "gpu_launches": launches,
+    }
     print(json.dumps(out), flush=True)
 
 
@@ -252,6 +499,8 @@ def main() -> None:
                     help="process-group backend of the multi-GPU path (gloo: ranks may share a GPU)")
     ap.add_argument("--force-dist", action="store_true",
                     help="run the sharded multi-GPU path even with one rank")
+    ap.add_argument("--no-verify-lpp1", action="store_true",
+                    help="cfg4/cfg5: skip the one-length-per-pass equality run")
     args = ap.parse_args()
     cfg = readgen.CONFIGS[args.config]
     if args.n:
@@ -266,6 +515,9 @@ def main() -> None:
     if world > 1 or args.force_dist:
         from paper_conf_ipps_goswamilsp18_b200 import dist
         dist.bench_main(args, cfg, METRIC, _peaks(), ClockSampler, _bus_id, cpu_baseline)
+        return
+    if cfg.name in ("cfg4", "cfg5"):
+        main_streaming(args, cfg)
         return
 
     import torch
@@ -300,7 +552,8 @@ def main() -> None:
     # ---- device-resident timed region
     sampler = ClockSampler(_bus_id(torch, 0))
     agg = {k: 0.0 for k in ["ms_table", "ms_sort", "ms_search", "ms_greedy"]}
-    cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes"]}  # summed over steps
+    cnt = {k: 0 for k in ["sort_launches", "search_launches", "passes",
+                          "greedy_pair_rounds"]}  # summed over steps
     sampler.start()
     torch.cuda.synchronize()
     launches0 = lz.kernel_launches()
@@ -366,7 +619,7 @@ def main() -> None:
         assert np.array_equal(outs[j][0].numpy(), ref_succ), f"lane {j} differs"
 
     peak = _peaks()
-    roof = roofline(st, n, L, l_min, args.steps, peak, clocks.get("sm_mhz"))
+    roof = roofline(st, n, L, l_min, args.steps, peak, ms_step, clocks.get("sm_mhz"))
     out = {
         "metric": METRIC, "value": value, "unit": "reads/s", "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
@@ -376,7 +629,9 @@ def main() -> None:
                    "lengths_per_pass": st["lengths_per_pass"], "passes": st["passes"] // args.steps,
                    "l2": "inputs larger than L2 (ASCII %.1f GB, key tables %.1f GB)"
                          % (n * L / 1e9, 16.0 * 2 * n * st["lengths_per_pass"] / 1e9)},
-        "overlap_edges_per_s": edges / (ms_step / 1e3),
+        # overlap edges = |P| (undirected read-end pairs); directed edges = 2|P|
+        "overlap_edges_per_s": st["n_pairs"] / (ms_step / 1e3),
+        "directed_overlap_edges_per_s": edges / (ms_step / 1e3),
         "read_end_pairs": st["n_pairs"], "greedy_pairs": st["n_greedy"],
         "fp_false_matches": st["fp_false_matches"], "greedy_rounds_max": st["rounds_max"],
         "e2e": {"value": n / (e2e_ms / 1e3), "unit": "reads/s", "ms_per_step": e2e_ms,
@@ -388,7 +643,7 @@ def main() -> None:
         "gpu_launches": launches,
     }
     if not args.no_cpu_baseline:
-        out["cpu_baseline"] = cpu_baseline(host.numpy(), l_min)
+        out["cpu_baseline"] = cpu_baseline(cfg, host.numpy())
     print(json.dumps(out), flush=True)
 
 

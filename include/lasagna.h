@@ -121,8 +121,12 @@ typedef struct {
     uint32_t sort_launches;    /* onesweep passes launched (each sorts a whole group)       */
     uint32_t search_launches;  /* search (join) launches, one per length                    */
     uint32_t bucketed;         /* 1: radix-partition path (partition.cu), 0: exact LSD path */
-    /* device time per phase, CUDA events on `stream` (ms) */
+    /* device time per phase, CUDA events on `stream` (ms).  ms_table covers a1 (when the
+     * staging is fused into the first pass), a2 and the level-1 partition: one kernel */
     float ms_table, ms_sort, ms_search, ms_greedy;
+    uint64_t greedy_pair_rounds; /* sum over greedy rounds of the candidate pairs visited    */
+    uint32_t partition_levels;   /* bucketed path: MSD partition levels (1..3); 0: exact path */
+    uint32_t reserved;
 } lasagna_stats;
 
 /* ---------------------------------------------------------------------------------------

@@ -73,6 +73,22 @@ __device__ __forceinline__ uint64_t canon_key(uint64_t H, uint64_t Hr, uint64_t 
     const uint64_t f = h < hr ? 0ull : (h > hr ? 1ull : 2ull);
     return (mix(c) & keep) | (f << vbits) | v;
 }
+// The bucketed path's form of the same entry (partition.cu): the top 8 bits of mix(min) pick
+// the level-1 region and are implied by the region an entry sits in, so the stored key drops
+// them and keeps the next 62 - vbits bits instead — 8 more fingerprint bits in every
+// comparison (R12: at vbits = 32, 30 stored + 8 implied = 38 bits instead of 30):
+//   key = (mix(min(H, Hr)) << 8) top (62 - vbits) bits | flag << vbits | v,  *d1 = mix >> 56.
+// `keep` is key_keep(vbits) in production; a test may clear low fingerprint bits from it.
+__device__ __forceinline__ uint64_t canon_key_d1(uint64_t H, uint64_t Hr, uint64_t keep,
+                                                 uint32_t vbits, uint64_t v, uint32_t *d1)
+{
+    const uint64_t h = exact61(H), hr = exact61(Hr);
+    const uint64_t c = h < hr ? h : hr;
+    const uint64_t f = h < hr ? 0ull : (h > hr ? 1ull : 2ull);
+    const uint64_t m = mix(c);
+    *d1 = (uint32_t)(m >> 56);
+    return ((m << 8) & keep) | (f << vbits) | v;
+}
 __device__ __forceinline__ uint32_t key_flag(uint64_t key, uint32_t vbits)
 {
     return (uint32_t)(key >> vbits) & 3u;

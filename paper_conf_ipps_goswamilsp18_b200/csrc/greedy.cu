@@ -82,12 +82,13 @@ __global__ void __launch_bounds__(GREEDY_THREADS)
 greedy_propose(const unsigned long long *pairs, const unsigned long long *count,
                unsigned long long cap, const uint32_t *claimed, unsigned long long *best,
                uint32_t epoch, unsigned long long *live, unsigned long long *live_count,
-               unsigned long long *reset, unsigned long long *book)
+               unsigned long long *reset, unsigned long long *book, unsigned long long *work)
 {
     const unsigned long long c = *count;
     const unsigned long long m = c < cap ? c : cap;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         *reset = 0;
+        atomicAdd(work, m);
         if (book) { // first round of a length: |P_l| bookkeeping
             atomicAdd(&book[1], c);
             atomicMax(&book[2], c);
@@ -185,13 +186,14 @@ __global__ void __launch_bounds__(FINISH_THREADS)
 greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
               unsigned long long *other, unsigned long long *other_count, uint32_t *claimed,
               unsigned long long *best, uint32_t epoch, uint32_t fast_rounds, uint32_t *succ,
-              uint8_t *olen, uint8_t l, unsigned long long *book)
+              uint8_t *olen, uint8_t l, unsigned long long *book, unsigned long long *work)
 {
     __shared__ unsigned long long s[TAIL_MAX];
     __shared__ uint32_t s_live, s_acc;
     uint32_t live = (uint32_t)*cur_count;
     uint32_t rounds = fast_rounds;
     if (threadIdx.x == 0) s_acc = 0;
+    if (threadIdx.x == 0 && live) atomicAdd(work, (unsigned long long)live);
     while (live > (uint32_t)TAIL_MAX) {
         for (uint32_t i = threadIdx.x; i < live; i += FINISH_THREADS) {
             const unsigned long long r = cur[i];
@@ -215,6 +217,7 @@ greedy_finish(unsigned long long *cur, const unsigned long long *cur_count,
         }
         __syncthreads();
         live = s_live;
+        if (threadIdx.x == 0 && live) atomicAdd(work, (unsigned long long)live);
         unsigned long long *t = cur;
         cur = other;
         other = t;
@@ -283,7 +286,8 @@ lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *
     for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
         greedy_propose<<<blocks, GREEDY_THREADS, 0, s>>>(X, ctr[(2 * r) % 3], g.cap, g.claimed, g.best,
                                                          e0 + r, Y, ctr[(2 * r + 1) % 3],
-                                                         ctr[(2 * r + 2) % 3], r == 0 ? g.book : nullptr);
+                                                         ctr[(2 * r + 2) % 3], r == 0 ? g.book : nullptr,
+                                                         g.work);
         LSG_LAUNCHED("greedy_propose");
         greedy_accept<<<blocks, GREEDY_THREADS, 0, s>>>(Y, ctr[(2 * r + 1) % 3], g.cap, g.claimed, g.best,
                                                         e0 + r, succ, olen, l, X, ctr[(2 * r + 2) % 3],
@@ -291,7 +295,8 @@ lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *
         LSG_LAUNCHED("greedy_accept");
     }
     greedy_finish<<<1, FINISH_THREADS, 0, s>>>(X, ctr[0], Y, ctr[1], g.claimed, g.best,
-                                               e0 + FAST_ROUNDS, FAST_ROUNDS, succ, olen, l, g.book);
+                                               e0 + FAST_ROUNDS, FAST_ROUNDS, succ, olen, l, g.book,
+                                               g.work);
     LSG_LAUNCHED("greedy_finish");
     return LASAGNA_OK;
 }

@@ -71,7 +71,9 @@ struct ScatterArgs {
     const uint64_t *packed;
     uint64_t n, read_offset;
     uint32_t L, stride, l_lo, l_hi, vbits;
-    uint64_t *out;      // [G][256][cap] level-1 regions (top 8 key bits); split: [G][256][2][cap]
+    uint64_t keep;      // stored fingerprint bits (key_keep(vbits); tests may clear low ones)
+    uint64_t *out;      // [G][256][cap] level-1 regions (top 8 bits of mix(min(H, Hr)), not
+                        // stored: common.cuh canon_key_d1); split: [G][256][2][cap]
                         // (half 0: flags 0/2 = build side, half 1: flag 1 = probe side)
     uint32_t *fill;     // [G][256] (split: [G][256][2])
     uint64_t cap;
@@ -88,9 +90,10 @@ struct RefineArgs {
     const uint64_t *in;
     const uint32_t *fill_in;
     uint64_t cap_in;
-    uint32_t dshift;    // this level's digit: bits [dshift, dshift + 8)
-    uint64_t *out;      // [regions][256][cap_out] (split: [regions][256][2][cap_out])
-    uint32_t *fill_out; // [regions][256] (split: [regions][256][2])
+    uint32_t dshift;    // this level's digit: key bits [dshift, dshift + dbits)
+    uint32_t dbits;     // 1..8
+    uint64_t *out;      // [regions][2^dbits][cap_out] (split: [regions][2^dbits][2][cap_out])
+    uint32_t *fill_out; // [regions][2^dbits] (split: [regions][2^dbits][2])
     uint64_t cap_out;
     uint32_t vbits;
     uint32_t *overflow;
@@ -113,6 +116,7 @@ struct GreedyBufs {
     unsigned long long *cnt, *cnt2;   // their fills (device); cnt: the input count
     unsigned long long *cnt3;         // third round counter (zero, like cnt2, on the first call)
     unsigned long long *book;         // device: [0] accepted, [1] sum |P_l|, [2] max |P_l|, [3] max rounds
+    unsigned long long *work;         // device: sum over rounds of the pairs a round visits
     unsigned long long *best;         // u64 [V]: epoch-tagged proposals, zeroed once per call
     uint32_t *claimed;                // bitmap of claimed read ends (2n bits)
     unsigned long long cap;

@@ -34,20 +34,36 @@ lasagna_status cuda_status(cudaError_t e, const char *what)
     return LASAGNA_ECUDA;
 }
 
+// Test hooks and tuning knobs come from the environment, read on every call (so a test can
+// set one in-process, around one call).  Production runs set none of them.
+static uint64_t env_u64(const char *name, uint64_t dflt)
+{
+    const char *e = getenv(name);
+    return (e && *e) ? strtoull(e, nullptr, 10) : dflt;
+}
+static bool env_flag(const char *name, char first)
+{
+    const char *e = getenv(name);
+    return e && e[0] == first;
+}
+
 // ------------------------------------------------------------------ planning
 // Geometry of the key tables:
 //   N = V entries per length (one canonical entry per vertex, common.cuh), V = 2n vertices
 //   key = mix(min(H, Hr)) top (62 - vbits) bits | flag << vbits | vertex id,
 //   vbits = ceil(log2 V)
-//   radix-sorted by the top T = 8P key bits, P = ceil((log2 N - 11.5) / 8) passes, so a
-//   T-bit bucket holds ~N / 2^T <= ~2.9K entries (one shared-memory join tile)
+//   grouped by the top T bits of mix(min(H, Hr)) so that a T-bit bucket holds
+//   ~N / 2^T <= ~2.9K entries (one shared-memory join window):
+//   P = ceil((log2 N - 11.5) / 8) levels; T = 8 (P - 1) + dlast, dlast = 8 for P <= 2 and
+//   ceil(log2 N - 11.5) - 16 for P = 3 (cfg4/cfg5: 4)
 struct Geometry {
     uint64_t n, V, N;
     uint32_t L, l_min, n_len, vbits, T;
-    // bucketed path (partition.cu): P = T/8 MSD levels, region capacities with slack
-    uint32_t P;
-    uint64_t cap1;          // level-1 region capacity (unsplit, P = 2)
-    uint64_t half1, half2;  // half-bucket capacities of the final level (P = 1 / P = 2)
+    // bucketed path (partition.cu): P MSD levels (8, 8, dlast bits), capacities with slack
+    uint32_t P, dlast;
+    uint64_t cap1, cap2;    // unsplit region capacities of levels 1 and 2 (when not final)
+    uint64_t half;          // half-bucket capacity of the final level
+    uint64_t n_buckets;     // final-level buckets per length (2^T)
 };
 
 // capacity of a region expecting `mean` keys: mean + 8 sigma + 32 (multinomial occupancy;
@@ -55,8 +71,7 @@ struct Geometry {
 static uint64_t region_cap(double mean)
 {
     // LASAGNA_TEST_TIGHT_REGIONS=1 (tests only): half-size regions force the overflow fallback
-    static const bool tight = getenv("LASAGNA_TEST_TIGHT_REGIONS") != nullptr;
-    if (tight) return ((uint64_t)(mean / 2) + 2) & ~1ull;
+    if (getenv("LASAGNA_TEST_TIGHT_REGIONS")) return ((uint64_t)(mean / 2) + 2) & ~1ull;
     uint64_t c = (uint64_t)std::ceil(mean + 8.0 * std::sqrt(mean) + 32.0);
     return (c + 1) & ~1ull;
 }
@@ -80,12 +95,22 @@ static Geometry geometry(uint64_t n, uint32_t L, uint32_t l_min)
     g.vbits = std::max<uint32_t>(1, ceil_log2(g.V));
     const double lg = g.N > 1 ? std::log2((double)g.N) : 0.0;
     int P = (int)std::ceil((lg - 11.5) / 8.0);
-    P = std::max(1, std::min(P, 4));
-    g.T = std::min<uint32_t>(8u * (uint32_t)P, 64u - FLAG_BITS - g.vbits);
-    g.P = g.T / 8;
+    P = std::max(1, std::min(P, 3)); // 2n < 2^32: log2 N - 11.5 < 20.5
+    // LASAGNA_TEST_LEVELS / LASAGNA_TEST_LAST_BITS (tests only): force the cfg4/cfg5 geometry
+    // (three levels, a short last digit) at sizes the oracle checks
+    P = (int)std::max<uint64_t>(1, std::min<uint64_t>(3, env_u64("LASAGNA_TEST_LEVELS", P)));
+    g.P = (uint32_t)P;
+    g.dlast = 8;
+    if (P == 3) {
+        const int d = (int)std::ceil(lg - 11.5) - 16;
+        g.dlast = (uint32_t)std::max(1, std::min(8, d));
+        g.dlast = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(8, env_u64("LASAGNA_TEST_LAST_BITS", g.dlast)));
+    }
+    g.T = 8u * (g.P - 1) + g.dlast;
+    g.n_buckets = 1ull << g.T;
     g.cap1 = region_cap((double)g.N / 256.0);
-    g.half1 = region_cap((double)g.N / 512.0);
-    g.half2 = region_cap((double)g.N / 131072.0);
+    g.cap2 = region_cap((double)g.N / 65536.0);
+    g.half = region_cap((double)g.N / (double)(2 * g.n_buckets));
     return g;
 }
 
@@ -95,14 +120,14 @@ struct Layout {
     uint32_t G;          // lengths per group
     uint64_t pool_cap;   // pair pool capacity (pairs)
     size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, fill1,
-        fill2, total;
+        fill2, fill3, total;
     size_t tabB_bytes;   // tabB's size (the level-2 regions; the a1 staging ring before them)
 };
 
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
 enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR_FOUND = 8,
-       CTR_POOL3 = 9, CTR64_N = 10 };
+       CTR_POOL3 = 9, CTR_WORK = 10, CTR64_N = 11 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -115,16 +140,20 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
         off += align256(bytes);
         return o;
     };
-    // tabA/tabB: the exact path's LSD ping-pong buffers, or the bucketed path's level-1 and
-    // level-2 regions (with slack)
+    // tabA/tabB: the exact path's LSD ping-pong buffers, or the bucketed path's levels with
+    // slack: level 1 in tabA, level 2 in tabB, level 3 (P = 3) in tabA again
     const size_t exact_b = (size_t)G * g.N * 8;
-    const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half1 : 256 * g.cap1) * 8;
-    const size_t lvl2_b = g.P >= 2 ? (size_t)G * 131072 * g.half2 * 8 : 0;
-    l.tabA = take(std::max(exact_b, lvl1_b));
+    const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half : 256 * g.cap1) * 8;
+    const size_t lvl2_b = g.P == 2   ? (size_t)G * 131072 * g.half * 8
+                          : g.P == 3 ? (size_t)G * 65536 * g.cap2 * 8
+                                     : 0;
+    const size_t lvl3_b = g.P == 3 ? (size_t)G * 2 * g.n_buckets * g.half * 8 : 0;
+    l.tabA = take(std::max({exact_b, lvl1_b, lvl3_b}));
     l.tabB_bytes = std::max(exact_b, lvl2_b);
     l.tabB = take(l.tabB_bytes);
     l.fill1 = take((size_t)G * 512 * 4);
-    l.fill2 = take(g.P >= 2 ? (size_t)G * 131072 * 4 : 4);
+    l.fill2 = take(g.P == 2 ? (size_t)G * 131072 * 4 : g.P == 3 ? (size_t)G * 65536 * 4 : 4);
+    l.fill3 = take(g.P == 3 ? (size_t)G * 2 * g.n_buckets * 4 : 4);
     l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
     l.status = take(l.status_bytes);
     l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
@@ -141,15 +170,11 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     return l;
 }
 
-// The bucketed path (partition.cu) serves T <= 16 (P <= 2); LASAGNA_PATH=exact forces the
-// exact LSD-sort path (also the fallback when a slack region overflows).
+// The bucketed path (partition.cu) serves every geometry (P <= 3); LASAGNA_PATH=exact forces
+// the exact LSD-sort path (also the fallback when a slack region overflows).
 static bool use_bucketed(const Geometry &g)
 {
-    static const bool force_exact = [] {
-        const char *e = getenv("LASAGNA_PATH");
-        return e && e[0] == 'e';
-    }();
-    return !force_exact && g.P >= 1 && g.P <= 2;
+    return !env_flag("LASAGNA_PATH", 'e') && g.P >= 1 && g.P <= 3;
 }
 
 static uint64_t default_pool_cap(const Geometry &g)
@@ -201,7 +226,7 @@ struct Run {
     const char *ascii_host = nullptr;     // ... from this page-locked host copy (chunked DMA)
     uint64_t *packed_out = nullptr;
     unsigned long long *first_bad = nullptr;
-    uint32_t *fill1, *fill2;
+    uint32_t *fill1, *fill2, *fill3;
     unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
     const uint32_t *claimed = nullptr; // greedy mode: the join drops pairs with a claimed end
@@ -214,6 +239,7 @@ struct Run {
         hist = at<uint32_t>(lay.hist);
         fill1 = at<uint32_t>(lay.fill1);
         fill2 = at<uint32_t>(lay.fill2);
+        fill3 = at<uint32_t>(lay.fill3);
         sctx.status = at<unsigned long long>(lay.status);
         sctx.status_bytes = lay.status_bytes;
         sctx.tile_ctrs = at<uint32_t>(lay.ctrs);
@@ -282,21 +308,16 @@ static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const c
 {
     const uint64_t n = base.n, L = base.L;
     // 512 Ki reads per chunk (~53 MB at L = 101); LASAGNA_TEST_A1_CHUNK (tests only) overrides
-    static const uint64_t want = [] {
-        const char *e = getenv("LASAGNA_TEST_A1_CHUNK");
-        const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
-        return v ? v : (uint64_t)512 * 1024;
-    }();
+    const uint64_t want = env_u64("LASAGNA_TEST_A1_CHUNK", 0) ? env_u64("LASAGNA_TEST_A1_CHUNK", 0)
+                                                               : (uint64_t)512 * 1024;
     const uint64_t chunk = std::max<uint64_t>(512, want / 512 * 512);
     const size_t slot_bytes = (size_t)chunk * L;
     const uint64_t nchunk = ceil_div(n, chunk);
     // as many ring slots as the region buffer holds, up to one per chunk (then the copy engine
     // never waits for a table pass, e.g. while another call's kernels hold the SMs), at most 64
-    static const uint64_t max_slots = [] { // LASAGNA_TEST_A1_SLOTS (tests only) lowers it
-        const char *e = getenv("LASAGNA_TEST_A1_SLOTS");
-        const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
-        return v >= 3 && v < 64 ? v : (uint64_t)64;
-    }();
+    // LASAGNA_TEST_A1_SLOTS (tests only) lowers it
+    const uint64_t ts = env_u64("LASAGNA_TEST_A1_SLOTS", 0);
+    const uint64_t max_slots = ts >= 3 && ts < 64 ? ts : 64;
     const uint64_t nslot = std::min<uint64_t>({nchunk, max_slots, r.lay.tabB_bytes / slot_bytes});
     if (nslot < std::min<uint64_t>(nchunk, 3)) return launch_scatter_table(base, r.s); // zero-copy
     unsigned char *ring = reinterpret_cast<unsigned char *>(r.tab[1]);
@@ -338,7 +359,19 @@ static lasagna_status scatter_from_host(Run &r, const ScatterArgs &base, const c
     return LASAGNA_OK;
 }
 
-// Build + sort the key tables of lengths [l_lo, l_hi]; returns which tab buffer is sorted.
+// Stored fingerprint bits of a bucketed key: bits [vbits + 2, 64) (the top 8 bits of the mixed
+// fingerprint are implied by the level-1 region).  LASAGNA_TEST_FP_BITS=b (tests only) keeps
+// just the top b of them, to measure the collision rate at a chosen key width (R12).
+static uint64_t stored_keep(const Geometry &g)
+{
+    uint64_t keep = ~((1ull << (g.vbits + FLAG_BITS)) - 1);
+    const uint64_t b = env_u64("LASAGNA_TEST_FP_BITS", 64);
+    if (b < 64 - g.vbits - FLAG_BITS) keep &= b ? ~0ull << (64 - b) : 0ull;
+    return keep;
+}
+
+// Build + partition the key tables of lengths [l_lo, l_hi] (level 1 fused with a2, then the
+// refine levels; the final buckets end in tabB for P = 2, tabA for P = 1 and P = 3).
 static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint32_t l_lo,
                                            uint32_t l_hi, PhaseTimer &tm, lasagna_stats *st)
 {
@@ -355,10 +388,11 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.l_lo = l_lo;
     sa.l_hi = l_hi;
     sa.vbits = g.vbits;
+    sa.keep = stored_keep(g);
     sa.out = r.tab[0];
     sa.fill = r.fill1;
     sa.split = g.P == 1; // one level: the level-1 regions are the (split) buckets
-    sa.cap = sa.split ? g.half1 : g.cap1;
+    sa.cap = sa.split ? g.half : g.cap1;
     sa.overflow = ovf;
     sa.ascii = r.ascii; // fused a1 (first group only)
     sa.packed_out = r.packed_out;
@@ -375,21 +409,36 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     }
     if ((rc = tm.stop()) != LASAGNA_OK) return rc;
     if (g.P >= 2) {
+        // level 2: the next 8 bits (the stored key's top byte)
         RefineArgs ra;
         ra.in = r.tab[0];
         ra.fill_in = r.fill1;
         ra.cap_in = g.cap1;
-        ra.dshift = 48;
+        ra.dshift = 56;
+        ra.dbits = 8;
         ra.out = r.tab[1];
         ra.fill_out = r.fill2;
-        ra.cap_out = g.half2;
+        ra.cap_out = g.P == 2 ? g.half : g.cap2;
         ra.vbits = g.vbits;
-        ra.split = true;
+        ra.split = g.P == 2;
         ra.overflow = ovf;
         if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
         if ((rc = launch_refine(ra, (uint64_t)G * 256, r.s)) != LASAGNA_OK) return rc;
+        if (g.P == 3) {
+            // level 3: dlast more bits, split into build and probe halves
+            ra.in = r.tab[1];
+            ra.fill_in = r.fill2;
+            ra.cap_in = g.cap2;
+            ra.dshift = 56 - g.dlast;
+            ra.dbits = g.dlast;
+            ra.out = r.tab[0];
+            ra.fill_out = r.fill3;
+            ra.cap_out = g.half;
+            ra.split = true;
+            if ((rc = launch_refine(ra, (uint64_t)G * 65536, r.s)) != LASAGNA_OK) return rc;
+        }
         if ((rc = tm.stop()) != LASAGNA_OK) return rc;
-        if (st) st->sort_launches += 1;
+        if (st) st->sort_launches += g.P - 1;
     }
     return LASAGNA_OK;
 }
@@ -435,14 +484,7 @@ static lasagna_status build_group(Run &r, const uint64_t *packed, uint32_t l_lo,
 // LASAGNA_JOIN_FILTER=1: the join drops pairs with an end claimed by a longer length (counted,
 // not stored).  Off by default: measured at cfg3 the claimed-bit reads cost the join more
 // (+2.5 ms) than the smaller pool saves the greedy (-1.2 ms); the greedy drops them instead.
-static bool join_filter()
-{
-    static const bool on = [] {
-        const char *e = getenv("LASAGNA_JOIN_FILTER");
-        return e && e[0] == '1';
-    }();
-    return on;
-}
+static bool join_filter() { return env_flag("LASAGNA_JOIN_FILTER", '1'); }
 
 // Join (search + verify) of length l into the pool; if m_out, synchronise and report the
 // pair count.
@@ -472,17 +514,11 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         BucketJoinArgs bj;
         bj.j = ja;
         bj.overflow = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
-        if (g.P >= 2) {
-            bj.buckets = r.tab[1] + (uint64_t)s * 131072 * g.half2;
-            bj.fills = r.fill2 + (uint64_t)s * 131072;
-            bj.half_cap = g.half2;
-            bj.n_buckets = 65536;
-        } else {
-            bj.buckets = r.tab[0] + (uint64_t)s * 512 * g.half1;
-            bj.fills = r.fill1 + (uint64_t)s * 512;
-            bj.half_cap = g.half1;
-            bj.n_buckets = 256;
-        }
+        // final level: [G][n_buckets][2][half] (tabB for P = 2, tabA for P = 1 and 3)
+        bj.buckets = (g.P == 2 ? r.tab[1] : r.tab[0]) + (uint64_t)s * 2 * g.n_buckets * g.half;
+        bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * g.n_buckets;
+        bj.half_cap = g.half;
+        bj.n_buckets = g.n_buckets;
         rc = launch_bucket_join(bj, r.s);
     } else {
         rc = launch_join(ja, r.s);
@@ -677,10 +713,10 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     uint32_t *claimed = r.at<uint32_t>(r.lay.claimed);
     r.claimed = claimed;
     if (ascii_dev) {
-        // a1: fused into the first partition pass when the fast path runs (T = 16, L <= 160),
+        // a1: fused into the first partition pass when the fast path runs (T >= 16, L <= 160),
         // otherwise a separate pack launch
         LSG_CUDA(cudaMemsetAsync(first_bad, 0xFF, 8, s));
-        if (use_bucketed(g) && g.P == 2 && L <= 160) {
+        if (use_bucketed(g) && g.P >= 2 && L <= 160) {
             r.ascii = reinterpret_cast<const unsigned char *>(ascii_dev);
             r.ascii_host = ascii_host;
             r.packed_out = packed_out;
@@ -697,6 +733,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     gb.cnt2 = r.ctr64 + CTR_POOL2;
     gb.cnt3 = r.ctr64 + CTR_POOL3;
     gb.book = r.ctr64 + CTR_BOOK;
+    gb.work = r.ctr64 + CTR_WORK;
     gb.best = r.at<unsigned long long>(r.lay.best);
     gb.claimed = claimed;
     gb.cap = cap;
@@ -769,6 +806,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         st.n_greedy = book[0];
         st.rounds_max = (uint32_t)book[3];
         st.fp_false_matches = h[CTR_FALSE];
+        st.greedy_pair_rounds = h[CTR_WORK];
+        st.partition_levels = r.bucketed ? g.P : 0;
         if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
         st.kernel_launches = launch_count() - launches0;
         *stats = st;
@@ -1010,6 +1049,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     gb.cnt2 = ctr64 + CTR_POOL2;
     gb.cnt3 = ctr64 + CTR_POOL3;
     gb.book = ctr64 + CTR_BOOK;
+    gb.work = ctr64 + CTR_WORK;
     gb.best = reinterpret_cast<unsigned long long *>(ws + o_best);
     gb.claimed = claimed;
     gb.cap = c1;

@@ -13,8 +13,11 @@
 //                         regions of that length with one atomic per (CTA, digit); no
 //                         histogram pass, no look-back (order inside a region is irrelevant)
 //   refine_kernel         level k -> k+1: one CTA owns one region and streams it in tiles,
-//                         splitting it by the next 8 bits into 256 sub-regions it alone
-//                         writes (CTA-local running offsets: no atomics, no look-back)
+//                         splitting it by the next dbits (<= 8) bits into 2^dbits sub-regions
+//                         it alone writes (CTA-local running offsets: no atomics, no
+//                         look-back).  T = 16 (cfg3): one refine; T = 16 + d (cfg4/cfg5, 2n
+//                         ~ 2.5e9): two, the second by d = 4 bits, so a final bucket holds
+//                         ~2.4 K entries like cfg3's ~1.1 K (one shared-memory join window)
 //   bucket_join_kernel    a5 over the final regions (= buckets, fills known): windows of
 //                         whole buckets go through the shared-memory hash join (joinwin.cuh)
 //
@@ -53,23 +56,14 @@ __device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t *wsum)
     return x - v + add;
 }
 
-// partition bin of a key: its digit, or (SPLIT, the final level) digit * 2 + list tag so that
-// each bucket stores its prefix entries and its suffix entries in two halves
-template <bool SPLIT>
-__device__ __forceinline__ uint32_t bin_of(uint64_t key, uint32_t dshift, uint32_t vbits)
-{
-    const uint32_t d = (uint32_t)(key >> dshift) & 255u;
-    if constexpr (SPLIT) return (d << 1) | (uint32_t)((key >> vbits) & 1);
-    else return d;
-}
-
 // ------------------------------------------------------------------ level 1: fused with a2
 // One thread per read, LPR lengths per partition round: the rolling streams (a2) produce the
 // two canonical keys of the read (vertex 2i and 2i+1, common.cuh) for each length; a round
 // ranks its 2 * LPR keys per thread by bin in shared memory (atomics: order inside a region is
 // irrelevant), reserves space in the regions of its lengths with one global atomic per
 // (CTA, bin), stages the keys by bin and writes them out in bin runs.  Bins are
-// q * NBL + bin_of(key) for the round's q-th length.
+// q * NBL + d1 (split: q * NBL + 2 d1 + flag bit) for the round's q-th length, d1 = the top 8
+// bits of the mixed canonical fingerprint, which the stored key no longer carries.
 template <int W, bool ASCII, bool SPLIT, int LPR>
 __global__ void __launch_bounds__(SC_THREADS, 2)
 scatter_table_kernel(ScatterArgs a)
@@ -79,8 +73,10 @@ scatter_table_kernel(ScatterArgs a)
     constexpr int BPT = NBIN / SC_THREADS; // bins per thread in the round's scan
     constexpr int KPT = 2 * LPR;           // keys per thread per round
     static_assert(NBIN % SC_THREADS == 0 && BPT >= 1 && BPT <= 4, "bins per thread");
-    // dynamic: stage[SC_THREADS * KPT] keys, then (ASCII) the CTA's staged read bytes
+    // dynamic: stage[SC_THREADS * KPT] keys, sbin[SC_THREADS * KPT] their bins, then (ASCII)
+    // the CTA's staged read bytes
     extern __shared__ __align__(16) uint64_t stage[];
+    unsigned short *sbin = reinterpret_cast<unsigned short *>(stage + SC_THREADS * KPT);
     __shared__ uint32_t cnt[NBIN], lstart[NBIN + 1], wsum[16];
     __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
 
@@ -90,7 +86,7 @@ scatter_table_kernel(ScatterArgs a)
     if constexpr (ASCII) {
         // a1 fused: stage this CTA's ASCII span (zero-copy from host memory over PCIe when
         // the caller passed page-locked host memory), pack, validate, keep the packed rows
-        unsigned char *sascii = reinterpret_cast<unsigned char *>(stage + SC_THREADS * KPT);
+        unsigned char *sascii = reinterpret_cast<unsigned char *>(sbin + SC_THREADS * KPT);
         const uint64_t r0 = (uint64_t)blockIdx.x * SC_THREADS;
         const uint64_t r1 = min64(a.n, r0 + SC_THREADS);
         const uint32_t off = stage_ascii(a.ascii, r0 * a.L, r1 * a.L, sascii, SC_THREADS);
@@ -116,14 +112,13 @@ scatter_table_kernel(ScatterArgs a)
     }
     for (uint32_t t = threadIdx.x; t < NBIN; t += SC_THREADS) cnt[t] = 0;
     __syncthreads();
-    const uint64_t keep = key_keep(a.vbits);
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
     const uint32_t nh = min(skip_halves(a.l_lo), 2u * W); // leading bases absorbed in chunks
     fp_skip<W>(x, y, nh, st);
     const uint32_t kskip = 16u * nh;
     uint64_t kk[KPT];
-    uint32_t rk[KPT];
+    uint32_t rk[KPT]; // bin << 16 | rank within the bin
     uint32_t kc = 0, lfirst = 0; // lengths buffered this round (block-uniform)
 #pragma unroll
     for (int w = 0; w < W; ++w) {
@@ -141,15 +136,21 @@ scatter_table_kernel(ScatterArgs a)
             if (l < a.l_lo) continue; // uniform across the block
             if (kc == 0) lfirst = l;
             if (valid) {
-                const uint64_t e0 = canon_key(st.P0, st.S1, keep, a.vbits, v0);
-                const uint64_t e1 = canon_key(st.P1, st.S0, keep, a.vbits, v0 + 1);
+                uint32_t d0, d1; // level-1 digits (implied by the region, not stored)
+                const uint64_t e0 = canon_key_d1(st.P0, st.S1, a.keep, a.vbits, v0, &d0);
+                const uint64_t e1 = canon_key_d1(st.P1, st.S0, a.keep, a.vbits, v0 + 1, &d1);
+                if constexpr (SPLIT) {
+                    d0 = (d0 << 1) | (uint32_t)((e0 >> a.vbits) & 1);
+                    d1 = (d1 << 1) | (uint32_t)((e1 >> a.vbits) & 1);
+                }
 #pragma unroll
                 for (int q = 0; q < LPR; ++q)
                     if ((uint32_t)q == kc) { // constant register indices after unrolling
                         kk[2 * q] = e0;
                         kk[2 * q + 1] = e1;
-                        rk[2 * q] = atomicAdd(&cnt[q * NBL + bin_of<SPLIT>(e0, 56, a.vbits)], 1u);
-                        rk[2 * q + 1] = atomicAdd(&cnt[q * NBL + bin_of<SPLIT>(e1, 56, a.vbits)], 1u);
+                        const uint32_t b0 = q * NBL + d0, b1 = q * NBL + d1;
+                        rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
+                        rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
                     }
             }
             ++kc;
@@ -187,25 +188,19 @@ scatter_table_kernel(ScatterArgs a)
             __syncthreads();
             if (valid) {
 #pragma unroll
-                for (int q = 0; q < LPR; ++q)
-                    if ((uint32_t)q < kc) {
-                        stage[lstart[q * NBL + bin_of<SPLIT>(kk[2 * q], 56, a.vbits)] + rk[2 * q]] = kk[2 * q];
-                        stage[lstart[q * NBL + bin_of<SPLIT>(kk[2 * q + 1], 56, a.vbits)] + rk[2 * q + 1]] =
-                            kk[2 * q + 1];
+                for (int q = 0; q < 2 * LPR; ++q)
+                    if ((uint32_t)q < 2 * kc) {
+                        const uint32_t b = rk[q] >> 16;
+                        const uint32_t u = lstart[b] + (rk[q] & 0xFFFFu);
+                        stage[u] = kk[q];
+                        sbin[u] = (unsigned short)b;
                     }
             }
             __syncthreads();
             const uint32_t total = lstart[NBIN];
-            uint32_t bnd[LPR]; // first stage slot of each length's bins
-#pragma unroll
-            for (int q = 0; q < LPR; ++q) bnd[q] = lstart[q * NBL];
             for (uint32_t u = threadIdx.x; u < total; u += SC_THREADS) {
-                const uint64_t key = stage[u];
-                uint32_t q = 0;
-#pragma unroll
-                for (int k = 1; k < LPR; ++k) q += u >= bnd[k];
-                const long long go = gofs[q * NBL + bin_of<SPLIT>(key, 56, a.vbits)];
-                if (go >= 0) a.out[go + u] = key;
+                const long long go = gofs[sbin[u]];
+                if (go >= 0) a.out[go + u] = stage[u];
             }
             kc = 0;
             // the next round's first barrier orders these reads before stage/lstart reuse
@@ -221,7 +216,7 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
         const unsigned blocks = (unsigned)ceil_div(args.n, SC_THREADS);
         const size_t ascii_b = args.ascii ? (size_t)SC_THREADS * args.L + 32 : 0; // + SWAR overread
         auto run = [&](auto kern, int lpr) -> lasagna_status {
-            const size_t smem = (size_t)SC_THREADS * 2 * lpr * 8 + ascii_b;
+            const size_t smem = (size_t)SC_THREADS * 2 * lpr * (8 + 2) + ascii_b;
             LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           (int)smem));
             kern<<<blocks, SC_THREADS, smem, s>>>(args);
@@ -245,19 +240,26 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
 refine_kernel(RefineArgs a)
 {
     constexpr int RF_TILE = RF_THREADS * RF_KPT;
-    constexpr int NB = SPLIT ? 512 : 256;
+    constexpr int NBMAX = 512; // 2^dbits bins (x 2 when split), dbits <= 8
     extern __shared__ __align__(128) uint64_t rsm[];
     uint64_t *inb = rsm;                 // [2][RF_TILE]
     uint64_t *rstage = rsm + 2 * RF_TILE; // [RF_TILE]
     __shared__ __align__(8) unsigned long long mbar[2];
-    __shared__ uint32_t cnt[NB], lstart[NB], running[NB], wsum[16];
-    __shared__ long long gofs[NB];
+    __shared__ uint32_t cnt[NBMAX], lstart[NBMAX], running[NBMAX], wsum[16];
+    __shared__ long long gofs[NBMAX];
+    const uint32_t nb = (1u << a.dbits) << (SPLIT ? 1 : 0);
+    const uint32_t dmask = (1u << a.dbits) - 1u;
+    auto binof = [&](uint64_t k) -> uint32_t {
+        const uint32_t d = (uint32_t)(k >> a.dshift) & dmask;
+        if constexpr (SPLIT) return (d << 1) | (uint32_t)((k >> a.vbits) & 1);
+        else return d;
+    };
     const uint64_t r = blockIdx.x;
     const uint32_t fill = a.fill_in[r];
     const uint64_t count = min64(fill, a.cap_in);
     const uint64_t *src = a.in + r * a.cap_in;
     const uint32_t ntiles = (uint32_t)ceil_div(count, RF_TILE);
-    if (threadIdx.x < NB) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
+    if (threadIdx.x < NBMAX) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
         mbar_init(&mbar[0], 1);
         mbar_init(&mbar[1], 1);
@@ -286,16 +288,16 @@ refine_kernel(RefineArgs a)
 #pragma unroll
         for (int q = 0; q < RF_KPT; ++q) {
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
-            if (idx < m) rk[q] = atomicAdd(&cnt[bin_of<SPLIT>(tin[idx], a.dshift, a.vbits)], 1u);
+            if (idx < m) rk[q] = atomicAdd(&cnt[binof(tin[idx])], 1u);
         }
         __syncthreads();
         uint32_t c = 0;
-        if (threadIdx.x < NB) {
+        if (threadIdx.x < nb) {
             c = cnt[threadIdx.x];
             cnt[threadIdx.x] = 0;
         }
-        const uint32_t ex = block_scan<NB>(c, wsum);
-        if (threadIdx.x < NB) {
+        const uint32_t ex = block_scan<RF_THREADS>(c, wsum);
+        if (threadIdx.x < nb) {
             lstart[threadIdx.x] = ex;
             const uint32_t run = running[threadIdx.x];
             if ((uint64_t)run + c > a.cap_out) {
@@ -303,7 +305,7 @@ refine_kernel(RefineArgs a)
                 *a.overflow = 1u;
             } else {
                 gofs[threadIdx.x] =
-                    (long long)((r * NB + threadIdx.x) * a.cap_out + run) - (long long)ex;
+                    (long long)((r * nb + threadIdx.x) * a.cap_out + run) - (long long)ex;
             }
         }
         __syncthreads();
@@ -312,22 +314,22 @@ refine_kernel(RefineArgs a)
             const uint32_t idx = q * RF_THREADS + threadIdx.x;
             if (idx < m) {
                 const uint64_t k = tin[idx];
-                rstage[lstart[bin_of<SPLIT>(k, a.dshift, a.vbits)] + rk[q]] = k;
+                rstage[lstart[binof(k)] + rk[q]] = k;
             }
         }
         __syncthreads();
 #pragma unroll 4
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
-            const long long go = gofs[bin_of<SPLIT>(k, a.dshift, a.vbits)];
+            const long long go = gofs[binof(k)];
             if (go >= 0) a.out[go + u] = k;
         }
         __syncthreads();
-        if (threadIdx.x < NB) running[threadIdx.x] += c;
+        if (threadIdx.x < nb) running[threadIdx.x] += c;
         __syncthreads();
     }
-    if (threadIdx.x < NB) {
-        a.fill_out[r * NB + threadIdx.x] = running[threadIdx.x];
+    if (threadIdx.x < nb) {
+        a.fill_out[r * nb + threadIdx.x] = running[threadIdx.x];
         if (running[threadIdx.x] > a.cap_out) *a.overflow = 1u;
     }
     if (threadIdx.x == 0 && fill > a.cap_in) *a.overflow = 1u;
@@ -336,6 +338,7 @@ refine_kernel(RefineArgs a)
 lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStream_t s)
 {
     if (n_regions == 0) return LASAGNA_OK;
+    if (args.dbits < 1 || args.dbits > 8) return LASAGNA_EINVAL;
     // tile of 16 keys per thread (one 512-thread CTA per SM, measured faster than 8 keys at
     // two CTAs per SM: 22 vs 30 ms at cfg3); LASAGNA_RF_KPT=8 selects the smaller tile
     static const int kpt = [] {

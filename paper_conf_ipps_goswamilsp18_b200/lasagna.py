@@ -34,7 +34,9 @@ class _Stats(ctypes.Structure):
                 ("bucketed", ctypes.c_uint32),
                 ("ms_table", ctypes.c_float), ("ms_sort", ctypes.c_float),
                 ("ms_search", ctypes.c_float),
-                ("ms_greedy", ctypes.c_float)]
+                ("ms_greedy", ctypes.c_float),
+                ("greedy_pair_rounds", ctypes.c_uint64), ("partition_levels", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -201,13 +203,19 @@ class GreedyGraph:
 
     def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0,
                  budget_bytes: int | None = None):
+        """budget_bytes: device memory for the WORKSPACE (lengths_per_pass = 0 lets the a8
+        planner pick the largest length group that fits it).  Default: 92 % of the free
+        memory less what the runner allocates besides the workspace (the outputs and the
+        packed rows from_ascii writes)."""
         self.n, self.L, self.l_min = n, L, l_min
         self.device = torch.device(device)
+        if self.device.type == "cuda" and self.device.index is None:
+            self.device = torch.device("cuda", torch.cuda.current_device())
         if lengths_per_pass == 0:
             if budget_bytes is None:
                 free, _ = torch.cuda.mem_get_info(self.device)
-                budget_bytes = int(free * 0.9)
-            lp, need = plan(n, L, l_min, budget_bytes)
+                budget_bytes = int(free * 0.92) - self.side_bytes(n, L)
+            lp, need = plan(n, L, l_min, max(0, budget_bytes))
             if lp == 0:
                 raise LasagnaError(ENOSPC, f"needs {need} bytes of workspace, budget {budget_bytes}")
             lengths_per_pass = lp
@@ -220,8 +228,30 @@ class GreedyGraph:
         self.succ = torch.empty(2 * n, dtype=torch.int32, device=self.device)
         self.olen = torch.empty(2 * n, dtype=torch.uint8, device=self.device)
 
+    @staticmethod
+    def side_bytes(n: int, L: int) -> int:
+        """Device bytes a runner holds besides its workspace: succ u32[2n], olen u8[2n], the
+        packed rows u64[n][W] and first_bad (from_ascii)."""
+        return 2 * n * 5 + n * 8 * words_per_read(L) + 4096
+
+    def _check_input(self, t: torch.Tensor, kind: str) -> None:
+        if kind == "packed":
+            shape, dtype = (self.n, words_per_read(self.L)), torch.int64
+        else:
+            shape, dtype = (self.n, self.L), torch.uint8
+        if t.dtype != dtype or tuple(t.shape) != shape:
+            raise ValueError(f"{kind} input must be a {dtype} tensor of shape {shape}, "
+                             f"got {t.dtype} {tuple(t.shape)}")
+        if not t.is_contiguous():
+            raise ValueError(f"{kind} input must be contiguous")
+        if t.is_cuda and t.device != self.device:
+            raise ValueError(f"{kind} input on {t.device}, runner on {self.device}")
+
     def __call__(self, packed: torch.Tensor, stats: bool = True) -> GraphResult:
         """a1-a7 on already packed reads (lasagna_greedy_graph)."""
+        self._check_input(packed, "packed")
+        if not packed.is_cuda:
+            raise ValueError("packed rows must be device memory")
         return self._run(lambda ws, st: lib().lasagna_greedy_graph(
             _ptr(packed), self.n, self.L, self.l_min, self.lengths_per_pass, _ptr(self.ws),
             ctypes.byref(ws), _ptr(self.succ), _ptr(self.olen), st, _stream(self.device)), stats)
@@ -229,9 +259,10 @@ class GreedyGraph:
     def from_ascii(self, ascii: torch.Tensor, stats: bool = True) -> GraphResult:
         """a1-a7 from (n, L) uint8 ASCII reads on the device or in page-locked host memory
         (lasagna_greedy_graph_ascii: staging fused into the first table pass)."""
+        ascii = ascii.contiguous()
         if not ascii.is_cuda and not ascii.is_pinned():
             raise ValueError("ascii must be a CUDA tensor or page-locked host memory")
-        ascii = ascii.contiguous()
+        self._check_input(ascii, "ascii")
         if getattr(self, "packed", None) is None:
             self.packed = torch.empty((self.n, words_per_read(self.L)), dtype=torch.int64,
                                       device=self.device)
@@ -272,8 +303,13 @@ class GraphPipeline:
         if dev.index is None:  # the worker threads select the device by index
             dev = torch.device(dev.type, torch.cuda.current_device())
         self.n, self.L, self.device = n, L, dev
-        self.runners = [GreedyGraph(n, L, l_min, self.device, lengths_per_pass) for _ in range(2)]
         self.bufs = [torch.empty((n, L), dtype=torch.uint8, device=self.device) for _ in range(2)]
+        # the two runners share what is free after the input buffers: half each, less what a
+        # runner holds besides its workspace
+        free, _ = torch.cuda.mem_get_info(self.device)
+        budget = int(free * 0.92) // 2 - GreedyGraph.side_bytes(n, L)
+        self.runners = [GreedyGraph(n, L, l_min, self.device, lengths_per_pass,
+                                    budget_bytes=budget) for _ in range(2)]
         self.copy = torch.cuda.Stream(self.device)
         self.lanes = [torch.cuda.Stream(self.device) for _ in range(2)]
 

@@ -66,6 +66,9 @@ def lib():
                                     ctypes.c_double, ctypes.c_uint64, ctypes.c_uint64,
                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
         L.readgen_reads.restype = ctypes.c_int
+        L.readgen_starts.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint32,
+                                     ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p]
+        L.readgen_starts.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -105,3 +108,22 @@ def config_reads(cfg: ReadConfig | str, n: int | None = None, seed: int | None =
         cfg = CONFIGS[cfg]
     return reads(cfg.seed if seed is None else seed, cfg.G, cfg.n if n is None else n,
                  cfg.L, cfg.p_err)
+
+
+def starts(seed: int, G: int, L: int, i0: int, i1: int) -> np.ndarray:
+    """Start positions of reads [i0, i1) (uint64), without generating their bases."""
+    out = np.empty(i1 - i0, dtype=np.uint64)
+    if lib().readgen_starts(seed, G, L, i0, i1, out.ctypes.data) != 0:
+        raise ValueError("readgen: invalid parameters")
+    return out
+
+
+def window_sample(cfg: ReadConfig | str, n_target: int) -> np.ndarray:
+    """Indices of the reads of a config that start in the genome window [0, f (G - L + 1)),
+    f = n_target / n: a sample of the SAME read set at the same coverage and error rate
+    (a prefix of the read list would have ~f times the coverage instead)."""
+    if isinstance(cfg, str):
+        cfg = CONFIGS[cfg]
+    st = starts(cfg.seed, cfg.G, cfg.L, 0, cfg.n)
+    lim = int(min(1.0, n_target / cfg.n) * (cfg.G - cfg.L + 1))
+    return np.nonzero(st < lim)[0]

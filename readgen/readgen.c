@@ -90,3 +90,18 @@ int readgen_reads(uint64_t seed, uint64_t G, uint32_t L, double p_err,
     }
     return 0;
 }
+
+/* Start positions only of reads [i0, i1) (the same draws readgen_reads makes; no bases):
+ * lets a caller pick the reads of a genome window — a coverage-preserving sample. */
+int readgen_starts(uint64_t seed, uint64_t G, uint32_t L, uint64_t i0, uint64_t i1,
+                   uint64_t *starts)
+{
+    if (L == 0 || (uint64_t)L > G) return -1;
+    const uint64_t ks = stream_key(seed, S_START);
+    const uint64_t span = G - L + 1;
+#pragma omp parallel for schedule(static)
+    for (int64_t ii = (int64_t)i0; ii < (int64_t)i1; ++ii)
+        starts[(uint64_t)ii - i0] =
+            (uint64_t)(((unsigned __int128)splitmix64(ks + (uint64_t)ii) * span) >> 64);
+    return 0;
+}

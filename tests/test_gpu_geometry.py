@@ -1,0 +1,207 @@
+"""GPU parity of the a8 semi-streaming paths and of every table geometry, against the oracle.
+
+The configs of BASELINE.json take three geometries of the bucketed (radix-partition) path:
+one level (T = 8, cfg1-sized), two levels (T = 16: cfg2, cfg3) and three levels (T = 20:
+cfg4, cfg5 with 2n ~ 2.5e9).  cfg4/cfg5 are too large for the oracle, so their geometry is
+forced here at cfg1/cfg2 sizes through test hooks (LASAGNA_TEST_LEVELS, LASAGNA_TEST_LAST_BITS;
+read by the library on every call).  Each test crosses a geometry with the semi-streaming
+driver's length groups (lengths_per_pass, a8: P:L61-67), the input form (packed
+rows, device ASCII, page-locked host ASCII streamed by DMA) and the exact LSD fallback path;
+every result must equal the oracle bit for bit (succ, olen, |P|, accepted pairs).
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import readgen
+
+gpu = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lz():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    import paper_conf_ipps_goswamilsp18_b200 as m
+    m.lib()
+    return m
+
+
+@pytest.fixture(scope="module")
+def cfg2():
+    """cfg2 (BASELINE configs[1]: 2.3 M reads of 100 bp, 1 % errors) and its oracle graph."""
+    cfg = readgen.CONFIGS["cfg2"]
+    reads = readgen.config_reads(cfg)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, cfg.l_min)
+    return cfg, reads, esucc, eolen, m, acc
+
+
+@pytest.fixture(scope="module")
+def cfg1():
+    cfg = readgen.CONFIGS["cfg1"]
+    reads = readgen.config_reads(cfg)
+    epl, epa, epb = oracle.overlaps(reads, cfg.l_min)
+    esucc, eolen, _ = oracle.greedy(cfg.n, epl, epa, epb)
+    return cfg, reads, (epl, epa, epb), esucc, eolen
+
+
+def _u32(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def _u8(t):
+    return t.cpu().numpy().view(np.uint8)
+
+
+def _same(r, esucc, eolen, m, acc):
+    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc, (r.stats, m, acc)
+    assert np.array_equal(_u32(r.succ), esucc)
+    assert np.array_equal(_u8(r.olen), eolen)
+
+
+@gpu
+@pytest.mark.parametrize("lpp", [1, 5])
+def test_two_level_multipass_from_packed(lz, cfg2, lpp):
+    """T = 16 (level-1 scatter + level-2 refine), lengths_per_pass 1 and 5: 37 and 8 device
+    passes over the resident packed reads."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=lpp)
+    assert r.stats["key_sort_bits"] == 16 and r.stats["bucketed"] == 1
+    assert r.stats["passes"] == -(-(cfg.L - cfg.l_min) // lpp)
+    _same(r, esucc, eolen, m, acc)
+
+
+@gpu
+@pytest.mark.parametrize("where", ["device", "pinned"])
+def test_two_level_multipass_from_ascii(lz, cfg2, where):
+    """a1 fused into the FIRST group's scatter (device ASCII, or page-locked host ASCII streamed
+    in by DMA chunks), later groups reading the packed rows that first pass wrote."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    t = torch.from_numpy(reads)
+    t = t.cuda() if where == "device" else t.pin_memory()
+    g = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda", lengths_per_pass=5)
+    r = g.from_ascii(t)
+    assert r.stats["passes"] == 8
+    _same(r, esucc, eolen, m, acc)
+    assert np.array_equal(g.packed.cpu().numpy().view(np.uint64),
+                          oracle.pack(reads, lz.words_per_read(cfg.L)))
+
+
+@gpu
+def test_exact_path_multipass(lz, cfg2, monkeypatch):
+    """The exact LSD path (table + onesweep passes + contiguous join) with several length
+    groups, from packed rows and from ASCII (a separate pack launch on that path)."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    monkeypatch.setenv("LASAGNA_PATH", "exact")
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=5)
+    assert r.stats["bucketed"] == 0 and r.stats["passes"] == 8
+    _same(r, esucc, eolen, m, acc)
+    g = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda", lengths_per_pass=7)
+    r = g.from_ascii(torch.from_numpy(reads).pin_memory())
+    assert r.stats["bucketed"] == 0
+    _same(r, esucc, eolen, m, acc)
+
+
+@gpu
+@pytest.mark.parametrize("lpp,src", [(0, "packed"), (5, "packed"), (5, "pinned"), (3, "device")])
+def test_three_level_geometry(lz, cfg2, monkeypatch, lpp, src):
+    """The cfg4/cfg5 geometry (three partition levels of 8, 8 and 4 bits: T = 20, 2^20 split
+    buckets per length) forced at cfg2 size: one pass and several, from packed rows, from
+    page-locked host ASCII (the DMA ring in the level-2 buffer) and from device ASCII."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    monkeypatch.setenv("LASAGNA_TEST_LEVELS", "3")
+    monkeypatch.setenv("LASAGNA_TEST_LAST_BITS", "4")
+    if src == "packed":
+        packed = lz.load_reads(torch.from_numpy(reads).cuda())
+        r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=lpp)
+    else:
+        t = torch.from_numpy(reads)
+        t = t.cuda() if src == "device" else t.pin_memory()
+        g = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda", lengths_per_pass=lpp)
+        r = g.from_ascii(t)
+    assert r.stats["key_sort_bits"] == 20 and r.stats["bucketed"] == 1, r.stats
+    assert r.stats["sort_launches"] == 2 * r.stats["passes"]
+    _same(r, esucc, eolen, m, acc)
+
+
+@gpu
+@pytest.mark.parametrize("levels,last", [("1", "8"), ("2", "8"), ("3", "4"), ("3", "1")])
+def test_forced_geometries_overlaps_cfg1(lz, cfg1, monkeypatch, levels, last):
+    """lasagna_overlaps and the greedy graph under every partition depth at cfg1 (T = 8, 16,
+    20 and 17): the full read-end pair list, element by element."""
+    import torch
+    cfg, reads, (epl, epa, epb), esucc, eolen = cfg1
+    monkeypatch.setenv("LASAGNA_TEST_LEVELS", levels)
+    monkeypatch.setenv("LASAGNA_TEST_LAST_BITS", last)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    pl, pa, pb = lz.overlaps(packed, cfg.n, cfg.L, cfg.l_min)
+    assert np.array_equal(_u32(pa), epa) and np.array_equal(_u32(pb), epb)
+    assert np.array_equal(_u8(pl), epl)
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=4)
+    T = {"1": 8, "2": 16, "3": 16 + int(last)}[levels]
+    assert r.stats["key_sort_bits"] == T and r.stats["bucketed"] == 1
+    assert np.array_equal(_u32(r.succ), esucc) and np.array_equal(_u8(r.olen), eolen)
+
+
+@gpu
+def test_pool_growth_retry_with_length_groups(lz, monkeypatch):
+    """A length with more verified pairs than the default pair pool (every length from 1, all
+    reads of a 20 kbp genome) under lengths_per_pass = 5: ENOSPC, the binding regrows the
+    workspace and retries; the graph equals the oracle."""
+    import torch
+    reads = readgen.reads(7, 20_000, 3000, 64, 0.01)
+    esucc, eolen, m, acc = oracle.greedy_graph(reads, 1)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, 3000, 64, 1, lengths_per_pass=5)
+    _same(r, esucc, eolen, m, acc)
+
+
+def _expected_false_matches(n: int, n_len: int, bits: float) -> float:
+    """R12 closed form: per length V/2 probe-side and V/2 build-side canonical entries agree
+    on `bits` bits of mix(min(H, Hr)) with probability 2^-bits."""
+    V = 2 * n
+    return n_len * (V / 2) ** 2 / 2.0 ** bits
+
+
+@gpu
+@pytest.mark.parametrize("fp_bits", [26, 30])
+def test_false_match_rate_at_chosen_key_width(lz, cfg2, monkeypatch, fp_bits):
+    """Hash-collision rate (north star: "checked on hash-collision rates").  A bucketed key
+    compares 8 implied bits (its level-1 region) plus its stored fingerprint bits; keeping only
+    the top `fp_bits` stored bits (test hook), the rejected hits at cfg2 must follow the R12
+    closed form with 8 + fp_bits bits (Poisson, 5 sigma) and the graph must stay exact."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    monkeypatch.setenv("LASAGNA_TEST_FP_BITS", str(fp_bits))
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min)
+    exp = _expected_false_matches(cfg.n, cfg.L - cfg.l_min, 8 + fp_bits)
+    assert exp > 100
+    obs = r.stats["fp_false_matches"]
+    assert abs(obs - exp) <= 5 * exp ** 0.5 + 0.02 * exp, (obs, exp)
+    _same(r, esucc, eolen, m, acc)
+
+
+def test_false_match_rate_vertex_bits_32_closed_form():
+    """at cfg4/cfg5 (vbits = 32) a key stores 62 - 32 = 30 fingerprint bits.  The
+    bucketed key stores the 30 bits BELOW the level-1 digit, which its region implies, so a
+    comparison covers 38 bits: (V/2)^2 / 2^38 ~ 5.7e6 rejected hits per length at cfg5 (~5 %
+    of the true pairs), against 1.45e9 (~15x the true pairs) if the region digit were stored."""
+    cfg = readgen.CONFIGS["cfg5"]
+    V = 2 * cfg.n
+    vbits = (V - 1).bit_length()
+    assert vbits == 32
+    per_len = _expected_false_matches(cfg.n, 1, (62 - vbits) + 8)
+    assert 3e6 < per_len < 1e7
+    true_per_len = 3.86e9 / (cfg.L - cfg.l_min)  # SURVEY 8(d) expected |P|
+    assert per_len < 0.1 * true_per_len
+    assert _expected_false_matches(cfg.n, 1, 62 - vbits) > 10 * true_per_len
