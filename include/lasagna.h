@@ -176,6 +176,30 @@ LASAGNA_API lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, 
                             uint32_t *lengths_per_pass, size_t *workspace_bytes);
 
 /* ---------------------------------------------------------------------------------------
+ * Compress (PAPER §III-D, Fig. 7): paths and contigs of the
+ * greedy string graph (succ/olen as lasagna_greedy_graph writes them; packed rows as a1).
+ *   A path starts at a seed — a vertex with in-degree 0 and out-degree 1 — and
+ *   follows succ until a vertex without an out-edge.  The overhang of a vertex is L - olen
+ *   with an out-edge, L without.  The contig of a path is the concatenation of
+ *   seq(v)[0 .. overhang(v)) over its vertices, ASCII ACGT.  Every path has a
+ *   complementary path (seed = its tail ^ 1) spelling the reverse complement; only the one
+ *   with the smaller seed id is emitted (R20).  Cycles (no seed) and edgeless reads give no
+ *   contig (R21).  Contigs are ordered by seed id.
+ *   contigs         device char[contig_capacity]: the contigs back to back
+ *   contig_offsets  device u64[count_capacity]: contig c = contigs[off[c] .. off[c+1])
+ *   contig_seed     device u32[count_capacity - 1] or NULL: the seed vertex of contig c
+ *   *n_contigs, *total_bases  host out.  A capacity below total_bases bases or n_contigs + 1
+ *                   offsets -> LASAGNA_ENOSPC (sizes reported, nothing written).
+ * workspace: device scratch (28 B per vertex); workspace == NULL -> query.  Synchronises. */
+LASAGNA_API lasagna_status lasagna_compress(const uint64_t *packed, uint64_t n, uint32_t L,
+                                            const uint32_t *succ, const uint8_t *olen,
+                                            void *workspace, size_t *workspace_bytes,
+                                            char *contigs, uint64_t contig_capacity,
+                                            uint64_t *contig_offsets, uint32_t *contig_seed,
+                                            uint64_t count_capacity, uint64_t *n_contigs,
+                                            uint64_t *total_bases, void *stream);
+
+/* ---------------------------------------------------------------------------------------
  * Phase entry points (exported for tests and the multi-GPU driver).
  *
  * a4 — stable LSD radix sort (K4 P:L144) of `count` u64 keys by bits

@@ -65,6 +65,8 @@ def lib():
         L.oracle_greedy.restype = u64
         L.oracle_greedy_graph.argtypes = [vp, u64, u32, u32, vp, vp, vp]
         L.oracle_greedy_graph.restype = u64
+        L.oracle_compress.argtypes = [vp, u64, u32, vp, vp, vp, vp, vp, vp]
+        L.oracle_compress.restype = u64
         _lib = L
     return _lib
 
@@ -176,3 +178,22 @@ def greedy_graph(reads, l_min: int):
     if m == 0xFFFFFFFFFFFFFFFF:
         raise ValueError("oracle: invalid reads or parameters")
     return succ, olen, m, int(ng.value)
+
+
+def compress(reads, succ, olen):
+    """Contigs of the greedy graph: (contigs bytes, offsets uint64[c+1],
+    seeds uint32[c]); contig k = contigs[offsets[k]:offsets[k+1]]."""
+    a = _ascii(reads)
+    n, L = a.shape
+    succ = np.ascontiguousarray(succ, dtype=np.uint32)
+    olen = np.ascontiguousarray(olen, dtype=np.uint8)
+    nc = ctypes.c_uint64(0)
+    tot = int(lib().oracle_compress(a.ctypes.data, n, L, succ.ctypes.data, olen.ctypes.data,
+                                    None, None, None, ctypes.byref(nc)))
+    c = int(nc.value)
+    buf = ctypes.create_string_buffer(max(1, tot))
+    offs = np.empty(c + 1, dtype=np.uint64)
+    seeds = np.empty(max(1, c), dtype=np.uint32)
+    lib().oracle_compress(a.ctypes.data, n, L, succ.ctypes.data, olen.ctypes.data, buf,
+                          offs.ctypes.data, seeds.ctypes.data, ctypes.byref(nc))
+    return buf.raw[:tot], offs, seeds[:c]

@@ -57,3 +57,30 @@ def greedy(n_reads: int, P: list[tuple[int, int, int]]):
         succ[b] = a ^ 1
         olen[a] = olen[b] = l
     return succ, olen
+
+
+def contigs(reads: list[str], succ: list[int], olen: list[int]) -> list[tuple[int, str]]:
+    """Compress (P:L176-192) straight from the text: seeds have in-degree 0 and out-degree 1;
+    a path follows succ to a vertex without an out-edge; each read contributes its first
+    overhang bases (L - olen, or L for the last); a path and its complementary path spell
+    reverse-complementary contigs, the one with the smaller seed is kept (R20).  Returns
+    [(seed, contig)] in seed order."""
+    seq = oriented_reads(reads)
+    L = len(seq[0])
+    V = len(seq)
+    has_in = [False] * V
+    for u in range(V):
+        if succ[u] != 0xFFFFFFFF:
+            has_in[succ[u]] = True
+    out = []
+    for s in range(V):
+        if has_in[s] or succ[s] == 0xFFFFFFFF:
+            continue
+        path = [s]
+        while succ[path[-1]] != 0xFFFFFFFF:
+            path.append(succ[path[-1]])
+        if not s < (path[-1] ^ 1):
+            continue
+        text = "".join(seq[v][: L - olen[v]] for v in path[:-1]) + seq[path[-1]]
+        out.append((s, text))
+    return out

@@ -5,10 +5,11 @@ include/lasagna.h); this package is its thin Python binding plus the multi-GPU d
 There is no CPU fallback.
 """
 from .lasagna import (  # noqa: F401
-    NONE, GraphPipeline, GraphResult, GreedyGraph, LasagnaError, fingerprints, greedy_graph, greedy_pairs,
-    kernel_launches,
-    lib, load_reads, overlaps, plan, sort_u64, words_per_read,
+    NONE, Contigs, GraphPipeline, GraphResult, GreedyGraph, LasagnaError, compress, fingerprints,
+    greedy_graph, greedy_pairs, kernel_launches, lib, load_reads, overlaps, plan, sort_u64,
+    words_per_read,
 )
 
-__all__ = ["NONE", "GraphPipeline", "GraphResult", "GreedyGraph", "LasagnaError", "fingerprints", "greedy_graph",
-           "greedy_pairs", "kernel_launches", "lib", "load_reads", "overlaps", "plan", "sort_u64", "words_per_read"]
+__all__ = ["NONE", "Contigs", "GraphPipeline", "GraphResult", "GreedyGraph", "LasagnaError",
+           "compress", "fingerprints", "greedy_graph", "greedy_pairs", "kernel_launches", "lib",
+           "load_reads", "overlaps", "plan", "sort_u64", "words_per_read"]

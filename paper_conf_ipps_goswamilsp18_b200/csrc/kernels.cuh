@@ -130,4 +130,11 @@ lasagna_status launch_gather_pairs(const uint64_t *order, uint64_t off, uint64_t
                                    cudaStream_t s);
 lasagna_status launch_lkeys(const uint8_t *pl, uint64_t count, uint64_t *keys, cudaStream_t s);
 
+// ---- Compress (compress.cu)
+lasagna_status compress_impl(const uint64_t *packed, uint64_t n, uint32_t L, const uint32_t *succ,
+                             const uint8_t *olen, void *workspace, size_t *workspace_bytes,
+                             char *contigs, uint64_t contig_capacity, uint64_t *contig_offsets,
+                             uint32_t *contig_seed, uint64_t count_capacity, uint64_t *n_contigs,
+                             uint64_t *total_bases, cudaStream_t s);
+
 } // namespace lsg

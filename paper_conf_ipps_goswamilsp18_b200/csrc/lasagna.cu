@@ -961,6 +961,37 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
     return LASAGNA_ECUDA;
 }
 
+lasagna_status lasagna_compress(const uint64_t *packed, uint64_t n, uint32_t L,
+                                const uint32_t *succ, const uint8_t *olen, void *workspace,
+                                size_t *workspace_bytes, char *contigs, uint64_t contig_capacity,
+                                uint64_t *contig_offsets, uint32_t *contig_seed,
+                                uint64_t count_capacity, uint64_t *n_contigs,
+                                uint64_t *total_bases, void *stream)
+{
+    g_err[0] = 0;
+    if (L < 2 || L > 256) {
+        set_error("L=%u out of range [2, 256]", L);
+        return LASAGNA_EINVAL;
+    }
+    if (n > 0x7FFFFFFFull) {
+        set_error("2n exceeds 0xFFFFFFFE vertex ids");
+        return LASAGNA_ERANGE;
+    }
+    if (!workspace_bytes || (workspace && (!n_contigs || !total_bases))) {
+        set_error("NULL size/count pointer");
+        return LASAGNA_EINVAL;
+    }
+    if (workspace && n && (!packed || !succ || !olen || !aligned(packed, 16) ||
+                           !aligned(succ, 4) || !aligned(workspace, 256) ||
+                           (contig_offsets && !aligned(contig_offsets, 8)))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    return compress_impl(packed, n, L, succ, olen, workspace, workspace_bytes, contigs,
+                         contig_capacity, contig_offsets, contig_seed, count_capacity, n_contigs,
+                         total_bases, (cudaStream_t)stream);
+}
+
 lasagna_status lasagna_sort_u64(uint64_t *keys, uint64_t *scratch, uint64_t count,
                                 uint32_t bit_lo, uint32_t bit_hi, void *workspace,
                                 size_t *workspace_bytes, void *stream)

@@ -79,6 +79,8 @@ def lib() -> ctypes.CDLL:
         "lasagna_plan": [u64, u32, u32, sz, pu32, psz],
         "lasagna_sort_u64": [vp, vp, u64, u32, u32, vp, psz, vp],
         "lasagna_greedy_pairs": [u64, vp, vp, vp, u64, vp, psz, vp, vp, pu32, vp],
+        "lasagna_compress": [vp, u64, u32, vp, vp, vp, psz, vp, u64, vp, vp, u64, pu64, pu64,
+                             vp],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
@@ -259,9 +261,9 @@ class GreedyGraph:
     def from_ascii(self, ascii: torch.Tensor, stats: bool = True) -> GraphResult:
         """a1-a7 from (n, L) uint8 ASCII reads on the device or in page-locked host memory
         (lasagna_greedy_graph_ascii: staging fused into the first table pass)."""
+        # device memory or page-locked host memory (torch-pinned or cudaHostRegister'ed): the
+        # library checks the pointer and rejects pageable memory with EINVAL
         ascii = ascii.contiguous()
-        if not ascii.is_cuda and not ascii.is_pinned():
-            raise ValueError("ascii must be a CUDA tensor or page-locked host memory")
         self._check_input(ascii, "ascii")
         if getattr(self, "packed", None) is None:
             self.packed = torch.empty((self.n, words_per_read(self.L)), dtype=torch.int64,
@@ -372,6 +374,39 @@ def greedy_graph(packed: torch.Tensor, n: int, L: int, l_min: int, lengths_per_p
     g = GreedyGraph(n, L, l_min, packed.device, lengths_per_pass)
     r = g(packed, stats)
     return GraphResult(r.succ.clone(), r.olen.clone(), r.stats)
+
+
+# ---------------------------------------------------------------------------- Compress
+@dataclass
+class Contigs:
+    bases: torch.Tensor    # uint8 [total]: ASCII contigs back to back
+    offsets: torch.Tensor  # int64 [c + 1]: contig k = bases[offsets[k]:offsets[k+1]]
+    seeds: torch.Tensor    # int32 [c]: seed vertex of each contig (u32 ids)
+
+
+def compress(packed: torch.Tensor, n: int, L: int, succ: torch.Tensor, olen: torch.Tensor,
+             workspace: torch.Tensor | None = None) -> Contigs:
+    """Paths and contigs of a greedy string graph (lasagna_compress; Fig. 7)."""
+    dev = packed.device
+    ws_bytes = ctypes.c_size_t(0)
+    nc, tot = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    f = lib().lasagna_compress
+    with torch.cuda.device(dev):
+        _check(f(None, n, L, None, None, None, ctypes.byref(ws_bytes), None, 0, None, None, 0,
+                 ctypes.byref(nc), ctypes.byref(tot), _stream(dev)))
+        if workspace is None or workspace.numel() < ws_bytes.value:
+            workspace = _workspace(ws_bytes.value, dev)
+        ws_bytes = ctypes.c_size_t(workspace.numel())
+        args = (_ptr(packed), n, L, _ptr(succ), _ptr(olen), _ptr(workspace), ctypes.byref(ws_bytes))
+        st = f(*args, None, 0, None, None, 0, ctypes.byref(nc), ctypes.byref(tot), _stream(dev))
+        if st != ENOSPC:
+            _check(st)
+        bases = torch.empty(max(1, tot.value), dtype=torch.uint8, device=dev)
+        offs = torch.empty(nc.value + 1, dtype=torch.int64, device=dev)
+        seeds = torch.empty(max(1, nc.value), dtype=torch.int32, device=dev)
+        _check(f(*args, _ptr(bases), tot.value, _ptr(offs), _ptr(seeds), nc.value + 1,
+                 ctypes.byref(nc), ctypes.byref(tot), _stream(dev)))
+    return Contigs(bases[:tot.value], offs, seeds[:nc.value])
 
 
 # ---------------------------------------------------------------------------- phase entry points
