@@ -153,6 +153,17 @@ __device__ __forceinline__ void rc_words(const uint64_t (&x)[W], uint32_t L, uin
     keep_low<W>(y, 2u * L);
 }
 
+// x[w] for a runtime (block-uniform) w < W without local-memory indexing: a register select
+template <int W>
+__device__ __forceinline__ uint64_t wsel(const uint64_t (&x)[W], uint32_t w)
+{
+    uint64_t r = x[0];
+#pragma unroll
+    for (int j = 1; j < W; ++j)
+        if (w == (uint32_t)j) r = x[j];
+    return r;
+}
+
 template <int W>
 __device__ __forceinline__ void load_read(const uint64_t *__restrict__ packed, uint32_t stride,
                                           uint64_t i, uint64_t (&x)[W])

@@ -66,7 +66,7 @@ __device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t *wsum)
 // bits of the mixed canonical fingerprint, which the stored key no longer carries.
 template <int W, bool ASCII, bool SPLIT, int LPR>
 __global__ void __launch_bounds__(SC_THREADS, 2)
-scatter_table_kernel(ScatterArgs a)
+scatter_table_kernel_v1(ScatterArgs a)
 {
     constexpr int NBL = SPLIT ? 512 : 256; // bins per length
     constexpr int NBIN = LPR * NBL;
@@ -208,6 +208,153 @@ scatter_table_kernel(ScatterArgs a)
     }
 }
 
+template <int W, bool ASCII, bool SPLIT, int LPR>
+__global__ void __launch_bounds__(SC_THREADS, 2)
+scatter_table_kernel(ScatterArgs a)
+{
+    constexpr int NBL = SPLIT ? 512 : 256; // bins per length
+    constexpr int NBIN = LPR * NBL;
+    constexpr int BPT = NBIN / SC_THREADS; // bins per thread in the round's scan
+    constexpr int KPT = 2 * LPR;           // keys per thread per round
+    static_assert(NBIN % SC_THREADS == 0 && BPT >= 1 && BPT <= 4, "bins per thread");
+    // dynamic: stage[SC_THREADS * KPT] keys, sbin[SC_THREADS * KPT] their bins, then (ASCII)
+    // the CTA's staged read bytes
+    extern __shared__ __align__(16) uint64_t stage[];
+    unsigned short *sbin = reinterpret_cast<unsigned short *>(stage + SC_THREADS * KPT);
+    __shared__ uint32_t cnt[NBIN], lstart[NBIN + 1], wsum[16];
+    __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
+
+    const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
+    const bool valid = i < a.n;
+    uint64_t x[W], y[W];
+    if constexpr (ASCII) {
+        // a1 fused: stage this CTA's ASCII span (zero-copy from host memory over PCIe when
+        // the caller passed page-locked host memory), pack, validate, keep the packed rows
+        unsigned char *sascii = reinterpret_cast<unsigned char *>(sbin + SC_THREADS * KPT);
+        const uint64_t r0 = (uint64_t)blockIdx.x * SC_THREADS;
+        const uint64_t r1 = min64(a.n, r0 + SC_THREADS);
+        const uint32_t off = stage_ascii(a.ascii, r0 * a.L, r1 * a.L, sascii, SC_THREADS);
+        __syncthreads();
+        if (valid) {
+            const bool ok = pack_row_regs_swar<W>(sascii + off + (uint64_t)threadIdx.x * a.L, a.L, x);
+            uint64_t *po = a.packed_out + i * a.stride;
+#pragma unroll
+            for (int j = 0; j < W; ++j) po[j] = x[j];
+            for (uint32_t j = W; j < a.stride; ++j) po[j] = 0;
+            if (!ok) atomicMin(a.first_bad, (unsigned long long)(a.read_offset + i));
+            rc_words<W>(x, a.L, y);
+        } else {
+#pragma unroll
+            for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
+        }
+    } else if (valid) {
+        load_read<W>(a.packed, a.stride, i, x);
+        rc_words<W>(x, a.L, y);
+    } else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
+    }
+    for (uint32_t t = threadIdx.x; t < NBIN; t += SC_THREADS) cnt[t] = 0;
+    __syncthreads();
+    const uint64_t v0 = 2 * (a.read_offset + i);
+    FpStreams st;
+    const uint32_t nh = min(skip_halves(a.l_lo), 2u * W); // leading bases absorbed in chunks
+    fp_skip<W>(x, y, nh, st);
+    // Base cursors over x (y is dead from here): tx holds base k of r in its low bits; ty
+    // holds base L-1-k of r in its top bits, i.e. base k of r' = RC(r) complemented.  A word
+    // boundary reloads a cursor from x with a register select (block-uniform branch).
+    uint32_t k = 16u * nh; // next base to consume (block-uniform)
+    uint64_t tx = wsel<W>(x, k >> 5) >> (2u * (k & 31u));
+    uint64_t ty;
+    {
+        const uint32_t m = a.L - 1u - k;
+        ty = wsel<W>(x, m >> 5) << (62u - 2u * (m & 31u));
+    }
+    auto step_base = [&](uint32_t kb) {
+        st.step((uint32_t)tx & 3u, (uint32_t)(ty >> 62) ^ 2u, kb);
+        tx >>= 2;
+        ty <<= 2;
+        if (((kb + 1u) & 31u) == 0u) tx = wsel<W>(x, (kb + 1u) >> 5);
+        const uint32_t m = a.L - 1u - kb;
+        if ((m & 31u) == 0u && m) ty = wsel<W>(x, (m >> 5) - 1u);
+    };
+    for (; k + 1u < a.l_lo; ++k) step_base(k); // bases before the first emitted length
+    uint64_t kk[KPT];
+    uint32_t rk[KPT]; // bin << 16 | rank within the bin
+    for (uint32_t lfirst = a.l_lo; lfirst <= a.l_hi; lfirst += LPR) {
+        const uint32_t kc = min((uint32_t)LPR, a.l_hi - lfirst + 1u); // lengths this round
+#pragma unroll
+        for (int q = 0; q < LPR; ++q) {
+            if ((uint32_t)q >= kc) break; // block-uniform
+            step_base(lfirst + q - 1u);    // the streams now hold length lfirst + q
+            if (valid) {
+                uint32_t d0, d1; // level-1 digits (implied by the region, not stored)
+                const uint64_t e0 = canon_key_d1(st.P0, st.S1, a.keep, a.vbits, v0, &d0);
+                const uint64_t e1 = canon_key_d1(st.P1, st.S0, a.keep, a.vbits, v0 + 1, &d1);
+                if constexpr (SPLIT) {
+                    d0 = (d0 << 1) | (uint32_t)((e0 >> a.vbits) & 1);
+                    d1 = (d1 << 1) | (uint32_t)((e1 >> a.vbits) & 1);
+                }
+                kk[2 * q] = e0;
+                kk[2 * q + 1] = e1;
+                const uint32_t b0 = q * NBL + d0, b1 = q * NBL + d1;
+                rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
+                rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
+            }
+        }
+        {
+            // ---- partition round for lengths lfirst .. lfirst + kc - 1
+            __syncthreads();
+            uint32_t c[BPT], bs[BPT], sum = 0;
+#pragma unroll
+            for (int b = 0; b < BPT; ++b) {
+                const uint32_t bin = threadIdx.x * BPT + b;
+                c[b] = cnt[bin];
+                cnt[bin] = 0;
+                const uint32_t q = bin / NBL;
+                bs[b] = (c[b] && q < kc)
+                            ? atomicAdd(&a.fill[(uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL], c[b])
+                            : 0u;
+                sum += c[b];
+            }
+            uint32_t run = block_scan<SC_THREADS>(sum, wsum);
+#pragma unroll
+            for (int b = 0; b < BPT; ++b) {
+                const uint32_t bin = threadIdx.x * BPT + b;
+                const uint32_t q = bin / NBL;
+                lstart[bin] = run;
+                if ((uint64_t)bs[b] + c[b] > a.cap) {
+                    gofs[bin] = -1;
+                    *a.overflow = 1u;
+                } else {
+                    gofs[bin] = (long long)(((uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL) * a.cap +
+                                            bs[b]) - (long long)run;
+                }
+                run += c[b];
+            }
+            if (threadIdx.x == SC_THREADS - 1) lstart[NBIN] = run;
+            __syncthreads();
+            if (valid) {
+#pragma unroll
+                for (int q = 0; q < 2 * LPR; ++q)
+                    if ((uint32_t)q < 2 * kc) {
+                        const uint32_t b = rk[q] >> 16;
+                        const uint32_t u = lstart[b] + (rk[q] & 0xFFFFu);
+                        stage[u] = kk[q];
+                        sbin[u] = (unsigned short)b;
+                    }
+            }
+            __syncthreads();
+            const uint32_t total = lstart[NBIN];
+            for (uint32_t u = threadIdx.x; u < total; u += SC_THREADS) {
+                const long long go = gofs[sbin[u]];
+                if (go >= 0) a.out[go + u] = stage[u];
+            }
+            // the next round's first barrier orders these reads before stage/lstart reuse
+        }
+    }
+}
+
 lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
 {
     if (args.n == 0) return LASAGNA_OK;
@@ -223,6 +370,15 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
             LSG_LAUNCHED("scatter_table_kernel");
             return LASAGNA_OK;
         };
+        // LASAGNA_SCATTER=1 (A/B measurements only): round-1 form of the kernel
+        const char *ev = getenv("LASAGNA_SCATTER");
+        if (ev && ev[0] == '1') {
+            if (args.split)
+                return args.ascii ? run(scatter_table_kernel_v1<W, true, true, 1>, 1)
+                                  : run(scatter_table_kernel_v1<W, false, true, 1>, 1);
+            return args.ascii ? run(scatter_table_kernel_v1<W, true, false, 4>, 4)
+                              : run(scatter_table_kernel_v1<W, false, false, 4>, 4);
+        }
         if (args.split)
             return args.ascii ? run(scatter_table_kernel<W, true, true, 1>, 1)
                               : run(scatter_table_kernel<W, false, true, 1>, 1);
