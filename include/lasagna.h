@@ -125,6 +125,9 @@ typedef struct {
      * staging is fused into the first pass), a2 and the level-1 partition: one kernel */
     float ms_table, ms_sort, ms_search, ms_greedy;
     uint64_t greedy_pair_rounds; /* sum over greedy rounds of the candidate pairs visited    */
+    uint64_t pruned_entries;     /* table entries dropped by claimed-end pruning (groups after
+                                    the first; then n_pairs counts only pairs of entries that
+                                    were live when their group was built, not the full |P|) */
     uint32_t partition_levels;   /* bucketed path: MSD partition levels (1..3); 0: exact path */
     uint32_t reserved;
 } lasagna_stats;

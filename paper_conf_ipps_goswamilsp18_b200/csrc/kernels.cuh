@@ -84,6 +84,11 @@ struct ScatterArgs {
     const unsigned char *ascii;
     uint64_t *packed_out;
     unsigned long long *first_bad;
+    // claimed-end pruning (may be null): the entry of vertex v is dropped when
+    // read end v^1 is already claimed (bitmap of 2n bits) — every pair it could produce
+    // contains v^1, which the greedy would reject; pruned entries are counted
+    const uint32_t *claimed = nullptr;
+    unsigned long long *pruned = nullptr;
 };
 lasagna_status launch_scatter_table(const ScatterArgs &a, cudaStream_t s);
 struct RefineArgs {
@@ -108,7 +113,8 @@ struct BucketJoinArgs {
     uint64_t half_cap, n_buckets;
     uint32_t *overflow;
 };
-lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s);
+lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s); // block windows
+lasagna_status launch_warp_join(const BucketJoinArgs &a, cudaStream_t s);   // warp per bucket
 
 // ---- a6/a7 (greedy.cu)
 struct GreedyBufs {

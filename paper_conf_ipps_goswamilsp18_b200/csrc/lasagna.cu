@@ -127,7 +127,7 @@ struct Layout {
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
 enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR_FOUND = 8,
-       CTR_POOL3 = 9, CTR_WORK = 10, CTR64_N = 11 };
+       CTR_POOL3 = 9, CTR_WORK = 10, CTR_PRUNED = 11, CTR64_N = 12 };
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -230,6 +230,7 @@ struct Run {
     unsigned long long *ctr64; // CTR_* counters
     unsigned long long *pool, *pool2;
     const uint32_t *claimed = nullptr; // greedy mode: the join drops pairs with a claimed end
+    bool prune = false; // this group's scatter drops entries whose read end is claimed (f1)
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
     void bind(void *workspace)
     {
@@ -395,6 +396,8 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.cap = sa.split ? g.half : g.cap1;
     sa.overflow = ovf;
     sa.ascii = r.ascii; // fused a1 (first group only)
+    sa.claimed = r.prune ? r.claimed : nullptr;
+    sa.pruned = r.ctr64 + CTR_PRUNED;
     sa.packed_out = r.packed_out;
     sa.first_bad = r.first_bad;
     const char *host = r.ascii_host;
@@ -519,7 +522,8 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * g.n_buckets;
         bj.half_cap = g.half;
         bj.n_buckets = g.n_buckets;
-        rc = launch_bucket_join(bj, r.s);
+        // one warp per bucket (warpjoin.cu); LASAGNA_JOIN=bulk (A/B only): block windows
+        rc = env_flag("LASAGNA_JOIN", 'b') ? launch_bucket_join(bj, r.s) : launch_warp_join(bj, r.s);
     } else {
         rc = launch_join(ja, r.s);
     }
@@ -764,6 +768,11 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     for (int64_t l_hi = (int64_t)L - 1; l_hi >= (int64_t)l_min; l_hi -= G) {
         const uint32_t l_lo = (uint32_t)std::max<int64_t>(l_min, l_hi - (int64_t)G + 1);
         int which = 0;
+        // f1: every group after the first is built after the greedy of all
+        // longer lengths, so its scatter drops the entries of claimed read ends (P:L152,
+        // a claimed end can never gain an edge).  LASAGNA_NO_PRUNE=1 keeps them (then
+        // n_pairs is the full |P|).
+        r.prune = l_hi != (int64_t)L - 1 && !env_flag("LASAGNA_NO_PRUNE", '1');
         if ((rc = build_group(r, packed, l_lo, (uint32_t)l_hi, &which, tm, &st)) != LASAGNA_OK)
             return rc;
         ++st.passes;
@@ -807,6 +816,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         st.rounds_max = (uint32_t)book[3];
         st.fp_false_matches = h[CTR_FALSE];
         st.greedy_pair_rounds = h[CTR_WORK];
+        st.pruned_entries = h[CTR_PRUNED];
         st.partition_levels = r.bucketed ? g.P : 0;
         if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
         st.kernel_launches = launch_count() - launches0;

@@ -279,6 +279,18 @@ scatter_table_kernel(ScatterArgs a)
         if ((m & 31u) == 0u && m) ty = wsel<W>(x, (m >> 5) - 1u);
     };
     for (; k + 1u < a.l_lo; ++k) step_base(k); // bases before the first emitted length
+    // claimed-end pruning: entry of v0 = 2i needs read end 2i+1 free, entry of 2i+1 needs 2i
+    bool live0 = valid, live1 = valid;
+    if (a.claimed && valid) {
+        const uint32_t cw = a.claimed[v0 >> 5] >> (uint32_t)(v0 & 31u);
+        live0 = ((cw >> 1) & 1u) == 0u;
+        live1 = (cw & 1u) == 0u;
+        if (a.pruned) {
+            uint32_t np = ((uint32_t)!live0 + (uint32_t)!live1) * (a.l_hi - a.l_lo + 1u);
+            for (int o = 16; o; o >>= 1) np += __shfl_xor_sync(0xffffffffu, np, o);
+            if ((threadIdx.x & 31) == 0 && np) atomicAdd(a.pruned, (unsigned long long)np);
+        }
+    }
     uint64_t kk[KPT];
     uint32_t rk[KPT]; // bin << 16 | rank within the bin
     for (uint32_t lfirst = a.l_lo; lfirst <= a.l_hi; lfirst += LPR) {
@@ -287,7 +299,8 @@ scatter_table_kernel(ScatterArgs a)
         for (int q = 0; q < LPR; ++q) {
             if ((uint32_t)q >= kc) break; // block-uniform
             step_base(lfirst + q - 1u);    // the streams now hold length lfirst + q
-            if (valid) {
+            rk[2 * q] = rk[2 * q + 1] = ~0u; // no key (pruned or no read)
+            if (live0 | live1) {
                 uint32_t d0, d1; // level-1 digits (implied by the region, not stored)
                 const uint64_t e0 = canon_key_d1(st.P0, st.S1, a.keep, a.vbits, v0, &d0);
                 const uint64_t e1 = canon_key_d1(st.P1, st.S0, a.keep, a.vbits, v0 + 1, &d1);
@@ -298,8 +311,8 @@ scatter_table_kernel(ScatterArgs a)
                 kk[2 * q] = e0;
                 kk[2 * q + 1] = e1;
                 const uint32_t b0 = q * NBL + d0, b1 = q * NBL + d1;
-                rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
-                rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
+                if (live0) rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
+                if (live1) rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
             }
         }
         {
@@ -334,10 +347,10 @@ scatter_table_kernel(ScatterArgs a)
             }
             if (threadIdx.x == SC_THREADS - 1) lstart[NBIN] = run;
             __syncthreads();
-            if (valid) {
+            if (live0 | live1) {
 #pragma unroll
                 for (int q = 0; q < 2 * LPR; ++q)
-                    if ((uint32_t)q < 2 * kc) {
+                    if ((uint32_t)q < 2 * kc && rk[q] != ~0u) {
                         const uint32_t b = rk[q] >> 16;
                         const uint32_t u = lstart[b] + (rk[q] & 0xFFFFu);
                         stage[u] = kk[q];

@@ -35,7 +35,8 @@ class _Stats(ctypes.Structure):
                 ("ms_table", ctypes.c_float), ("ms_sort", ctypes.c_float),
                 ("ms_search", ctypes.c_float),
                 ("ms_greedy", ctypes.c_float),
-                ("greedy_pair_rounds", ctypes.c_uint64), ("partition_levels", ctypes.c_uint32),
+                ("greedy_pair_rounds", ctypes.c_uint64), ("pruned_entries", ctypes.c_uint64),
+                ("partition_levels", ctypes.c_uint32),
                 ("reserved", ctypes.c_uint32)]
 
     def as_dict(self) -> dict:

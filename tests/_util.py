@@ -80,3 +80,22 @@ def check_graph(reads: np.ndarray, l_min: int, succ: np.ndarray, olen: np.ndarra
         free_b = ~has[np.asarray(pb, dtype=np.int64)]
         assert not np.any(free_a & free_b), "greedy result is not maximal"
     return len(us)
+
+
+def pruning_expectations(L: int, l_min: int, G: int, pairs, olen) -> tuple[int, int]:
+    """What claimed-end pruning must report for length groups of G lengths
+    (L-1 down to l_min): a read end x is claimed at length olen[x] (the greedy claims every end
+    at most once), so when the group whose top length is l_hi is built, exactly the ends with
+    olen[x] > l_hi are claimed.  The entry of vertex x^1 at each length of that group is then
+    dropped (pruned entries), and a pair (l, a, b) is still found iff neither a nor b was
+    claimed before its group.  Returns (pairs found, entries pruned)."""
+    pl, pa, pb = (np.asarray(t) for t in pairs)
+    olen = np.asarray(olen, dtype=np.int64)
+    top = L - 1 - ((L - 1 - pl.astype(np.int64)) // G) * G  # l_hi of each pair's group
+    found = int(np.count_nonzero((olen[pa] <= top) & (olen[pb] <= top)))
+    counts = np.bincount(olen, minlength=256)  # ends claimed at each length (0: never)
+    pruned = 0
+    for l_hi in range(L - 1 - G, l_min - 1, -G):
+        g = min(G, l_hi - l_min + 1)
+        pruned += g * int(counts[l_hi + 1:].sum())
+    return found, pruned

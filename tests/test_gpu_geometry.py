@@ -16,6 +16,7 @@ import pytest
 
 import oracle
 import readgen
+from tests._util import pruning_expectations
 
 gpu = pytest.mark.gpu
 
@@ -30,13 +31,18 @@ def lz():
     return m
 
 
+_P2 = {}
+
+
 @pytest.fixture(scope="module")
 def cfg2():
     """cfg2 (BASELINE configs[1]: 2.3 M reads of 100 bp, 1 % errors) and its oracle graph."""
     cfg = readgen.CONFIGS["cfg2"]
     reads = readgen.config_reads(cfg)
-    esucc, eolen, m, acc = oracle.greedy_graph(reads, cfg.l_min)
-    return cfg, reads, esucc, eolen, m, acc
+    P = oracle.overlaps(reads, cfg.l_min)
+    esucc, eolen, acc = oracle.greedy(cfg.n, *P)
+    _P2["P"] = P
+    return cfg, reads, esucc, eolen, len(P[0]), acc
 
 
 @pytest.fixture(scope="module")
@@ -56,10 +62,19 @@ def _u8(t):
     return t.cpu().numpy().view(np.uint8)
 
 
-def _same(r, esucc, eolen, m, acc):
-    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc, (r.stats, m, acc)
+def _same(r, esucc, eolen, m, acc, L=100, l_min=63):
+    """Bit-exact graph; |P| exact on one pass, or the claimed-end pruning counts of several
+    (tests/_util.pruning_expectations, from the oracle's pairs and claim lengths)."""
+    st = r.stats
+    assert st["n_greedy"] == acc, (st, acc)
     assert np.array_equal(_u32(r.succ), esucc)
     assert np.array_equal(_u8(r.olen), eolen)
+    if st["passes"] > 1 and st["bucketed"]:
+        found, pruned = pruning_expectations(L, l_min, st["lengths_per_pass"], _P2["P"], eolen)
+        assert (st["n_pairs"], st["pruned_entries"]) == (found, pruned), (st, found, pruned)
+        assert found < m and pruned > 0
+    else:
+        assert st["n_pairs"] == m and st["pruned_entries"] == 0, (st, m)
 
 
 @gpu
@@ -159,10 +174,13 @@ def test_pool_growth_retry_with_length_groups(lz, monkeypatch):
     workspace and retries; the graph equals the oracle."""
     import torch
     reads = readgen.reads(7, 20_000, 3000, 64, 0.01)
-    esucc, eolen, m, acc = oracle.greedy_graph(reads, 1)
+    P = oracle.overlaps(reads, 1)
+    esucc, eolen, acc = oracle.greedy(3000, *P)
     packed = lz.load_reads(torch.from_numpy(reads).cuda())
     r = lz.greedy_graph(packed, 3000, 64, 1, lengths_per_pass=5)
-    _same(r, esucc, eolen, m, acc)
+    assert np.array_equal(_u32(r.succ), esucc) and np.array_equal(_u8(r.olen), eolen)
+    found, pruned = pruning_expectations(64, 1, 5, P, eolen)
+    assert (r.stats["n_pairs"], r.stats["pruned_entries"]) == (found, pruned)
 
 
 def _expected_false_matches(n: int, n_len: int, bits: float) -> float:
@@ -205,3 +223,16 @@ def test_false_match_rate_vertex_bits_32_closed_form():
     true_per_len = 3.86e9 / (cfg.L - cfg.l_min)  # SURVEY 8(d) expected |P|
     assert per_len < 0.1 * true_per_len
     assert _expected_false_matches(cfg.n, 1, 62 - vbits) > 10 * true_per_len
+
+
+@gpu
+def test_pruning_off_gives_full_pair_count(lz, cfg2, monkeypatch):
+    """LASAGNA_NO_PRUNE=1: several passes, nothing pruned, |P| exact, same graph."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    monkeypatch.setenv("LASAGNA_NO_PRUNE", "1")
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=5)
+    assert r.stats["passes"] == 8 and r.stats["pruned_entries"] == 0
+    assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc
+    assert np.array_equal(_u32(r.succ), esucc) and np.array_equal(_u8(r.olen), eolen)

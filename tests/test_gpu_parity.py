@@ -16,7 +16,7 @@ import pytest
 import oracle
 import readgen
 from oracle import brute
-from tests._util import NONE, check_graph, golden, to_array
+from tests._util import NONE, check_graph, golden, pruning_expectations, to_array
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -247,7 +247,10 @@ def test_cfg1_parity(lz):
         r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=lpp)
         assert np.array_equal(_np(r.succ, np.uint32), esucc), lpp
         assert np.array_equal(_np(r.olen, np.uint8), eolen), lpp
-        assert r.stats["n_pairs"] == len(epl)
+        # later groups drop the entries of claimed read ends (claimed-end pruning)
+        G = r.stats["lengths_per_pass"]
+        assert (r.stats["n_pairs"], r.stats["pruned_entries"]) == pruning_expectations(
+            cfg.L, cfg.l_min, G, (epl, epa, epb), eolen), lpp
     check_graph(reads, cfg.l_min, esucc, eolen, (epl, epa, epb))
 
 
