@@ -108,6 +108,75 @@ __device__ __forceinline__ void fp_skip(const uint64_t (&x)[W], const uint64_t (
     st.P0 = fold61(P0), st.P1 = fold61(P1), st.S0 = fold61(S0), st.S1 = fold61(S1);
 }
 
+// Stream states after exactly the first nb bases of r (x) and r' (y), any nb <= 32 W
+// (block-uniform): whole 16-base half-words as in fp_skip, then the remaining nb mod 16 bases
+// as one or two chunks of k <= 8 bases.  A forward chunk of k bases is chunk8_fwd of its
+// bases moved to the top k positions (P <- P 5^k + value); the ascending-power streams
+// evaluate their polynomial from the highest base down, so the partial chunk comes first.
+__device__ __forceinline__ uint32_t pow5_small(uint32_t k)
+{
+    uint32_t p = 1;
+    for (uint32_t t = 0; t < k; ++t) p *= 5u;
+    return p;
+}
+template <int W>
+__device__ __forceinline__ void fp_absorb(const uint64_t (&x)[W], const uint64_t (&y)[W],
+                                          uint32_t nb, FpStreams &st)
+{
+    const uint32_t nh = nb >> 4, rem = nb & 15u;
+    uint64_t P0 = 0, P1 = 0, S0 = 0, S1 = 0;
+#pragma unroll
+    for (int h = 0; h < 2 * W; ++h) {
+        if ((uint32_t)h >= nh) break;
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1)));
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1)));
+        P0 = mulsmall61(P0, POW5_8) + chunk8_fwd(hx);
+        P0 = mulsmall61(P0, POW5_8) + chunk8_fwd(hx >> 16);
+        P1 = mulsmall61(P1, POW5_8) + chunk8_fwd(hy);
+        P1 = mulsmall61(P1, POW5_8) + chunk8_fwd(hy >> 16);
+    }
+    // the partial half-word nh (bases 16 nh .. 16 nh + rem - 1), rem < 16
+    uint32_t px = 0, py = 0;
+    if (rem) {
+        px = (uint32_t)(wsel<W>(x, nh >> 1) >> (32 * (nh & 1)));
+        py = (uint32_t)(wsel<W>(y, nh >> 1) >> (32 * (nh & 1)));
+        const uint32_t mask = rem == 16 ? 0xFFFFFFFFu : ((1u << (2 * rem)) - 1u);
+        px &= mask;
+        py &= mask;
+        const uint32_t k1 = min(rem, 8u), k2 = rem - k1; // forward: low chunk first
+        const uint32_t m1 = pow5_small(k1);
+        P0 = mulsmall61(P0, m1) + chunk8_fwd((px & 0xFFFFu) << (2 * (8 - k1)));
+        P1 = mulsmall61(P1, m1) + chunk8_fwd((py & 0xFFFFu) << (2 * (8 - k1)));
+        if (k2) {
+            const uint32_t m2 = pow5_small(k2);
+            P0 = mulsmall61(P0, m2) + chunk8_fwd(((px >> 16) << (2 * (8 - k2))) & 0xFFFFu);
+            P1 = mulsmall61(P1, m2) + chunk8_fwd(((py >> 16) << (2 * (8 - k2))) & 0xFFFFu);
+        }
+        // ascending-power streams: the partial (highest) bases first, high chunk first
+        const uint32_t cx = px ^ (0xAAAAAAAAu & mask), cy = py ^ (0xAAAAAAAAu & mask);
+        if (k2) {
+            S1 = chunk8_bwd(cx >> 16);
+            S0 = chunk8_bwd(cy >> 16);
+            S1 = mulsmall61(S1, m1) + chunk8_bwd(cx & 0xFFFFu);
+            S0 = mulsmall61(S0, m1) + chunk8_bwd(cy & 0xFFFFu);
+        } else {
+            S1 = chunk8_bwd(cx & 0xFFFFu);
+            S0 = chunk8_bwd(cy & 0xFFFFu);
+        }
+    }
+#pragma unroll
+    for (int h = 2 * W - 1; h >= 0; --h) {
+        if ((uint32_t)h >= nh) continue;
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        S1 = mulsmall61(S1, POW5_8) + chunk8_bwd(hx >> 16);
+        S1 = mulsmall61(S1, POW5_8) + chunk8_bwd(hx);
+        S0 = mulsmall61(S0, POW5_8) + chunk8_bwd(hy >> 16);
+        S0 = mulsmall61(S0, POW5_8) + chunk8_bwd(hy);
+    }
+    st.P0 = fold61(P0), st.P1 = fold61(P1), st.S0 = fold61(S0), st.S1 = fold61(S1);
+}
+
 // half-words a kernel whose first emitted length is l_first can absorb (bases < l_first - 1)
 __host__ __device__ __forceinline__ uint32_t skip_halves(uint32_t l_first)
 {

@@ -258,12 +258,12 @@ scatter_table_kernel(ScatterArgs a)
     __syncthreads();
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
-    const uint32_t nh = min(skip_halves(a.l_lo), 2u * W); // leading bases absorbed in chunks
-    fp_skip<W>(x, y, nh, st);
+    // the l_lo - 1 bases before the first emitted length, absorbed in 8-base chunks
+    fp_absorb<W>(x, y, a.l_lo - 1u, st);
     // Base cursors over x (y is dead from here): tx holds base k of r in its low bits; ty
     // holds base L-1-k of r in its top bits, i.e. base k of r' = RC(r) complemented.  A word
     // boundary reloads a cursor from x with a register select (block-uniform branch).
-    uint32_t k = 16u * nh; // next base to consume (block-uniform)
+    const uint32_t k = a.l_lo - 1u; // next base to consume (block-uniform)
     uint64_t tx = wsel<W>(x, k >> 5) >> (2u * (k & 31u));
     uint64_t ty;
     {
@@ -278,18 +278,17 @@ scatter_table_kernel(ScatterArgs a)
         const uint32_t m = a.L - 1u - kb;
         if ((m & 31u) == 0u && m) ty = wsel<W>(x, (m >> 5) - 1u);
     };
-    for (; k + 1u < a.l_lo; ++k) step_base(k); // bases before the first emitted length
     // claimed-end pruning: entry of v0 = 2i needs read end 2i+1 free, entry of 2i+1 needs 2i
     bool live0 = valid, live1 = valid;
-    if (a.claimed && valid) {
-        const uint32_t cw = a.claimed[v0 >> 5] >> (uint32_t)(v0 & 31u);
-        live0 = ((cw >> 1) & 1u) == 0u;
-        live1 = (cw & 1u) == 0u;
-        if (a.pruned) {
-            uint32_t np = ((uint32_t)!live0 + (uint32_t)!live1) * (a.l_hi - a.l_lo + 1u);
-            for (int o = 16; o; o >>= 1) np += __shfl_xor_sync(0xffffffffu, np, o);
-            if ((threadIdx.x & 31) == 0 && np) atomicAdd(a.pruned, (unsigned long long)np);
+    if (a.claimed) { // block-uniform
+        if (valid) {
+            const uint32_t cw = a.claimed[v0 >> 5] >> (uint32_t)(v0 & 31u);
+            live0 = ((cw >> 1) & 1u) == 0u;
+            live1 = (cw & 1u) == 0u;
         }
+        uint32_t np = valid ? ((uint32_t)!live0 + (uint32_t)!live1) * (a.l_hi - a.l_lo + 1u) : 0u;
+        for (int o = 16; o; o >>= 1) np += __shfl_xor_sync(0xffffffffu, np, o);
+        if ((threadIdx.x & 31) == 0 && np && a.pruned) atomicAdd(a.pruned, (unsigned long long)np);
     }
     uint64_t kk[KPT];
     uint32_t rk[KPT]; // bin << 16 | rank within the bin

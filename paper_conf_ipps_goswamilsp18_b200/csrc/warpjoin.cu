@@ -125,8 +125,16 @@ warp_join_kernel(BucketJoinArgs b)
     uint32_t epoch = 0;
     unsigned long long nfalse = 0;
     const uint64_t nw = (uint64_t)gridDim.x * WJ_WARPS;
-    for (uint64_t bk = (uint64_t)blockIdx.x * WJ_WARPS + wid; bk < b.n_buckets; bk += nw) {
-        uint32_t fP = b.fills[2 * bk], fS = b.fills[2 * bk + 1];
+    // the fills of the warp's next bucket are loaded one bucket ahead, and once they are in,
+    // lane 0 prefetches that bucket's two halves into L2 (cp.async.bulk.prefetch) while the
+    // warp still works on the current one
+    uint64_t bk = (uint64_t)blockIdx.x * WJ_WARPS + wid;
+    uint32_t nfP = 0, nfS = 0;
+    if (bk < b.n_buckets) nfP = b.fills[2 * bk], nfS = b.fills[2 * bk + 1];
+    for (; bk < b.n_buckets; bk += nw) {
+        uint32_t fP = nfP, fS = nfS;
+        const uint64_t bn = bk + nw;
+        if (bn < b.n_buckets) nfP = b.fills[2 * bn], nfS = b.fills[2 * bn + 1];
         if (fP > b.half_cap || fS > b.half_cap) {
             if (lane == 0) *b.overflow = 1u; // the call is redone on the exact path
             fP = (uint32_t)min64(fP, b.half_cap);
@@ -148,16 +156,39 @@ warp_join_kernel(BucketJoinArgs b)
                 epoch = 1;
             }
             __syncwarp();
-            // 1. copy + hash the build chunk
+            // 1. copy + hash the build chunk, WJ_U loads per lane in flight
             bool h2 = false;
-            for (uint32_t j = lane; j < nb; j += 32) {
-                const uint64_t e = P[c0 + j];
-                S.key[j] = e;
-                h2 |= (e & flag2bit) != 0;
-                const uint32_t old = atomicExch(&S.head[(uint32_t)(e >> kshift) & (WJ_HS - 1)], (epoch << 16) | j);
-                S.next[j] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : (unsigned short)0xFFFFu;
+            for (uint32_t j0 = 0; j0 < nb; j0 += 32 * WJ_U) {
+                uint64_t be[WJ_U];
+#pragma unroll
+                for (int u = 0; u < WJ_U; ++u) {
+                    const uint32_t j = j0 + u * 32 + lane;
+                    be[u] = j < nb ? P[c0 + j] : 0ull;
+                }
+#pragma unroll
+                for (int u = 0; u < WJ_U; ++u) {
+                    const uint32_t j = j0 + u * 32 + lane;
+                    if (j < nb) {
+                        const uint64_t e = be[u];
+                        S.key[j] = e;
+                        h2 |= (e & flag2bit) != 0;
+                        const uint32_t old =
+                            atomicExch(&S.head[(uint32_t)(e >> kshift) & (WJ_HS - 1)], (epoch << 16) | j);
+                        S.next[j] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu)
+                                                         : (unsigned short)0xFFFFu;
+                    }
+                }
             }
             if (fP <= (uint32_t)WJ_SB) has2 = __any_sync(0xffffffffu, h2);
+            if (c0 == 0 && lane == 0 && bn < b.n_buckets) {
+                const uint64_t *Pn = b.buckets + bn * 2 * b.half_cap;
+                const uint32_t bp = (uint32_t)min64(nfP, b.half_cap) * 8u, bs = (uint32_t)min64(nfS, b.half_cap) * 8u;
+                if (bp >= 16)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(Pn), "r"(bp & ~15u) : "memory");
+                if (bs >= 16)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(Pn + b.half_cap), "r"(bs & ~15u)
+                                 : "memory");
+            }
             __syncwarp();
             // 2. the probe half, WJ_U loads per lane in flight
             for (uint32_t t0 = 0; t0 < fS; t0 += 32 * WJ_U) {
