@@ -115,6 +115,7 @@ struct BucketJoinArgs {
 };
 lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s); // block windows
 lasagna_status launch_warp_join(const BucketJoinArgs &a, cudaStream_t s);   // warp per bucket
+bool warp_join_fits(const BucketJoinArgs &a); // a bucket half fits a warp's staging slice
 
 // ---- a6/a7 (greedy.cu)
 struct GreedyBufs {

@@ -522,8 +522,10 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * g.n_buckets;
         bj.half_cap = g.half;
         bj.n_buckets = g.n_buckets;
-        // one warp per bucket (warpjoin.cu); LASAGNA_JOIN=bulk (A/B only): block windows
-        rc = env_flag("LASAGNA_JOIN", 'b') ? launch_bucket_join(bj, r.s) : launch_warp_join(bj, r.s);
+        // one warp per bucket (warpjoin.cu) when a half fits a warp's slice, else block
+        // windows (partition.cu); LASAGNA_JOIN=bulk (A/B only) forces the block windows
+        rc = (env_flag("LASAGNA_JOIN", 'b') || !warp_join_fits(bj)) ? launch_bucket_join(bj, r.s)
+                                                                    : launch_warp_join(bj, r.s);
     } else {
         rc = launch_join(ja, r.s);
     }

@@ -13,27 +13,28 @@
 //   3. candidates (equal stored key bits, different reads) go to a per-warp buffer; when it
 //      fills, the warp verifies them on the 2-bit bases, one per lane (R12), and appends the
 //      verified read-end pairs (a << 32) | b with ONE global atomic per flush.
-// No block barrier anywhere: the warps of a CTA drift independently, so one warp's loads
-// overlap another's hashing.  A bucket with more build entries than a slice holds is joined
-// chunk by chunk (every chunk against the whole probe list).
+// No block barrier anywhere: the warps of a CTA drift independently.  Each warp double-
+// buffers its buckets: while it joins bucket k out of shared memory, the copy engine brings
+// bucket k + 1's two halves in (cp.async.bulk issued by lane 0, one mbarrier per buffer), so
+// the warp never waits on a global load.  Used when a half fits a slice (half capacity <=
+// WJ_SB: cfg1-cfg4 geometries); larger halves take the block-window join.
 #include "kernels.cuh"
 
 namespace lsg {
 
-constexpr int WJ_WARPS = 16;   // warps per CTA (one CTA per SM)
-constexpr int WJ_SB = 768;     // build entries per slice (cfg3 half capacity: 747)
+constexpr int WJ_WARPS = 7;    // warps per CTA (one CTA per SM; the slices fill shared memory)
+constexpr int WJ_SB = 768;     // entries per staged half (cfg3 half capacity: 747)
 constexpr int WJ_HS = 1024;    // chain heads per slice
 constexpr int WJ_CAND = 128;   // staged candidates per warp
 constexpr int WJ_FLUSH = 96;   // flush when this many are staged at a warp-uniform point
-constexpr int WJ_U = 4;        // probe loads in flight per lane
 
-struct WarpSlice {
-    unsigned long long key[WJ_SB];
-    uint32_t head[WJ_HS];   // (epoch << 16) | index
+struct alignas(128) WarpSlice {
+    unsigned long long buf[2][2][WJ_SB]; // [buffer][build, probe half][entry]
+    uint32_t head[WJ_HS];                // (epoch << 16) | index
     unsigned short next[WJ_SB];
     unsigned long long cand[WJ_CAND];
+    unsigned long long mbar[2];
     uint32_t ncand;
-    uint32_t pad[3];
 };
 
 // verify and append the staged candidates (warp-uniform call)
@@ -75,13 +76,14 @@ __device__ __forceinline__ void wj_flush(const JoinArgs &a, WarpSlice &S, unsign
 
 // probe entry e (vertex w, flag 1 or 2) against the slice's hash table
 template <int W>
-__device__ __forceinline__ void wj_probe(const JoinArgs &a, WarpSlice &S, uint64_t e, uint32_t epoch,
-                                         uint32_t kshift, uint64_t vmask, unsigned long long &nfalse)
+__device__ __forceinline__ void wj_probe(const JoinArgs &a, WarpSlice &S, const unsigned long long *key,
+                                         uint64_t e, uint32_t epoch, uint32_t kshift, uint64_t vmask,
+                                         unsigned long long &nfalse)
 {
     const uint32_t hv = S.head[(uint32_t)(e >> kshift) & (WJ_HS - 1)];
     uint32_t s = (hv >> 16) == epoch ? (hv & 0xFFFFu) : 0xFFFFu;
     while (s != 0xFFFFu) {
-        const uint64_t p = S.key[s];
+        const uint64_t p = key[s];
         if (((p ^ e) >> kshift) == 0) {
             const uint32_t w = (uint32_t)(e & vmask), v = (uint32_t)(p & vmask);
             // R9 (different reads); two flag-2 entries find each other twice: keep w < v
@@ -108,11 +110,33 @@ __device__ __forceinline__ void wj_probe(const JoinArgs &a, WarpSlice &S, uint64
     }
 }
 
+// lane 0: start the copies of bucket bk's halves (fills fP, fS) into buffer c
+__device__ __forceinline__ void wj_issue(const BucketJoinArgs &b, WarpSlice &S, int c, uint64_t bk,
+                                         uint32_t fP, uint32_t fS)
+{
+    const uint32_t bp = ((fP + 1u) & ~1u) * 8u, bs = ((fS + 1u) & ~1u) * 8u; // 16-byte units
+    const uint32_t bar = smem_u32(&S.mbar[c]);
+    fence_proxy_async(); // the buffer was last read by the generic proxy
+    if (bp + bs == 0) {
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+        return;
+    }
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bp + bs)
+                 : "memory");
+    const uint64_t *P = b.buckets + bk * 2 * b.half_cap;
+    if (bp)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     ::"r"(smem_u32(S.buf[c][0])), "l"(P), "r"(bp), "r"(bar) : "memory");
+    if (bs)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     ::"r"(smem_u32(S.buf[c][1])), "l"(P + b.half_cap), "r"(bs), "r"(bar) : "memory");
+}
+
 template <int W>
 __global__ void __launch_bounds__(WJ_WARPS * 32, 1)
 warp_join_kernel(BucketJoinArgs b)
 {
-    extern __shared__ __align__(16) unsigned char wjsm[];
+    extern __shared__ __align__(128) unsigned char wjsm[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpSlice &S = reinterpret_cast<WarpSlice *>(wjsm)[wid];
     const JoinArgs &a = b.j;
@@ -120,100 +144,75 @@ warp_join_kernel(BucketJoinArgs b)
     const uint64_t vmask = (1ull << a.vbits) - 1;
     const uint64_t flag2bit = 2ull << a.vbits;
     for (uint32_t t = lane; t < (uint32_t)WJ_HS; t += 32) S.head[t] = 0;
-    if (lane == 0) S.ncand = 0;
+    if (lane == 0) {
+        S.ncand = 0;
+        mbar_init(&S.mbar[0], 1);
+        mbar_init(&S.mbar[1], 1);
+        fence_mbar_init();
+    }
     __syncwarp();
-    uint32_t epoch = 0;
+    uint32_t epoch = 0, phases = 0; // bit c: parity of the next completion of mbar[c]
     unsigned long long nfalse = 0;
     const uint64_t nw = (uint64_t)gridDim.x * WJ_WARPS;
-    // the fills of the warp's next bucket are loaded one bucket ahead, and once they are in,
-    // lane 0 prefetches that bucket's two halves into L2 (cp.async.bulk.prefetch) while the
-    // warp still works on the current one
     uint64_t bk = (uint64_t)blockIdx.x * WJ_WARPS + wid;
-    uint32_t nfP = 0, nfS = 0;
-    if (bk < b.n_buckets) nfP = b.fills[2 * bk], nfS = b.fills[2 * bk + 1];
-    for (; bk < b.n_buckets; bk += nw) {
-        uint32_t fP = nfP, fS = nfS;
-        const uint64_t bn = bk + nw;
-        if (bn < b.n_buckets) nfP = b.fills[2 * bn], nfS = b.fills[2 * bn + 1];
+    auto fills = [&](uint64_t k, uint32_t &fP, uint32_t &fS) {
+        fP = b.fills[2 * k];
+        fS = b.fills[2 * k + 1];
         if (fP > b.half_cap || fS > b.half_cap) {
             if (lane == 0) *b.overflow = 1u; // the call is redone on the exact path
             fP = (uint32_t)min64(fP, b.half_cap);
             fS = (uint32_t)min64(fS, b.half_cap);
         }
-        const uint64_t *P = b.buckets + bk * 2 * b.half_cap;
-        const uint64_t *Q = P + b.half_cap;
-        // flag-2 build entries also probe; with several chunks every chunk must see all of them
-        bool has2 = false;
-        if (fP > (uint32_t)WJ_SB) {
-            for (uint32_t j = lane; j < fP; j += 32) has2 |= (P[j] & flag2bit) != 0;
-            has2 = __any_sync(0xffffffffu, has2);
+    };
+    uint32_t fP = 0, fS = 0;
+    if (bk < b.n_buckets) {
+        fills(bk, fP, fS);
+        if (lane == 0) wj_issue(b, S, 0, bk, fP, fS);
+    }
+    for (int c = 0; bk < b.n_buckets; bk += nw, c ^= 1) {
+        // start the next bucket's copies into the other buffer (free: its last bucket is done)
+        const uint64_t bn = bk + nw;
+        uint32_t nP = 0, nS = 0;
+        if (bn < b.n_buckets) {
+            fills(bn, nP, nS);
+            __syncwarp();
+            if (lane == 0) wj_issue(b, S, c ^ 1, bn, nP, nS);
         }
-        for (uint32_t c0 = 0; c0 < fP; c0 += WJ_SB) {
-            const uint32_t nb = min((uint32_t)WJ_SB, fP - c0);
-            if (++epoch == 0x10000u) {
-                __syncwarp();
-                for (uint32_t t = lane; t < (uint32_t)WJ_HS; t += 32) S.head[t] = 0;
-                epoch = 1;
-            }
+        mbar_wait(&S.mbar[c], (phases >> c) & 1u);
+        phases ^= 1u << c;
+        const unsigned long long *Pb = S.buf[c][0], *Qb = S.buf[c][1];
+        if (++epoch == 0x10000u) {
+            for (uint32_t t = lane; t < (uint32_t)WJ_HS; t += 32) S.head[t] = 0;
+            epoch = 1;
             __syncwarp();
-            // 1. copy + hash the build chunk, WJ_U loads per lane in flight
-            bool h2 = false;
-            for (uint32_t j0 = 0; j0 < nb; j0 += 32 * WJ_U) {
-                uint64_t be[WJ_U];
-#pragma unroll
-                for (int u = 0; u < WJ_U; ++u) {
-                    const uint32_t j = j0 + u * 32 + lane;
-                    be[u] = j < nb ? P[c0 + j] : 0ull;
-                }
-#pragma unroll
-                for (int u = 0; u < WJ_U; ++u) {
-                    const uint32_t j = j0 + u * 32 + lane;
-                    if (j < nb) {
-                        const uint64_t e = be[u];
-                        S.key[j] = e;
-                        h2 |= (e & flag2bit) != 0;
-                        const uint32_t old =
-                            atomicExch(&S.head[(uint32_t)(e >> kshift) & (WJ_HS - 1)], (epoch << 16) | j);
-                        S.next[j] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu)
-                                                         : (unsigned short)0xFFFFu;
-                    }
-                }
-            }
-            if (fP <= (uint32_t)WJ_SB) has2 = __any_sync(0xffffffffu, h2);
-            if (c0 == 0 && lane == 0 && bn < b.n_buckets) {
-                const uint64_t *Pn = b.buckets + bn * 2 * b.half_cap;
-                const uint32_t bp = (uint32_t)min64(nfP, b.half_cap) * 8u, bs = (uint32_t)min64(nfS, b.half_cap) * 8u;
-                if (bp >= 16)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(Pn), "r"(bp & ~15u) : "memory");
-                if (bs >= 16)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(Pn + b.half_cap), "r"(bs & ~15u)
-                                 : "memory");
-            }
+        }
+        // 1. hash the build half
+        bool h2 = false;
+        for (uint32_t j = lane; j < fP; j += 32) {
+            const uint64_t e = Pb[j];
+            h2 |= (e & flag2bit) != 0;
+            const uint32_t old = atomicExch(&S.head[(uint32_t)(e >> kshift) & (WJ_HS - 1)], (epoch << 16) | j);
+            S.next[j] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : (unsigned short)0xFFFFu;
+        }
+        const bool has2 = __any_sync(0xffffffffu, h2);
+        __syncwarp();
+        // 2. the probe half (and flag-2 build entries, rare)
+        for (uint32_t t0 = 0; t0 < fS; t0 += 32) {
+            if (t0 + lane < fS) wj_probe<W>(a, S, Pb, Qb[t0 + lane], epoch, kshift, vmask, nfalse);
             __syncwarp();
-            // 2. the probe half, WJ_U loads per lane in flight
-            for (uint32_t t0 = 0; t0 < fS; t0 += 32 * WJ_U) {
-                uint64_t pe[WJ_U];
-#pragma unroll
-                for (int u = 0; u < WJ_U; ++u) {
-                    const uint32_t t = t0 + u * 32 + lane;
-                    pe[u] = t < fS ? Q[t] : 0ull;
-                }
-#pragma unroll
-                for (int u = 0; u < WJ_U; ++u)
-                    if (t0 + u * 32 + lane < fS) wj_probe<W>(a, S, pe[u], epoch, kshift, vmask, nfalse);
-                __syncwarp();
-                if (S.ncand >= (uint32_t)WJ_FLUSH) wj_flush<W>(a, S, nfalse);
-            }
-            // flag-2 build entries as probes (palindromic prefixes or H == Hr: rare)
-            if (has2) {
-                for (uint32_t j = lane; j < fP; j += 32) {
-                    const uint64_t e = P[j];
-                    if (e & flag2bit) wj_probe<W>(a, S, e, epoch, kshift, vmask, nfalse);
-                }
+            if (S.ncand >= (uint32_t)WJ_FLUSH) wj_flush<W>(a, S, nfalse);
+        }
+        if (has2) {
+            for (uint32_t j0 = 0; j0 < fP; j0 += 32) {
+                const uint32_t j = j0 + lane;
+                if (j < fP && (Pb[j] & flag2bit)) wj_probe<W>(a, S, Pb, Pb[j], epoch, kshift, vmask, nfalse);
                 __syncwarp();
                 if (S.ncand >= (uint32_t)WJ_FLUSH) wj_flush<W>(a, S, nfalse);
             }
         }
+        __syncwarp(); // buffer c is read: the next issue may overwrite it
+        fP = nP;
+        fS = nS;
     }
     __syncwarp();
     wj_flush<W>(a, S, nfalse);
@@ -221,9 +220,12 @@ warp_join_kernel(BucketJoinArgs b)
     if (lane == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
 
+bool warp_join_fits(const BucketJoinArgs &args) { return args.half_cap <= (uint64_t)WJ_SB; }
+
 lasagna_status launch_warp_join(const BucketJoinArgs &args, cudaStream_t s)
 {
     if (args.n_buckets == 0) return LASAGNA_OK;
+    if (!warp_join_fits(args) || (args.half_cap & 1)) return LASAGNA_EINVAL;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
         const size_t smem = sizeof(WarpSlice) * WJ_WARPS;
