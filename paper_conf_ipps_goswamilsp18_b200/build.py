@@ -46,19 +46,39 @@ def nvcc() -> str:
     raise RuntimeError("nvcc not found: cannot build liblasagna.so")
 
 
+def _compile(src: str, obj: str) -> subprocess.CompletedProcess:
+    return subprocess.run([nvcc(), *NVCC_FLAGS, "-I", INCLUDE, "-c", "-o", obj, src],
+                          capture_output=True, text=True)
+
+
 def build(verbose: bool = False, force: bool = False) -> str:
+    """Compile every csrc/*.cu to an object in parallel (one nvcc per translation unit; no
+    device code crosses units), then link the shared library."""
     if not force and not stale():
         return SO
-    cmd = [nvcc(), *NVCC_FLAGS, "-shared", "-I", INCLUDE, "-o", SO + ".tmp", *sources()]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+    from concurrent.futures import ThreadPoolExecutor
+
+    objdir = os.path.join(PKG, ".obj")
+    os.makedirs(objdir, exist_ok=True)
+    srcs = sources()
+    objs = [os.path.join(objdir, os.path.basename(f)[:-3] + ".o") for f in srcs]
+    with ThreadPoolExecutor(max_workers=min(len(srcs), os.cpu_count() or 4)) as ex:
+        results = list(ex.map(_compile, srcs, objs))
+    logs = []
+    for f, r in zip(srcs, results):
+        logs.append(f"== {os.path.basename(f)}\n" + r.stdout + r.stderr)
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed on {f}:\n" + r.stdout + r.stderr)
+    link = [nvcc(), "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", SO + ".tmp", *objs]
+    r = subprocess.run(link, capture_output=True, text=True)
     if r.returncode != 0:
-        raise RuntimeError("nvcc failed:\n" + r.stdout + r.stderr)
+        raise RuntimeError("link failed:\n" + r.stdout + r.stderr)
     os.replace(SO + ".tmp", SO)
     log = os.path.join(PKG, "build.log")
     with open(log, "w") as f:
-        f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
+        f.write(" ".join([nvcc(), *NVCC_FLAGS, "-c"]) + "\n" + "".join(logs))
     if verbose:
-        print(r.stdout + r.stderr)
+        print("".join(logs))
     return SO
 
 

@@ -89,7 +89,21 @@ struct ScatterArgs {
     // contains v^1, which the greedy would reject; pruned entries are counted
     const uint32_t *claimed = nullptr;
     unsigned long long *pruned = nullptr;
+    // hash-range shards (multi-GPU, not split): level-1 digit d belongs to rank
+    // o = d * dest_g >> 8, whose digits start at first(o) = ceil(256 o / dest_g); region of
+    // (length s, digit d) = (o * G + s) * nb_pad + d - first(o), nb_pad = ceil(256 / dest_g),
+    // so every rank's regions of all G lengths are one contiguous slice of out/fill (equal
+    // split sizes for the all-to-all).  dest_g = 1, nb_pad = 256: the single-GPU [G][256].
+    uint32_t dest_g = 1, nb_pad = 256;
 };
+// region index of (segment s of G, level-1 digit d) under ScatterArgs' shard layout
+__host__ __device__ __forceinline__ uint64_t shard_region(uint32_t s, uint32_t G, uint32_t d,
+                                                          uint32_t dest_g, uint32_t nb_pad)
+{
+    const uint32_t o = (d * dest_g) >> 8;
+    const uint32_t first = (o * 256u + dest_g - 1u) / dest_g;
+    return ((uint64_t)o * G + s) * nb_pad + (d - first);
+}
 lasagna_status launch_scatter_table(const ScatterArgs &a, cudaStream_t s);
 struct RefineArgs {
     const uint64_t *in;
@@ -103,7 +117,12 @@ struct RefineArgs {
     uint32_t vbits;
     uint32_t *overflow;
     bool split;
+    // multi-GPU: region r of the output gathers the input regions k * src_stride + r of
+    // n_src senders (1 <= n_src <= MAX_REFINE_SRC); single GPU: n_src = 1
+    uint32_t n_src = 1;
+    uint64_t src_stride = 0;
 };
+constexpr uint32_t MAX_REFINE_SRC = 64;
 lasagna_status launch_refine(const RefineArgs &a, uint64_t n_regions, cudaStream_t s);
 struct BucketJoinArgs {
     JoinArgs j;               // packed, L, stride, l, vbits, pairs, cap, count, false_matches
@@ -131,6 +150,38 @@ struct GreedyBufs {
 };
 lasagna_status greedy_length(GreedyBufs &g, uint8_t l, uint32_t *succ, uint8_t *olen,
                              cudaStream_t s);
+
+// ---- a6/a7, two launches per length (greedy_rounds.cu), single GPU or sharded over ranks
+constexpr uint32_t MAX_PEERS = 8;
+// per-rank u64 counters (PeerRank::ctr, PC_N words, zeroed once per call)
+enum { PC_RING = 0,    // [3] live-list counts of the round phases
+       PC_BOOK = 3,    // [4] accepted, sum |P_l|, max |P_l|, max rounds (as GreedyBufs::book)
+       PC_WORK = 7,    // sum over rounds of the pairs visited
+       PC_EPOCH = 8,   // last proposal epoch used (0: none)
+       PC_ARRIVE = 9, PC_GEN = 10,   // barrier of one rank's blocks
+       PC_XARRIVE = 11, PC_XCOUNT = 12, // cross-rank barrier: arrivals, barriers completed
+       PC_ROUNDS = 13, PC_TAILIN = 14, PC_N = 16 };
+struct PeerRank {
+    unsigned long long *pool, *pool2; // this rank's candidate pairs (pool) and scratch list
+    const unsigned long long *in_count; // device: pairs in pool (the join's counter)
+    unsigned long long *ctr;          // PC_N words
+    unsigned long long *best;         // owned slice of the epoch-tagged proposals
+    uint32_t *claimed;                // owned slice of the claimed bitmap
+    uint32_t *succ;                   // owned slices of the outputs
+    uint8_t *olen;
+    unsigned long long *tail;         // rank 0: gathered survivors (GR_TAIL_MAX pairs)
+};
+struct GreedyPeers {
+    PeerRank r[MAX_PEERS];
+    uint32_t g = 1;           // ranks
+    uint64_t slice = 0;       // read ends per rank (multiple of 32): end x on rank x / slice
+    unsigned long long cap = 0; // pool capacity
+    uint32_t rank0 = 0;       // first rank this launch runs (multi-GPU: my rank)
+    uint32_t nranks_here = 1; // ranks this launch runs (> 1: one-GPU test of the protocol)
+    uint32_t bpr = 0;         // blocks per rank (0: the co-resident maximum / 2)
+};
+constexpr uint32_t GR_TAIL_CAP = 4096;
+lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t s);
 lasagna_status launch_gather_pairs(const uint64_t *order, uint64_t off, uint64_t m,
                                    const uint32_t *pa, const uint32_t *pb,
                                    unsigned long long *pool, unsigned long long *cnt,

@@ -127,7 +127,31 @@ struct Layout {
 constexpr size_t CTR_BYTES = 4096 * 4 + 1024;
 // u64 counters after the sort tile counters
 enum { CTR_POOL = 0, CTR_FALSE = 1, CTR_POOL2 = 2, CTR_OVERFLOW = 3, CTR_BOOK = 4, CTR_FOUND = 8,
-       CTR_POOL3 = 9, CTR_WORK = 10, CTR_PRUNED = 11, CTR64_N = 12 };
+       CTR_POOL3 = 9, CTR_WORK = 10, CTR_PRUNED = 11, CTR_PEER = 16, CTR64_N = CTR_PEER + PC_N };
+
+// The greedy: two launches per length (greedy_rounds.cu); LASAGNA_GREEDY=old (A/B only) runs
+// the seven-launch form (greedy.cu)
+static bool old_greedy() { return env_flag("LASAGNA_GREEDY", 'o'); }
+
+// a one-rank GreedyPeers over a call's buffers
+static GreedyPeers single_peers(const GreedyBufs &gb, unsigned long long *ctr_peer, uint32_t *succ,
+                                uint8_t *olen, uint64_t V)
+{
+    GreedyPeers p;
+    p.r[0].pool = gb.pool;
+    p.r[0].pool2 = gb.pool2;
+    p.r[0].in_count = gb.cnt;
+    p.r[0].ctr = ctr_peer;
+    p.r[0].best = gb.best;
+    p.r[0].claimed = gb.claimed;
+    p.r[0].succ = succ;
+    p.r[0].olen = olen;
+    p.r[0].tail = nullptr;
+    p.g = 1;
+    p.slice = V;
+    p.cap = gb.cap;
+    return p;
+}
 
 static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
 {
@@ -522,10 +546,11 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * g.n_buckets;
         bj.half_cap = g.half;
         bj.n_buckets = g.n_buckets;
-        // one warp per bucket (warpjoin.cu) when a half fits a warp's slice, else block
-        // windows (partition.cu); LASAGNA_JOIN=bulk (A/B only) forces the block windows
-        rc = (env_flag("LASAGNA_JOIN", 'b') || !warp_join_fits(bj)) ? launch_bucket_join(bj, r.s)
-                                                                    : launch_warp_join(bj, r.s);
+        // block windows (partition.cu); LASAGNA_JOIN=warp (A/B only): one warp per bucket
+        // (warpjoin.cu) when a half fits a warp's slice — measured slower at cfg3 (31.9 vs
+        // 17.1 ms per step)
+        rc = (env_flag("LASAGNA_JOIN", 'w') && warp_join_fits(bj)) ? launch_warp_join(bj, r.s)
+                                                                   : launch_bucket_join(bj, r.s);
     } else {
         rc = launch_join(ja, r.s);
     }
@@ -744,6 +769,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     gb.claimed = claimed;
     gb.cap = cap;
     gb.epoch = 1;
+    const GreedyPeers peers = single_peers(gb, r.ctr64 + CTR_PEER, succ, olen, g.V);
 
   for (int attempt = 0; attempt < 2; ++attempt) {
     r.bucketed = attempt == 0 && use_bucketed(g);
@@ -787,7 +813,9 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
             ++st.search_launches;
             if ((rc = tm.start(PH_GREEDY)) != LASAGNA_OK) return rc;
-            if ((rc = greedy_length(gb, (uint8_t)l, succ, olen, s)) != LASAGNA_OK) return rc;
+            if ((rc = old_greedy() ? greedy_length(gb, (uint8_t)l, succ, olen, s)
+                                   : greedy_length_peers(peers, (uint8_t)l, s)) != LASAGNA_OK)
+                return rc;
             if ((rc = tm.stop()) != LASAGNA_OK) return rc;
         }
     }
@@ -804,7 +832,8 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         }
     }
     if (r.bucketed && h[CTR_OVERFLOW]) continue; // a slack region overflowed: exact path
-    const unsigned long long *book = h + CTR_BOOK;
+    const unsigned long long *book = old_greedy() ? h + CTR_BOOK : h + CTR_PEER + PC_BOOK;
+    const unsigned long long work = old_greedy() ? h[CTR_WORK] : h[CTR_PEER + PC_WORK];
     if (book[2] > cap) {
         const uint64_t need = book[2] + book[2] / 4;
         *workspace_bytes = layout(g, G, need, true).total;
@@ -817,7 +846,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         st.n_greedy = book[0];
         st.rounds_max = (uint32_t)book[3];
         st.fp_false_matches = h[CTR_FALSE];
-        st.greedy_pair_rounds = h[CTR_WORK];
+        st.greedy_pair_rounds = work;
         st.pruned_entries = h[CTR_PRUNED];
         st.partition_levels = r.bucketed ? g.P : 0;
         if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
@@ -1098,6 +1127,7 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
     gb.cap = c1;
     gb.epoch = 1;
     LSG_CUDA(cudaMemsetAsync(gb.best, 0, V * 8, s));
+    const GreedyPeers peers = single_peers(gb, ctr64 + CTR_PEER, succ, olen, V);
     uint64_t pos = 0;
     for (int d = 0; d < 256; ++d) { // digit d = 255 - l: longest lengths first
         const uint64_t m = h[d];
@@ -1105,11 +1135,14 @@ extern "C" lasagna_status lasagna_greedy_pairs(uint64_t n, const uint8_t *pl, co
         const uint8_t l = (uint8_t)(255 - d);
         if ((rc = launch_gather_pairs(keys[which], pos, m, pa, pb, gb.pool, gb.cnt, s)) != LASAGNA_OK)
             return rc;
-        if ((rc = greedy_length(gb, l, succ, olen, s)) != LASAGNA_OK) return rc;
+        if ((rc = old_greedy() ? greedy_length(gb, l, succ, olen, s)
+                               : greedy_length_peers(peers, l, s)) != LASAGNA_OK)
+            return rc;
         pos += m;
     }
     unsigned long long bk[4];
-    LSG_CUDA(cudaMemcpyAsync(bk, gb.book, sizeof bk, cudaMemcpyDeviceToHost, s));
+    LSG_CUDA(cudaMemcpyAsync(bk, old_greedy() ? gb.book : ctr64 + CTR_PEER + PC_BOOK, sizeof bk,
+                             cudaMemcpyDeviceToHost, s));
     LSG_CUDA(cudaStreamSynchronize(s));
     if (rounds) *rounds = (uint32_t)bk[3];
     return LASAGNA_OK;

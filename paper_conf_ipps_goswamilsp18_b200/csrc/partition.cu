@@ -318,29 +318,29 @@ scatter_table_kernel(ScatterArgs a)
             // ---- partition round for lengths lfirst .. lfirst + kc - 1
             __syncthreads();
             uint32_t c[BPT], bs[BPT], sum = 0;
+            uint64_t rg[BPT];
 #pragma unroll
             for (int b = 0; b < BPT; ++b) {
                 const uint32_t bin = threadIdx.x * BPT + b;
                 c[b] = cnt[bin];
                 cnt[bin] = 0;
                 const uint32_t q = bin / NBL;
-                bs[b] = (c[b] && q < kc)
-                            ? atomicAdd(&a.fill[(uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL], c[b])
-                            : 0u;
+                rg[b] = SPLIT ? (uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL
+                              : shard_region(lfirst - a.l_lo + q, a.l_hi - a.l_lo + 1u, bin % NBL,
+                                             a.dest_g, a.nb_pad);
+                bs[b] = (c[b] && q < kc) ? atomicAdd(&a.fill[rg[b]], c[b]) : 0u;
                 sum += c[b];
             }
             uint32_t run = block_scan<SC_THREADS>(sum, wsum);
 #pragma unroll
             for (int b = 0; b < BPT; ++b) {
                 const uint32_t bin = threadIdx.x * BPT + b;
-                const uint32_t q = bin / NBL;
                 lstart[bin] = run;
                 if ((uint64_t)bs[b] + c[b] > a.cap) {
                     gofs[bin] = -1;
                     *a.overflow = 1u;
                 } else {
-                    gofs[bin] = (long long)(((uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL) * a.cap +
-                                            bs[b]) - (long long)run;
+                    gofs[bin] = (long long)(rg[b] * a.cap + bs[b]) - (long long)run;
                 }
                 run += c[b];
             }
@@ -423,10 +423,21 @@ refine_kernel(RefineArgs a)
         else return d;
     };
     const uint64_t r = blockIdx.x;
-    const uint32_t fill = a.fill_in[r];
-    const uint64_t count = min64(fill, a.cap_in);
-    const uint64_t *src = a.in + r * a.cap_in;
-    const uint32_t ntiles = (uint32_t)ceil_div(count, RF_TILE);
+    // the region's entries: n_src source segments (multi-GPU: one per sending rank), region
+    // k * src_stride + r of `in`, streamed as one sequence of tiles
+    __shared__ uint32_t stile[MAX_REFINE_SRC + 1];
+    __shared__ uint64_t scount[MAX_REFINE_SRC];
+    if (threadIdx.x == 0) {
+        uint32_t acc = 0;
+        for (uint32_t k = 0; k < a.n_src; ++k) {
+            const uint32_t f = a.fill_in[k * a.src_stride + r];
+            if (f > a.cap_in) *a.overflow = 1u;
+            scount[k] = min64(f, a.cap_in);
+            stile[k] = acc;
+            acc += (uint32_t)ceil_div(scount[k], RF_TILE);
+        }
+        stile[a.n_src] = acc;
+    }
     if (threadIdx.x < NBMAX) cnt[threadIdx.x] = 0, running[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
         mbar_init(&mbar[0], 1);
@@ -434,21 +445,35 @@ refine_kernel(RefineArgs a)
         fence_mbar_init();
     }
     __syncthreads();
-    // bytes of tile t (rounded up to 16: the region capacity is even, so the rounding stays
-    // inside the region)
-    auto tile_bytes = [&](uint32_t t) {
-        const uint64_t m = min64(RF_TILE, count - (uint64_t)t * RF_TILE);
-        return (uint32_t)(((m * 8) + 15) & ~15ull);
+    const uint32_t ntiles = stile[a.n_src];
+    // source segment of tile t, and its first entry / length inside that segment
+    auto tile_src = [&](uint32_t t, const uint64_t **p, uint32_t *m) {
+        uint32_t k = 0;
+        while (t >= stile[k + 1]) ++k;
+        const uint64_t t0 = (uint64_t)(t - stile[k]) * RF_TILE;
+        *p = a.in + ((uint64_t)k * a.src_stride + r) * a.cap_in + t0;
+        *m = (uint32_t)min64(RF_TILE, scount[k] - t0);
     };
-    if (threadIdx.x == 0 && ntiles) bulk_load(inb, src, tile_bytes(0), &mbar[0]);
+    // bytes of a tile of m entries (rounded up to 16: the region capacity is even, so the
+    // rounding stays inside the region)
+    auto tile_bytes = [](uint32_t m) { return (uint32_t)((((uint64_t)m * 8) + 15) & ~15ull); };
+    if (threadIdx.x == 0 && ntiles) {
+        const uint64_t *p;
+        uint32_t m;
+        tile_src(0, &p, &m);
+        bulk_load(inb, p, tile_bytes(m), &mbar[0]);
+    }
     for (uint32_t t = 0; t < ntiles; ++t) {
         const uint32_t bsel = t & 1;
-        const uint64_t t0 = (uint64_t)t * RF_TILE;
-        const uint32_t m = (uint32_t)min64(RF_TILE, count - t0);
+        const uint64_t *pcur;
+        uint32_t m;
+        tile_src(t, &pcur, &m);
         if (threadIdx.x == 0 && t + 1 < ntiles) {
+            const uint64_t *p;
+            uint32_t mn;
+            tile_src(t + 1, &p, &mn);
             fence_proxy_async();
-            bulk_load(inb + (bsel ^ 1) * RF_TILE, src + t0 + RF_TILE, tile_bytes(t + 1),
-                      &mbar[bsel ^ 1]);
+            bulk_load(inb + (bsel ^ 1) * RF_TILE, p, tile_bytes(mn), &mbar[bsel ^ 1]);
         }
         mbar_wait(&mbar[bsel], (t >> 1) & 1);
         const uint64_t *tin = inb + bsel * RF_TILE;
@@ -500,13 +525,13 @@ refine_kernel(RefineArgs a)
         a.fill_out[r * nb + threadIdx.x] = running[threadIdx.x];
         if (running[threadIdx.x] > a.cap_out) *a.overflow = 1u;
     }
-    if (threadIdx.x == 0 && fill > a.cap_in) *a.overflow = 1u;
 }
 
 lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStream_t s)
 {
     if (n_regions == 0) return LASAGNA_OK;
     if (args.dbits < 1 || args.dbits > 8) return LASAGNA_EINVAL;
+    if (args.n_src < 1 || args.n_src > MAX_REFINE_SRC) return LASAGNA_EINVAL;
     // tile of 16 keys per thread (one 512-thread CTA per SM, measured faster than 8 keys at
     // two CTAs per SM: 22 vs 30 ms at cfg3); LASAGNA_RF_KPT=8 selects the smaller tile
     static const int kpt = [] {

@@ -694,9 +694,14 @@ def test_greedy_graph_extreme_lengths(lz, L, l_min, n, G, p_err):
     import torch
     reads = readgen.reads(7, G, n, L, p_err)
     esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
+    P = oracle.overlaps(reads, l_min)
     for src in (torch.from_numpy(reads).cuda(), torch.from_numpy(reads).pin_memory()):
         r = lz.greedy_graph(lz.load_reads(src), n, L, l_min)
-        assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc, (r.stats, m, acc)
+        # more than 64 lengths run in several groups: later groups are pruned (f1), so the
+        # pairs found are the live ones (tests/_util.py pruning_expectations)
+        G = r.stats["lengths_per_pass"]
+        found = pruning_expectations(L, l_min, G, P, eolen)[0] if r.stats["bucketed"] else m
+        assert r.stats["n_pairs"] == found and r.stats["n_greedy"] == acc, (r.stats, found, acc)
         assert np.array_equal(_np(r.succ, np.uint32), esucc)
         assert np.array_equal(_np(r.olen, np.uint8), eolen)
     pl, pa, pb = lz.overlaps(lz.load_reads(torch.from_numpy(reads).cuda()), n, L, l_min)
