@@ -518,6 +518,8 @@ def main() -> None:
                     help="process-group backend of the multi-GPU path (gloo: ranks may share a GPU)")
     ap.add_argument("--force-dist", action="store_true",
                     help="run the sharded multi-GPU path even with one rank")
+    ap.add_argument("--dist-path", default="fast", choices=["fast", "exact"],
+                    help="multi-GPU path: bucketed kernels + sharded greedy, or the exact LSD path")
     ap.add_argument("--no-verify-lpp1", action="store_true",
                     help="cfg4/cfg5: skip the one-length-per-pass equality run")
     args = ap.parse_args()

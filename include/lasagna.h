@@ -7,7 +7,8 @@
  * Conventions (every entry point):
  *   - extern "C"; plain pointers and sizes only.  `stream` is a cudaStream_t (NULL = legacy
  *     default stream) on the CURRENT device; all device work is stream-ordered on it.
- *   - The caller owns every buffer.  The library allocates no device memory: scratch comes
+ *   - The caller owns every buffer.  The library allocates no device memory (except
+ *     lasagna_peer_alloc, the IPC-shareable buffers of the multi-GPU greedy): scratch comes
  *     from a caller-provided workspace whose size the caller obtains first (workspace == NULL
  *     -> *workspace_bytes is set and nothing runs).  Device pointers must be 256-byte aligned
  *     (any torch CUDA tensor's data_ptr() is).
@@ -272,6 +273,107 @@ LASAGNA_API lasagna_status lasagna_join(const uint64_t *keys, uint64_t count,
                                         const uint64_t *packed_all, uint64_t n_total, uint32_t L,
                                         uint32_t l, uint64_t *pairs, uint64_t capacity,
                                         uint64_t *counters, void *stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Sharded FAST path (the multi-GPU driver's default).  g = world ranks,
+ * one process per GPU.  Rank r holds the reads [r n_pad, min(n_total, (r+1) n_pad)) with
+ * n_pad = lasagna_shard_geom.n_pad (ceil(n_total / g) rounded up to 16), and OWNS the read ends
+ * [r slice, (r+1) slice), slice = 2 n_pad, for the greedy.  The level-1 digit d (top 8 bits of
+ * the mixed canonical fingerprint) belongs to rank o = floor(d g / 256): the hash-range
+ * partition of P:L333 (the paper's shuffle P:L204, re-keyed by fingerprint).  Per length group
+ * [l_lo, l_hi] (G <= 64 lengths):
+ *   1. lasagna_shard_scatter: keys of the rank's reads into `send`, [g][G][nb_pad][cap1] u64
+ *      (+ fills [g][G][nb_pad] u32): the slice for rank o is contiguous and equally sized;
+ *   2. the caller exchanges send -> recv and send_fill -> recv_fill with two all-to-alls of
+ *      EQUAL split sizes (G nb_pad cap1 keys, G nb_pad fills per rank pair): no count
+ *      exchange, no host synchronisation;
+ *   3. lasagna_shard_partition: the remaining radix levels over the g received slices;
+ *   4. per length l (descending): lasagna_shard_join into the rank's pair pool, then
+ *      lasagna_greedy_shard_length.
+ * counters: device u64[4], zeroed by the caller once per call: [0] nonzero = a slack region
+ * overflowed (the result is incomplete: rerun on the exact path), [1] entries pruned (claimed
+ * ends, f1), [2] reserved, [3] rejected fingerprint matches.  All calls are asynchronous.
+ */
+typedef struct {
+    uint32_t levels;       /* MSD partition levels (2 or 3)                                  */
+    uint32_t last_bits;    /* bits of the last level                                        */
+    uint32_t nb_pad;       /* level-1 digits per rank, padded: ceil(256 / g)                 */
+    uint32_t vbits;        /* vertex-id bits of a key                                        */
+    uint64_t n_pad;        /* reads per rank                                                 */
+    uint64_t slice;        /* read ends owned per rank (2 n_pad, a multiple of 32)           */
+    uint64_t cap1;         /* level-1 region capacity (keys)                                 */
+    uint64_t send_entries; /* keys of send (= of recv) PER LENGTH: g nb_pad cap1             */
+    uint64_t fill_words;   /* u32 fills of send_fill (= of recv_fill) PER LENGTH: g nb_pad    */
+    uint64_t part_bytes;   /* workspace of lasagna_shard_partition for ONE length            */
+    uint64_t buckets;      /* final buckets per length on one rank                           */
+} lasagna_shard_geom;
+
+LASAGNA_API lasagna_status lasagna_shard_geometry(uint64_t n_total, uint32_t world, uint32_t L,
+                                                  uint32_t l_min, lasagna_shard_geom *out);
+/* workspace bytes of lasagna_shard_partition for a group of `lengths` lengths */
+LASAGNA_API lasagna_status lasagna_shard_part_bytes(uint64_t n_total, uint32_t world, uint32_t L,
+                                                    uint32_t l_min, uint32_t lengths, size_t *bytes);
+/* packed_local: the rank's packed rows (device); read_offset = r n_pad; claimed: the rank's
+ * slice of the claimed-end bitmap (device, slice/32 words) or NULL (no pruning). */
+LASAGNA_API lasagna_status lasagna_shard_scatter(const uint64_t *packed_local, uint64_t n_local,
+                                                 uint64_t read_offset, uint64_t n_total,
+                                                 uint32_t world, uint32_t L, uint32_t l_min,
+                                                 uint32_t l_lo, uint32_t l_hi,
+                                                 const uint32_t *claimed, uint64_t *send,
+                                                 uint32_t *send_fill, uint64_t *counters,
+                                                 void *stream);
+/* recv/recv_fill: the g received slices, sender-major; part: lasagna_shard_part_bytes bytes. */
+LASAGNA_API lasagna_status lasagna_shard_partition(const uint64_t *recv, const uint32_t *recv_fill,
+                                                   uint64_t n_total, uint32_t world, uint32_t L,
+                                                   uint32_t l_min, uint32_t l_lo, uint32_t l_hi,
+                                                   void *part, uint64_t *counters, void *stream);
+/* a5 of length l over this rank's buckets: verified pairs (a << 32) | b, a < b, written to
+ * pool (device u64[capacity]); *pool_count (device u64) is zeroed, then counts every pair found
+ * (may exceed capacity: overflow).  packed_all: the packed rows of all n_total reads. */
+LASAGNA_API lasagna_status lasagna_shard_join(const void *part, uint64_t n_total, uint32_t world,
+                                              uint32_t L, uint32_t l_min, uint32_t l_lo,
+                                              uint32_t l_hi, uint32_t l,
+                                              const uint64_t *packed_all, uint64_t *pool,
+                                              uint64_t capacity, uint64_t *pool_count,
+                                              uint64_t *counters, void *stream);
+
+/* a6/a7 sharded (the reduce step P:L206-210): the greedy of length l over the
+ * pairs every rank's pool holds, each rank owning best/claimed/succ/olen of its slice of read
+ * ends.  ranks[q] describes rank q with pointers VALID IN THIS PROCESS (peer memory opened with
+ * lasagna_peer_open: NVLink loads, stores and atomics); the ranks meet at device-side barriers
+ * in their ctr words, so every rank must make the same sequence of calls.  rank = -1 runs all
+ * `world` ranks in one launch (one GPU: a test of the protocol).  Result: the single-GPU
+ * greedy over the union of the pools, bit for bit.
+ *   pool, pool2   device u64[capacity]: the rank's pairs (count *pool_count) and scratch
+ *   ctr           device u64[16], zeroed before the call's first length: [3] pairs accepted,
+ *                 [4] sum of |P_l|, [5] max |P_l|, [6] max rounds, [7] pairs visited
+ *   best          device u64[slice], zeroed before the first length
+ *   claimed       device u32[slice/32], zeroed before the first length (bit x: end x claimed)
+ *   succ, olen    device u32[slice] (LASAGNA_NONE), u8[slice] (0) initialised by the caller
+ *   tail          rank 0: device u64[4096] (the gathered survivors); others may be NULL
+ * world = 1: slice is ignored (one rank owns every end). */
+typedef struct {
+    uint64_t *pool, *pool2;
+    uint64_t *pool_count; /* the pair count; the rounds reuse it as a list counter */
+    uint64_t *ctr;
+    uint64_t *best;
+    uint32_t *claimed;
+    uint32_t *succ;
+    uint8_t *olen;
+    uint64_t *tail;
+} lasagna_greedy_rank;
+LASAGNA_API lasagna_status lasagna_greedy_shard_length(const lasagna_greedy_rank *ranks,
+                                                       uint32_t world, int32_t rank,
+                                                       uint64_t slice, uint64_t capacity,
+                                                       uint32_t l, void *stream);
+
+/* Peer memory (CUDA IPC): the one place the library allocates device memory.  alloc returns a
+ * device buffer and its 64-byte IPC handle; another process opens it with peer_open (the
+ * device pointer is valid there until peer_close); free releases the owner's buffer. */
+LASAGNA_API lasagna_status lasagna_peer_alloc(size_t bytes, void **dev_ptr, void *handle);
+LASAGNA_API lasagna_status lasagna_peer_free(void *dev_ptr);
+LASAGNA_API lasagna_status lasagna_peer_open(const void *handle, void **dev_ptr);
+LASAGNA_API lasagna_status lasagna_peer_close(void *dev_ptr);
 
 #ifdef __cplusplus
 }

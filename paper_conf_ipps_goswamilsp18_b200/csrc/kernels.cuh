@@ -160,10 +160,10 @@ enum { PC_RING = 0,    // [3] live-list counts of the round phases
        PC_EPOCH = 8,   // last proposal epoch used (0: none)
        PC_ARRIVE = 9, PC_GEN = 10,   // barrier of one rank's blocks
        PC_XARRIVE = 11, PC_XCOUNT = 12, // cross-rank barrier: arrivals, barriers completed
-       PC_ROUNDS = 13, PC_TAILIN = 14, PC_N = 16 };
+       PC_TAILEPOCH = 13, PC_TAILIN = 14, PC_N = 16 }; // rank 0's last tail epoch; survivors
 struct PeerRank {
     unsigned long long *pool, *pool2; // this rank's candidate pairs (pool) and scratch list
-    const unsigned long long *in_count; // device: pairs in pool (the join's counter)
+    unsigned long long *in_count;     // device: pairs in pool (the join's counter; ring slot 0)
     unsigned long long *ctr;          // PC_N words
     unsigned long long *best;         // owned slice of the epoch-tagged proposals
     uint32_t *claimed;                // owned slice of the claimed bitmap
@@ -178,7 +178,7 @@ struct GreedyPeers {
     unsigned long long cap = 0; // pool capacity
     uint32_t rank0 = 0;       // first rank this launch runs (multi-GPU: my rank)
     uint32_t nranks_here = 1; // ranks this launch runs (> 1: one-GPU test of the protocol)
-    uint32_t bpr = 0;         // blocks per rank (0: the co-resident maximum / 2)
+    uint32_t bpr = 0;         // blocks per rank (0: sized from cap)
 };
 constexpr uint32_t GR_TAIL_CAP = 4096;
 lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t s);

@@ -1281,3 +1281,362 @@ lasagna_status lasagna_join(const uint64_t *keys, uint64_t count, const uint64_t
 }
 
 } // extern "C"
+
+// ==================================================================== sharded fast path
+// The multi-GPU driver on the bucketed kernels (P:L204 shuffle re-keyed by
+// fingerprint, the paper's future work P:L333).  Rank r holds reads [r n_pad, (r+1) n_pad).
+//   lasagna_shard_scatter    a1..a3 + level 1 of its reads, regions in hash-range shard order
+//                            (rank o owns level-1 digits [ceil(256 o / g), ceil(256 (o+1) / g)))
+//   (caller) all-to-all      equal split sizes: rank o's regions of the G lengths are one
+//                            contiguous slice of every sender's buffer
+//   lasagna_shard_partition  the remaining levels over the g received slices (multi-source refine)
+//   lasagna_shard_join       a5 of one length over this rank's buckets
+//   lasagna_greedy_shard_length  a6/a7 over peer memory (greedy_rounds.cu)
+namespace lsg {
+
+struct ShardGeom {
+    Geometry g; // geometry of the n_total-read set, at least two levels
+    uint32_t world, nb_pad;
+    uint64_t n_pad, slice, cap1;
+};
+
+static ShardGeom shard_geom(uint64_t n_total, uint32_t world, uint32_t L, uint32_t l_min)
+{
+    ShardGeom s;
+    s.g = geometry(n_total, L, l_min);
+    if (s.g.P < 2) { // one level would leave nothing to refine after the exchange
+        s.g.P = 2;
+        s.g.dlast = 8;
+        s.g.T = 16;
+        s.g.n_buckets = 1ull << 16;
+        s.g.half = region_cap((double)s.g.N / (double)(2 * s.g.n_buckets));
+    }
+    s.world = world;
+    s.nb_pad = (256 + world - 1) / world;
+    s.n_pad = (ceil_div(n_total, world) + 15) & ~15ull; // a rank's ends: whole bitmap words
+    s.slice = 2 * s.n_pad;
+    s.cap1 = region_cap(2.0 * (double)s.n_pad / 256.0);
+    return s;
+}
+
+struct ShardPart {
+    size_t out2, fill2, out3, fill3, total;
+};
+
+// workspace of lasagna_shard_partition for G lengths: R = G nb_pad level-1 regions
+static ShardPart shard_part_layout(const ShardGeom &sg, uint32_t G)
+{
+    const Geometry &g = sg.g;
+    const uint64_t R = (uint64_t)G * sg.nb_pad;
+    ShardPart p;
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        size_t o = off;
+        off += align256(bytes);
+        return o;
+    };
+    if (g.P == 2) {
+        p.out2 = take(R * 256 * 2 * g.half * 8);
+        p.fill2 = take(R * 512 * 4);
+        p.out3 = p.fill3 = 0;
+    } else {
+        p.out2 = take(R * 256 * g.cap2 * 8);
+        p.fill2 = take(R * 256 * 4);
+        const uint64_t nb3 = 1ull << g.dlast;
+        p.out3 = take(R * 256 * nb3 * 2 * g.half * 8);
+        p.fill3 = take(R * 256 * nb3 * 2 * 4);
+    }
+    p.total = off;
+    return p;
+}
+
+static lasagna_status shard_check(uint64_t n_total, uint32_t world, uint32_t L, uint32_t l_min,
+                                  uint32_t l_lo, uint32_t l_hi)
+{
+    lasagna_status rc = check_shape(n_total, L, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (world < 1 || world > MAX_PEERS) {
+        set_error("world=%u out of range [1, %u]", world, MAX_PEERS);
+        return LASAGNA_EINVAL;
+    }
+    if (l_lo < l_min || l_hi < l_lo || l_hi >= L || l_hi - l_lo + 1 > 64) {
+        set_error("bad length group [%u, %u]", l_lo, l_hi);
+        return LASAGNA_EINVAL;
+    }
+    return LASAGNA_OK;
+}
+
+} // namespace lsg
+
+extern "C" {
+
+lasagna_status lasagna_shard_geometry(uint64_t n_total, uint32_t world, uint32_t L, uint32_t l_min,
+                                      lasagna_shard_geom *out)
+{
+    g_err[0] = 0;
+    lasagna_status rc = shard_check(n_total, world, L, l_min, l_min, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (!out) {
+        set_error("NULL output");
+        return LASAGNA_EINVAL;
+    }
+    const ShardGeom sg = shard_geom(n_total, world, L, l_min);
+    out->levels = sg.g.P;
+    out->last_bits = sg.g.dlast;
+    out->nb_pad = sg.nb_pad;
+    out->vbits = sg.g.vbits;
+    out->n_pad = sg.n_pad;
+    out->slice = sg.slice;
+    out->cap1 = sg.cap1;
+    out->send_entries = (uint64_t)world * sg.nb_pad * sg.cap1;
+    out->fill_words = (uint64_t)world * sg.nb_pad;
+    out->part_bytes = shard_part_layout(sg, 1).total;
+    out->buckets = (uint64_t)sg.nb_pad * 256 * (sg.g.P == 3 ? (1ull << sg.g.dlast) : 1ull);
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_shard_part_bytes(uint64_t n_total, uint32_t world, uint32_t L,
+                                        uint32_t l_min, uint32_t lengths, size_t *bytes)
+{
+    g_err[0] = 0;
+    lasagna_status rc = shard_check(n_total, world, L, l_min, l_min, l_min);
+    if (rc != LASAGNA_OK) return rc;
+    if (!bytes || lengths < 1 || lengths > 64) {
+        set_error("NULL output or lengths out of [1, 64]");
+        return LASAGNA_EINVAL;
+    }
+    *bytes = shard_part_layout(shard_geom(n_total, world, L, l_min), lengths).total;
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_shard_scatter(const uint64_t *packed_local, uint64_t n_local,
+                                     uint64_t read_offset, uint64_t n_total, uint32_t world,
+                                     uint32_t L, uint32_t l_min, uint32_t l_lo, uint32_t l_hi,
+                                     const uint32_t *claimed, uint64_t *send, uint32_t *send_fill,
+                                     uint64_t *counters, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = shard_check(n_total, world, L, l_min, l_lo, l_hi);
+    if (rc != LASAGNA_OK) return rc;
+    const ShardGeom sg = shard_geom(n_total, world, L, l_min);
+    if (read_offset % sg.n_pad || n_local > sg.n_pad || read_offset + n_local > n_total) {
+        set_error("read range [%llu, +%llu) is not a shard of n_pad=%llu", (unsigned long long)read_offset,
+                  (unsigned long long)n_local, (unsigned long long)sg.n_pad);
+        return LASAGNA_EINVAL;
+    }
+    if (!send || !send_fill || !counters || (n_local && !packed_local) || !aligned(send, 16) ||
+        !aligned(counters, 8) || (packed_local && !aligned(packed_local, 16))) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint32_t G = l_hi - l_lo + 1;
+    LSG_CUDA(cudaMemsetAsync(send_fill, 0, (size_t)G * world * sg.nb_pad * 4, s));
+    if (n_local == 0) return LASAGNA_OK;
+    ScatterArgs sa;
+    sa.packed = packed_local;
+    sa.n = n_local;
+    sa.read_offset = read_offset;
+    sa.L = L;
+    sa.stride = stride_for(L);
+    sa.l_lo = l_lo;
+    sa.l_hi = l_hi;
+    sa.vbits = sg.g.vbits;
+    sa.keep = stored_keep(sg.g);
+    sa.out = send;
+    sa.fill = send_fill;
+    sa.split = false;
+    sa.cap = sg.cap1;
+    sa.overflow = reinterpret_cast<uint32_t *>(counters);
+    sa.ascii = nullptr;
+    sa.packed_out = nullptr;
+    sa.first_bad = nullptr;
+    // the caller's bitmap holds this rank's ends [2 read_offset, ...): index it globally
+    sa.claimed = claimed ? claimed - (2 * read_offset) / 32 : nullptr;
+    sa.pruned = reinterpret_cast<unsigned long long *>(counters) + 1;
+    sa.dest_g = world;
+    sa.nb_pad = sg.nb_pad;
+    return launch_scatter_table(sa, s);
+}
+
+lasagna_status lasagna_shard_partition(const uint64_t *recv, const uint32_t *recv_fill,
+                                       uint64_t n_total, uint32_t world, uint32_t L,
+                                       uint32_t l_min, uint32_t l_lo, uint32_t l_hi, void *part,
+                                       uint64_t *counters, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = shard_check(n_total, world, L, l_min, l_lo, l_hi);
+    if (rc != LASAGNA_OK) return rc;
+    if (!recv || !recv_fill || !part || !counters || !aligned(part, 256) || !aligned(recv, 16)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    const ShardGeom sg = shard_geom(n_total, world, L, l_min);
+    const Geometry &g = sg.g;
+    const uint32_t G = l_hi - l_lo + 1;
+    const ShardPart pl = shard_part_layout(sg, G);
+    char *ws = (char *)part;
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t R = (uint64_t)G * sg.nb_pad;
+    RefineArgs ra;
+    ra.in = recv;
+    ra.fill_in = recv_fill;
+    ra.cap_in = sg.cap1;
+    ra.dshift = 56;
+    ra.dbits = 8;
+    ra.out = reinterpret_cast<uint64_t *>(ws + pl.out2);
+    ra.fill_out = reinterpret_cast<uint32_t *>(ws + pl.fill2);
+    ra.cap_out = g.P == 2 ? g.half : g.cap2;
+    ra.vbits = g.vbits;
+    ra.split = g.P == 2;
+    ra.overflow = reinterpret_cast<uint32_t *>(counters);
+    ra.n_src = world;
+    ra.src_stride = R; // sender k's slice for this rank: regions [k R, (k+1) R) of recv
+    if ((rc = launch_refine(ra, R, s)) != LASAGNA_OK) return rc;
+    if (g.P == 3) {
+        ra.in = reinterpret_cast<uint64_t *>(ws + pl.out2);
+        ra.fill_in = reinterpret_cast<uint32_t *>(ws + pl.fill2);
+        ra.cap_in = g.cap2;
+        ra.dshift = 56 - g.dlast;
+        ra.dbits = g.dlast;
+        ra.out = reinterpret_cast<uint64_t *>(ws + pl.out3);
+        ra.fill_out = reinterpret_cast<uint32_t *>(ws + pl.fill3);
+        ra.cap_out = g.half;
+        ra.split = true;
+        ra.n_src = 1;
+        ra.src_stride = 0;
+        if ((rc = launch_refine(ra, R * 256, s)) != LASAGNA_OK) return rc;
+    }
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_shard_join(const void *part, uint64_t n_total, uint32_t world, uint32_t L,
+                                  uint32_t l_min, uint32_t l_lo, uint32_t l_hi, uint32_t l,
+                                  const uint64_t *packed_all, uint64_t *pool, uint64_t capacity,
+                                  uint64_t *pool_count, uint64_t *counters, void *stream)
+{
+    g_err[0] = 0;
+    lasagna_status rc = shard_check(n_total, world, L, l_min, l_lo, l_hi);
+    if (rc != LASAGNA_OK) return rc;
+    if (l < l_lo || l > l_hi) {
+        set_error("length %u outside the group [%u, %u]", l, l_lo, l_hi);
+        return LASAGNA_EINVAL;
+    }
+    if (!part || !packed_all || !pool_count || !counters || (capacity && !pool) ||
+        !aligned(part, 256) || !aligned(packed_all, 16)) {
+        set_error("NULL or misaligned pointer");
+        return LASAGNA_EINVAL;
+    }
+    const ShardGeom sg = shard_geom(n_total, world, L, l_min);
+    const Geometry &g = sg.g;
+    const uint32_t G = l_hi - l_lo + 1;
+    const ShardPart pl = shard_part_layout(sg, G);
+    char *ws = (char *)const_cast<void *>(part);
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t nbk = (uint64_t)sg.nb_pad * 256 * (g.P == 3 ? (1ull << g.dlast) : 1ull);
+    const uint32_t seg = l - l_lo;
+    LSG_CUDA(cudaMemsetAsync(pool_count, 0, 8, s));
+    BucketJoinArgs bj;
+    bj.j.packed = packed_all;
+    bj.j.keys = nullptr;
+    bj.j.N = 0;
+    bj.j.L = L;
+    bj.j.stride = stride_for(L);
+    bj.j.l = l;
+    bj.j.vbits = g.vbits;
+    bj.j.T = g.T;
+    bj.j.pairs = reinterpret_cast<unsigned long long *>(pool);
+    bj.j.cap = capacity;
+    bj.j.count = reinterpret_cast<unsigned long long *>(pool_count);
+    bj.j.false_matches = reinterpret_cast<unsigned long long *>(counters) + 3;
+    bj.j.claimed = nullptr;
+    bj.j.found = nullptr;
+    bj.overflow = reinterpret_cast<uint32_t *>(counters);
+    const size_t ob = g.P == 2 ? pl.out2 : pl.out3, of = g.P == 2 ? pl.fill2 : pl.fill3;
+    bj.buckets = reinterpret_cast<uint64_t *>(ws + ob) + (uint64_t)seg * nbk * 2 * g.half;
+    bj.fills = reinterpret_cast<uint32_t *>(ws + of) + (uint64_t)seg * nbk * 2;
+    bj.half_cap = g.half;
+    bj.n_buckets = nbk;
+    if ((rc = launch_bucket_join(bj, s)) != LASAGNA_OK) return rc;
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_greedy_shard_length(const lasagna_greedy_rank *ranks, uint32_t world,
+                                           int32_t rank, uint64_t slice, uint64_t capacity,
+                                           uint32_t l, void *stream)
+{
+    g_err[0] = 0;
+    if (!ranks || world < 1 || world > MAX_PEERS || rank < -1 || rank >= (int32_t)world ||
+        l < 1 || l > 255 || (world > 1 && (slice == 0 || slice % 32 || capacity < GR_TAIL_CAP))) {
+        set_error("bad rank layout (world=%u rank=%d slice=%llu) or length %u", world, rank,
+                  (unsigned long long)slice, l);
+        return LASAGNA_EINVAL;
+    }
+    GreedyPeers p;
+    for (uint32_t q = 0; q < world; ++q) {
+        const lasagna_greedy_rank &x = ranks[q];
+        p.r[q].pool = reinterpret_cast<unsigned long long *>(x.pool);
+        p.r[q].pool2 = reinterpret_cast<unsigned long long *>(x.pool2);
+        p.r[q].in_count = reinterpret_cast<unsigned long long *>(x.pool_count);
+        p.r[q].ctr = reinterpret_cast<unsigned long long *>(x.ctr);
+        p.r[q].best = reinterpret_cast<unsigned long long *>(x.best);
+        p.r[q].claimed = x.claimed;
+        p.r[q].succ = x.succ;
+        p.r[q].olen = x.olen;
+        p.r[q].tail = reinterpret_cast<unsigned long long *>(x.tail);
+    }
+    p.g = world;
+    p.slice = world > 1 ? slice : ~0ull >> 1;
+    p.cap = capacity;
+    p.rank0 = rank < 0 ? 0 : (uint32_t)rank;
+    p.nranks_here = rank < 0 ? world : 1;
+    return greedy_length_peers(p, (uint8_t)l, (cudaStream_t)stream);
+}
+
+lasagna_status lasagna_peer_alloc(size_t bytes, void **dev_ptr, void *handle)
+{
+    g_err[0] = 0;
+    if (!dev_ptr || !handle || bytes == 0) {
+        set_error("NULL output or zero size");
+        return LASAGNA_EINVAL;
+    }
+    LSG_CUDA(cudaMalloc(dev_ptr, bytes));
+    cudaIpcMemHandle_t h;
+    cudaError_t e = cudaIpcGetMemHandle(&h, *dev_ptr);
+    if (e != cudaSuccess) {
+        cudaFree(*dev_ptr);
+        *dev_ptr = nullptr;
+        return cuda_status(e, "cudaIpcGetMemHandle");
+    }
+    memcpy(handle, &h, sizeof h);
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_peer_free(void *dev_ptr)
+{
+    g_err[0] = 0;
+    LSG_CUDA(cudaFree(dev_ptr));
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_peer_open(const void *handle, void **dev_ptr)
+{
+    g_err[0] = 0;
+    if (!handle || !dev_ptr) {
+        set_error("NULL handle or output");
+        return LASAGNA_EINVAL;
+    }
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof h);
+    LSG_CUDA(cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+    return LASAGNA_OK;
+}
+
+lasagna_status lasagna_peer_close(void *dev_ptr)
+{
+    g_err[0] = 0;
+    LSG_CUDA(cudaIpcCloseMemHandle(dev_ptr));
+    return LASAGNA_OK;
+}
+
+} // extern "C"

@@ -222,6 +222,7 @@ scatter_table_kernel(ScatterArgs a)
     extern __shared__ __align__(16) uint64_t stage[];
     unsigned short *sbin = reinterpret_cast<unsigned short *>(stage + SC_THREADS * KPT);
     __shared__ uint32_t cnt[NBIN], lstart[NBIN + 1], wsum[16];
+    __shared__ uint32_t rbase[SPLIT ? 1 : 256]; // region of (segment 0, digit d); + s * nb_pad
     __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
 
     const uint64_t i = (uint64_t)blockIdx.x * SC_THREADS + threadIdx.x;
@@ -255,6 +256,9 @@ scatter_table_kernel(ScatterArgs a)
         for (int j = 0; j < W; ++j) x[j] = y[j] = 0;
     }
     for (uint32_t t = threadIdx.x; t < NBIN; t += SC_THREADS) cnt[t] = 0;
+    if (!SPLIT)
+        for (uint32_t d = threadIdx.x; d < 256; d += SC_THREADS)
+            rbase[d] = (uint32_t)shard_region(0, a.l_hi - a.l_lo + 1u, d, a.dest_g, a.nb_pad);
     __syncthreads();
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
@@ -326,8 +330,7 @@ scatter_table_kernel(ScatterArgs a)
                 cnt[bin] = 0;
                 const uint32_t q = bin / NBL;
                 rg[b] = SPLIT ? (uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL
-                              : shard_region(lfirst - a.l_lo + q, a.l_hi - a.l_lo + 1u, bin % NBL,
-                                             a.dest_g, a.nb_pad);
+                              : (uint64_t)rbase[bin % NBL] + (uint64_t)(lfirst - a.l_lo + q) * a.nb_pad;
                 bs[b] = (c[b] && q < kc) ? atomicAdd(&a.fill[rg[b]], c[b]) : 0u;
                 sum += c[b];
             }

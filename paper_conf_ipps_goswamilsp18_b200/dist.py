@@ -274,19 +274,321 @@ def greedy_graph(ascii_local: torch.Tensor, n_total: int, L: int, l_min: int, ba
     return succ, olen, stats
 
 
+# ------------------------------------------------------------------------------ fast path
+class _DevView:
+    """A raw device buffer seen by torch (``__cuda_array_interface__``, zero copy): the
+    library-allocated peer arena is initialised and gathered with ordinary tensor ops."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1",
+                                         "data": (ptr, False), "version": 3}
+
+
+def _arena_layout(slice_: int) -> dict:
+    """Byte offsets of one rank's peer arena: best u64[slice], claimed u32[slice/32],
+    succ u32[slice], olen u8[slice], ctr u64[16], tail u64[4096] (256-byte aligned)."""
+    off, lay = 0, {}
+    for name, nbytes in (("best", 8 * slice_), ("claimed", slice_ // 8), ("succ", 4 * slice_),
+                         ("olen", slice_), ("ctr", 16 * 8), ("tail", 4096 * 8)):
+        lay[name] = off
+        off += -(-max(nbytes, 1) // 256) * 256
+    lay["total"] = off
+    return lay
+
+
+class PeerArena:
+    """This rank's IPC-shareable greedy state and the peers' arenas opened in this process."""
+
+    def __init__(self, slice_: int, device, group):
+        self.L = lz.lib()
+        self.lay = _arena_layout(slice_)
+        self.slice = slice_
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.group = group
+        ptr = ctypes.c_void_p()
+        handle = ctypes.create_string_buffer(64)
+        lz._check(self.L.lasagna_peer_alloc(self.lay["total"], ctypes.byref(ptr), handle))
+        self.base = ptr.value
+        self.view = torch.as_tensor(_DevView(self.base, self.lay["total"]), device=device)
+        self.view.zero_()
+        self.tensor("succ", torch.int32).fill_(-1)  # LASAGNA_NONE
+        self.bases = [0] * self.world
+        self.opened = []
+        if self.world > 1:
+            handles = [None] * self.world
+            dist.all_gather_object(handles, handle.raw, group=group)
+            for q, h in enumerate(handles):
+                if q == self.rank:
+                    self.bases[q] = self.base
+                    continue
+                pq = ctypes.c_void_p()
+                lz._check(self.L.lasagna_peer_open(ctypes.create_string_buffer(h, 64),
+                                                   ctypes.byref(pq)))
+                self.bases[q] = pq.value
+                self.opened.append(pq.value)
+        else:
+            self.bases[0] = self.base
+
+    def tensor(self, name: str, dtype) -> torch.Tensor:
+        n = {"best": 8 * self.slice, "claimed": self.slice // 8, "succ": 4 * self.slice,
+             "olen": self.slice, "ctr": 128, "tail": 4096 * 8}[name]
+        return self.view[self.lay[name]:self.lay[name] + n].view(dtype)
+
+    def ptr(self, q: int, name: str) -> int:
+        return self.bases[q] + self.lay[name]
+
+    def close(self):
+        torch.cuda.synchronize()
+        if self.world > 1:
+            dist.barrier(group=self.group)  # no peer still reads or writes my arena
+        for p in self.opened:
+            self.L.lasagna_peer_close(ctypes.c_void_p(p))
+        self.opened = []
+        if self.base:
+            self.view = None
+            self.L.lasagna_peer_free(ctypes.c_void_p(self.base))
+            self.base = 0
+
+
+def shard_geometry(n_total: int, world: int, L: int, l_min: int) -> "lz.ShardGeom":
+    geo = lz.ShardGeom()
+    lz._check(lz.lib().lasagna_shard_geometry(n_total, world, L, l_min, ctypes.byref(geo)))
+    return geo
+
+
+def fast_shard_range(n_total: int, world: int, rank: int):
+    """Reads [lo, hi) of `rank` on the fast path: slices of n_pad = ceil(n/g) rounded up to
+    16 rows (a rank's 2 n_pad read ends fill whole words of the claimed bitmap)."""
+    n_pad = ((-(-n_total // world) if n_total else 0) + 15) // 16 * 16
+    lo = min(n_total, rank * n_pad)
+    return lo, min(n_total, lo + n_pad), n_pad
+
+
+class RegionOverflow(RuntimeError):
+    """A slack region of the sharded partition overflowed: rerun on the exact path."""
+
+
+class _Phases:
+    """CUDA-event pairs per phase on the call's stream, read once at the end (no host sync
+    inside the call)."""
+
+    def __init__(self, on: bool):
+        self.on = on
+        self.recs: list[tuple[str, torch.cuda.Event, torch.cuda.Event]] = []
+        self.launches = {"scatter": 0, "refine": 0, "join": 0, "greedy_lengths": 0}
+
+    def start(self, name):
+        if not self.on:
+            return None
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        self.recs.append((name, a, b))
+        return b
+
+    @staticmethod
+    def stop(b):
+        if b is not None:
+            b.record()
+
+    def totals(self) -> dict:
+        out: dict[str, float] = {}
+        for name, a, b in self.recs:
+            out[name] = out.get(name, 0.0) + a.elapsed_time(b)
+        return out
+
+
+def greedy_graph_fast(ascii_local: torch.Tensor, n_total: int, L: int, l_min: int, group=None,
+                      lengths_per_pass: int = 0, pair_capacity: int | None = None,
+                      timing: bool = False):
+    """Greedy string graph over the ranks of `group` on the bucketed kernels (include/lasagna.h
+    "Sharded FAST path"): per length group one fused scatter of the local reads, two equal-split
+    all-to-alls, the multi-source refine, then per length the join and the sharded greedy over
+    peer memory.  No host synchronisation between the first scatter and the end of the call.
+    Rank r holds reads fast_shard_range(n_total, g, r).  Returns (succ, olen, stats), identical
+    on every rank."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    Lb = lz.lib()
+    dev = ascii_local.device if ascii_local.is_cuda else torch.device("cuda", torch.cuda.current_device())
+    geo = shard_geometry(n_total, world, L, l_min)
+    lo, hi, n_pad = fast_shard_range(n_total, world, rank)
+    assert n_pad == geo.n_pad and ascii_local.shape[0] == hi - lo, (n_pad, geo.n_pad, ascii_local.shape)
+    n_local = hi - lo
+    s = lz._stream(dev)
+    C = _Coll(group, dev)
+    W = lz.words_per_read(L)
+    # 1. packed reads: local pack, all-gather (padded slices) -> every rank verifies any hit
+    buf = torch.zeros((n_pad, W), dtype=torch.int64, device=dev)
+    if n_local:
+        buf[:n_local] = lz.load_reads(ascii_local, device=dev)
+    packed_all = torch.empty(world * n_pad * W, dtype=torch.int64, device=dev)
+    C.all_gather_into_tensor(packed_all, buf.reshape(-1))
+    packed_all = packed_all.view(world * n_pad, W)
+    packed_local = packed_all[lo:lo + n_pad]
+    n_len = L - l_min
+    G = n_len if lengths_per_pass <= 0 else min(lengths_per_pass, n_len)
+    G = min(G, 64)
+    cap = pair_capacity if pair_capacity is not None else max(1 << 20, (2 * n_total) // 8)
+    pool = torch.empty(cap, dtype=torch.int64, device=dev)
+    pool2 = torch.empty(cap, dtype=torch.int64, device=dev)
+    pool_count = torch.zeros(1, dtype=torch.int64, device=dev)
+    counters = torch.zeros(4, dtype=torch.int64, device=dev)
+    arena = PeerArena(int(geo.slice), dev, group)
+    ph = _Phases(timing)
+    try:
+        ranks = (lz.GreedyRank * world)()
+        for q in range(world):
+            ranks[q].ctr = arena.ptr(q, "ctr")
+            ranks[q].best = arena.ptr(q, "best")
+            ranks[q].claimed = arena.ptr(q, "claimed")
+            ranks[q].succ = arena.ptr(q, "succ")
+            ranks[q].olen = arena.ptr(q, "olen")
+            ranks[q].tail = arena.ptr(q, "tail")
+        ranks[rank].pool = pool.data_ptr()
+        ranks[rank].pool2 = pool2.data_ptr()
+        ranks[rank].pool_count = pool_count.data_ptr()
+        claimed_mine = arena.ptr(rank, "claimed")
+        first = True
+        for l_hi in range(L - 1, l_min - 1, -G):
+            l_lo = max(l_min, l_hi - G + 1)
+            Gc = l_hi - l_lo + 1
+            # 2. a1..a3 + level 1 of my reads, regions in shard order (pruned after group 1)
+            send = torch.empty(Gc * geo.send_entries, dtype=torch.int64, device=dev)
+            send_fill = torch.empty(Gc * geo.fill_words, dtype=torch.int32, device=dev)
+            t = ph.start("scatter")
+            lz._check(Lb.lasagna_shard_scatter(
+                lz._ptr(packed_local), n_local, lo, n_total, world, L, l_min, l_lo, l_hi,
+                None if first else ctypes.c_void_p(claimed_mine), lz._ptr(send),
+                lz._ptr(send_fill), lz._ptr(counters), s))
+            ph.stop(t)
+            ph.launches["scatter"] += 1
+            first = False
+            # 3. the hash-range shuffle: equal split sizes, nothing to count or synchronise
+            recv = torch.empty_like(send)
+            recv_fill = torch.empty_like(send_fill)
+            t = ph.start("exchange")
+            C.all_to_all_single(recv, send)
+            C.all_to_all_single(recv_fill, send_fill)
+            ph.stop(t)
+            del send, send_fill
+            nbytes = ctypes.c_size_t(0)
+            lz._check(Lb.lasagna_shard_part_bytes(n_total, world, L, l_min, Gc, ctypes.byref(nbytes)))
+            part = lz._workspace(nbytes.value, dev)
+            t = ph.start("refine")
+            lz._check(Lb.lasagna_shard_partition(lz._ptr(recv), lz._ptr(recv_fill), n_total, world,
+                                                 L, l_min, l_lo, l_hi, lz._ptr(part),
+                                                 lz._ptr(counters), s))
+            ph.stop(t)
+            ph.launches["refine"] += int(geo.levels) - 1
+            del recv, recv_fill
+            # 4. per length: join (my buckets) and the sharded greedy (everyone's pairs)
+            for l in range(l_hi, l_lo - 1, -1):
+                t = ph.start("join")
+                lz._check(Lb.lasagna_shard_join(lz._ptr(part), n_total, world, L, l_min, l_lo,
+                                                l_hi, l, lz._ptr(packed_all), lz._ptr(pool), cap,
+                                                lz._ptr(pool_count), lz._ptr(counters), s))
+                ph.stop(t)
+                t = ph.start("greedy")
+                lz._check(Lb.lasagna_greedy_shard_length(ranks, world, rank, int(geo.slice), cap,
+                                                         l, s))
+                ph.stop(t)
+                ph.launches["join"] += 1
+                ph.launches["greedy_lengths"] += 1
+            del part
+        # 5. outcome: region overflow or pool overflow anywhere -> every rank reruns
+        ctr = arena.tensor("ctr", torch.int64)
+        flags = torch.stack([counters[0].clamp(max=1), ctr[5]]).to(torch.int64)
+        C.all_reduce(flags, op=dist.ReduceOp.MAX)
+        ovf, max_pl = (int(x) for x in flags.tolist())
+        if ovf:
+            raise RegionOverflow("a slack region overflowed")
+        if max_pl > cap:
+            need = max_pl * 5 // 4 + 1
+        else:
+            need = 0
+            # the graph: every rank's slices of succ/olen, all-gathered
+            slice_ = int(geo.slice)
+            succ_all = torch.empty(world * slice_, dtype=torch.int32, device=dev)
+            olen_all = torch.empty(world * slice_, dtype=torch.uint8, device=dev)
+            C.all_gather_into_tensor(succ_all, arena.tensor("succ", torch.int32).clone())
+            C.all_gather_into_tensor(olen_all, arena.tensor("olen", torch.uint8).clone())
+            tot = torch.stack([ctr[4], ctr[3], counters[1], counters[3]]).clone()
+            C.all_reduce(tot)
+            mx = ctr[6:7].clone()
+            C.all_reduce(mx, op=dist.ReduceOp.MAX)
+            n_pairs, n_greedy, pruned, false_m = (int(x) for x in tot.tolist())
+            stats = {"n_pairs": n_pairs, "n_greedy": n_greedy, "pruned_entries": pruned,
+                     "fp_false_matches": false_m, "rounds_max": int(mx.item()),
+                     "lengths_per_pass": G, "partition_levels": int(geo.levels), "path": "fast",
+                     "greedy_pair_rounds": int(ctr[7].item()), "n_local": n_local,
+                     "launches": dict(ph.launches)}
+            if timing:
+                torch.cuda.synchronize()
+                stats["ms"] = ph.totals()
+            out = (succ_all[:2 * n_total], olen_all[:2 * n_total], stats)
+    finally:
+        arena.close()
+    if need:
+        return greedy_graph_fast(ascii_local, n_total, L, l_min, group, lengths_per_pass, need)
+    return out
+
+
 def lz_words(L: int) -> int:
     w = (L + 31) // 32
     return 1 if w <= 1 else 2 if w <= 2 else 4 if w <= 4 else 8
 
 
 # ------------------------------------------------------------------------------ bench (N > 1)
+def _fast_roofline(st: dict, n_total: int, L: int, l_min: int, world: int, peak: dict,
+                   ms_step: float, steps: int) -> dict:
+    """Algorithmic bytes per launch of this rank's phases over their
+    CUDA-event times: scatter 8 B per key written (+ packed rows read), refine 16 B per key
+    and level, join 8 B per key read + 64 B per verified candidate, greedy 64 B per pair-round.
+    Exchange: the bytes this rank sends over NVLink (all-to-all of its level-1 regions)."""
+    ms = {k: v / steps for k, v in st.get("ms", {}).items()}
+    la = {k: v / steps for k, v in st["launches"].items()}
+    n_len = L - l_min
+    N_rank = 2 * n_total / world                 # keys per length per rank after the exchange
+    W = lz_words(L)
+    per_len_keys = 2 * st["n_local"]
+    bytes_ = {
+        "scatter_table_kernel": 8.0 * per_len_keys * n_len + 8.0 * W * st["n_local"],
+        "refine_kernel": 16.0 * N_rank * n_len * max(1, st["partition_levels"] - 1),
+        "bucket_join_kernel": 8.0 * N_rank * n_len + 64.0 * (st["n_pairs"] + st["fp_false_matches"]) / world,
+        "greedy": 64.0 * st["greedy_pair_rounds"] / steps,
+        "exchange": 8.0 * per_len_keys * n_len * 1.02,
+    }
+    keymap = {"scatter_table_kernel": "scatter", "refine_kernel": "refine",
+              "bucket_join_kernel": "join", "greedy": "greedy", "exchange": "exchange"}
+    phases = {}
+    for k, b in bytes_.items():
+        t = ms.get(keymap[k], 0.0)
+        phases[k] = {"ms_per_step": t, "bytes_per_step": b,
+                     "gbs": b / (t / 1e3) / 1e9 if t > 0 else None}
+    hbm = {k: v for k, v in phases.items() if k not in ("exchange", "greedy")}
+    name = max(hbm, key=lambda k: hbm[k]["ms_per_step"])
+    ach = hbm[name]["gbs"] or 0.0
+    step_bytes = sum(v["bytes_per_step"] for k, v in phases.items() if k != "exchange")
+    step_gbs = step_bytes / (ms_step / 1e3) / 1e9
+    return {"bound": "hbm", "kernel": name, "achieved": round(ach, 1), "peak": peak["hbm_gbs"],
+            "peak_source": peak["source"], "unit": "GB/s", "frac": round(ach / peak["hbm_gbs"], 4),
+            "traffic": None, "per_rank": True,
+            "step": {"bytes": step_bytes, "achieved": round(step_gbs, 1),
+                     "frac": round(step_gbs / peak["hbm_gbs"], 4)},
+            "phases": phases}
+
+
 def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> None:
     """`bench.py` under torchrun: strong scaling at fixed n (every rank holds 1/g of the reads),
-    barrier + synchronize around exactly K steps, time = max over ranks."""
+    barrier + synchronize around exactly K steps, time = max over ranks.  Default path: the
+    sharded fast path (greedy_graph_fast); --dist-path exact runs the round-1 exact path."""
     import readgen
     for k, v in (("RANK", "0"), ("WORLD_SIZE", "1"), ("MASTER_ADDR", "127.0.0.1"),
                  ("MASTER_PORT", "29517")):
         os.environ.setdefault(k, v)  # --force-dist without torchrun: a one-rank group
+    os.environ.setdefault("NCCL_DEBUG", "INFO")  # the communicator's rank count in the log
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -295,16 +597,23 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
     else:
         dist.init_process_group("gloo")
     world, rank = dist.get_world_size(), dist.get_rank()
+    fast = getattr(args, "dist_path", "fast") == "fast"
     n, L, l_min = cfg.n, cfg.L, cfg.l_min
-    lo, hi, _ = shard_range(n, world, rank)
+    lo, hi, _ = fast_shard_range(n, world, rank) if fast else shard_range(n, world, rank)
     host = torch.empty((hi - lo, L), dtype=torch.uint8).pin_memory()
     readgen.reads_into(host.data_ptr(), cfg.seed, cfg.G, L, cfg.p_err, lo, hi)
     dev_ascii = host.to(dev)
     be = CudaBackend(dev)
     stream = torch.cuda.current_stream(dev)
 
-    def step(src, d2h: bool):
-        succ, olen, st = greedy_graph(src, n, L, l_min, be, lengths_per_pass=args.lengths_per_pass)
+    def step(src, d2h: bool, timing: bool = False):
+        if fast:
+            succ, olen, st = greedy_graph_fast(src.to(dev, non_blocking=True), n, L, l_min,
+                                               lengths_per_pass=args.lengths_per_pass,
+                                               timing=timing)
+        else:
+            succ, olen, st = greedy_graph(src, n, L, l_min, be,
+                                          lengths_per_pass=args.lengths_per_pass)
         if d2h:
             succ.cpu(), olen.cpu()
         return st
@@ -328,6 +637,8 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
     clocks = sampler.stop()
     ms = torch.tensor([e0.elapsed_time(e1) / args.steps], device=dev)
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    # one more step with phase events (outside the timed region) for the roofline
+    st_t = step(dev_ascii, False, timing=True) if fast else None
     # end to end from pinned host ASCII
     dist.barrier()
     torch.cuda.synchronize()
@@ -349,15 +660,20 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
             "config": {"workload": f"{cfg.name}: {cfg.note}", "n": n, "L": L, "l_min": l_min,
                        "G": cfg.G, "p_err": cfg.p_err, "seed": cfg.seed,
                        "parallelism": f"hash-range x{world}",
+                       "dist_path": "fast (scatter -> equal-split all-to-all -> refine -> join -> "
+                                    "sharded greedy over peer memory)" if fast else "exact",
                        "l2": "inputs larger than L2"},
-            "overlap_edges_per_s": 2 * st["n_pairs"] / (ms_step / 1e3),
-            "read_end_pairs": st["n_pairs"],
+            "overlap_edges_per_s": st["n_pairs"] / (ms_step / 1e3),
+            "read_end_pairs": st["n_pairs"], "greedy_pairs": st.get("n_greedy"),
             "e2e": {"value": n / (e2e_ms / 1e3), "unit": "reads/s", "ms_per_step": e2e_ms,
                     "h2d_bytes_per_step": n * L, "d2h_bytes_per_step": 2 * n * 5},
-            "roofline": None,
+            "roofline": (_fast_roofline(st_t, n, L, l_min, world, peak, ms_step, 1)
+                         if st_t else None),
             "clocks": clocks,
             "gpu_launches": launches,
         }
+        if world == 1 and not getattr(args, "no_cpu_baseline", False):
+            out["cpu_baseline"] = cpu_baseline(cfg, host.numpy())
         print(json.dumps(out), flush=True)
     dist.barrier()
     dist.destroy_process_group()

@@ -43,6 +43,21 @@ class _Stats(ctypes.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class ShardGeom(ctypes.Structure):
+    """lasagna_shard_geom (include/lasagna.h): sizes of the sharded fast path."""
+    _fields_ = [("levels", ctypes.c_uint32), ("last_bits", ctypes.c_uint32),
+                ("nb_pad", ctypes.c_uint32), ("vbits", ctypes.c_uint32),
+                ("n_pad", ctypes.c_uint64), ("slice", ctypes.c_uint64), ("cap1", ctypes.c_uint64),
+                ("send_entries", ctypes.c_uint64), ("fill_words", ctypes.c_uint64),
+                ("part_bytes", ctypes.c_uint64), ("buckets", ctypes.c_uint64)]
+
+
+class GreedyRank(ctypes.Structure):
+    """lasagna_greedy_rank: one rank's buffers, as device pointers valid in this process."""
+    _fields_ = [(k, ctypes.c_void_p) for k in
+                ("pool", "pool2", "pool_count", "ctr", "best", "claimed", "succ", "olen", "tail")]
+
+
 _lib = None
 
 
@@ -82,6 +97,17 @@ def lib() -> ctypes.CDLL:
         "lasagna_greedy_pairs": [u64, vp, vp, vp, u64, vp, psz, vp, vp, pu32, vp],
         "lasagna_compress": [vp, u64, u32, vp, vp, vp, psz, vp, u64, vp, vp, u64, pu64, pu64,
                              vp],
+        "lasagna_shard_geometry": [u64, u32, u32, u32, ctypes.POINTER(ShardGeom)],
+        "lasagna_shard_part_bytes": [u64, u32, u32, u32, u32, psz],
+        "lasagna_shard_scatter": [vp, u64, u64, u64, u32, u32, u32, u32, u32, vp, vp, vp, vp, vp],
+        "lasagna_shard_partition": [vp, vp, u64, u32, u32, u32, u32, u32, vp, vp, vp],
+        "lasagna_shard_join": [vp, u64, u32, u32, u32, u32, u32, u32, vp, vp, u64, vp, vp, vp],
+        "lasagna_greedy_shard_length": [ctypes.POINTER(GreedyRank), u32, ctypes.c_int32, u64,
+                                        u64, u32, vp],
+        "lasagna_peer_alloc": [sz, ctypes.POINTER(ctypes.c_void_p), vp],
+        "lasagna_peer_free": [vp],
+        "lasagna_peer_open": [vp, ctypes.POINTER(ctypes.c_void_p)],
+        "lasagna_peer_close": [vp],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
