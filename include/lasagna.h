@@ -130,7 +130,8 @@ typedef struct {
                                     the first; then n_pairs counts only pairs of entries that
                                     were live when their group was built, not the full |P|) */
     uint32_t partition_levels;   /* bucketed path: MSD partition levels (1..3); 0: exact path */
-    uint32_t reserved;
+    uint32_t hash_subpasses;     /* K > 1: each length built and joined in K hash-range
+                                    sub-passes (the workspace holds no whole length; f4) */
 } lasagna_stats;
 
 /* ---------------------------------------------------------------------------------------
@@ -145,6 +146,9 @@ typedef struct {
  * lengths_per_pass: lengths whose tables are built per device pass (a8 semi-streaming);
  *   0 = all of [l_min, L-1] in one pass.  The call uses the largest group <= this that fits
  *   *workspace_bytes; the query (workspace == NULL) reports the size for lengths_per_pass.
+ *   When not even one length's tables fit, each length is built and joined in K hash-range
+ *   sub-passes (K a power of two <= 256, the smallest that fits; stats->hash_subpasses): the
+ *   B200 replacement of the paper's external merge (Alg. 1).
  * Returns LASAGNA_ENOSPC with *workspace_bytes raised when a length produced more candidate
  * pairs than the workspace's pair pool holds (call again with the larger workspace).
  */
@@ -174,8 +178,10 @@ LASAGNA_API lasagna_status lasagna_greedy_graph_ascii(const char *ascii, uint64_
                                                       lasagna_stats *stats, void *stream);
 
 /* Planner for the semi-streaming driver (a8): the largest
- * lengths_per_pass whose workspace fits `budget_bytes`, and that workspace size.  Returns
- * LASAGNA_ENOSPC when even one length per pass does not fit (*workspace_bytes = minimum). */
+ * lengths_per_pass whose workspace fits `budget_bytes`, and that workspace size; below one
+ * whole length, lengths_per_pass = 1 and the workspace of the fewest hash-range sub-passes
+ * that fit.  Returns LASAGNA_ENOSPC when not even 256 sub-passes fit (*workspace_bytes =
+ * minimum). */
 LASAGNA_API lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budget_bytes,
                             uint32_t *lengths_per_pass, size_t *workspace_bytes);
 

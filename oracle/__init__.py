@@ -61,6 +61,8 @@ def lib():
         L.oracle_pack.argtypes = [vp, u64, u32, u32, vp]
         L.oracle_overlaps.argtypes = [vp, u64, u32, u32, u64, vp, vp, vp]
         L.oracle_overlaps.restype = u64
+        L.oracle_overlaps_approx.argtypes = [vp, u64, u32, u32, u64, u64, u64, u64, u64, vp, vp, vp]
+        L.oracle_overlaps_approx.restype = u64
         L.oracle_greedy.argtypes = [u64, u64, vp, vp, vp, vp, vp]
         L.oracle_greedy.restype = u64
         L.oracle_greedy_graph.argtypes = [vp, u64, u32, u32, vp, vp, vp]
@@ -152,6 +154,27 @@ def overlaps(reads, l_min: int):
     pb = np.empty(m, dtype=np.uint32)
     lib().oracle_overlaps(a.ctypes.data, n, L, l_min, m, pl.ctypes.data, pa.ctypes.data,
                           pb.ctypes.data)
+    return pl, pa, pb
+
+
+SIGMA2 = 7                   # the approximate mode's second fingerprint: radix 7,
+Q2 = (1 << 64) - 59          # the largest prime below 2^64 (reading R22)
+
+
+def overlaps_approx(reads, l_min: int, sigma2: int = SIGMA2, q2: int = Q2, sigma1: int = SIGMA,
+                    q1: int = Q):
+    """Approximate mode: pairs whose (F(sigma1, q1), F(sigma2, q2)) fingerprints of
+    suffix and prefix agree, by Algorithm 2 on the P_l / S_l lists; (l, a, b) as overlaps()."""
+    a = _ascii(reads)
+    n, L = a.shape
+    args = (a.ctypes.data, n, L, l_min, sigma1, q1, sigma2, q2)
+    m = int(lib().oracle_overlaps_approx(*args, 0, None, None, None))
+    if m == 0xFFFFFFFFFFFFFFFF:
+        raise ValueError("oracle: invalid reads or parameters")
+    pl = np.empty(m, dtype=np.uint8)
+    pa = np.empty(m, dtype=np.uint32)
+    pb = np.empty(m, dtype=np.uint32)
+    lib().oracle_overlaps_approx(*args, m, pl.ctypes.data, pa.ctypes.data, pb.ctypes.data)
     return pl, pa, pb
 
 

@@ -95,6 +95,9 @@ struct ScatterArgs {
     // so every rank's regions of all G lengths are one contiguous slice of out/fill (equal
     // split sizes for the all-to-all).  dest_g = 1, nb_pad = 256: the single-GPU [G][256].
     uint32_t dest_g = 1, nb_pad = 256;
+    // hash-range sub-pass (single GPU, tables larger than the workspace): keep only the keys
+    // whose level-1 digit belongs to range keep_owner of dest_g, regions numbered from 0
+    int32_t keep_owner = -1;
 };
 // region index of (segment s of G, level-1 digit d) under ScatterArgs' shard layout
 __host__ __device__ __forceinline__ uint64_t shard_region(uint32_t s, uint32_t G, uint32_t d,

@@ -118,6 +118,7 @@ static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
     uint32_t G;          // lengths per group
+    uint32_t K;          // hash-range sub-passes per length (1: whole tables)
     uint64_t pool_cap;   // pair pool capacity (pairs)
     size_t tabA, tabB, status, status_bytes, hist, ctrs, pool, pool2, best, claimed, fill1,
         fill2, fill3, total;
@@ -153,11 +154,15 @@ static GreedyPeers single_peers(const GreedyBufs &gb, unsigned long long *ctr_pe
     return p;
 }
 
-static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy)
+// K > 1 (hash-range sub-passes, one length per pass): the tables hold only the level-1 digits
+// of one of K ranges at a time (nb = ceil(256 / K) digits, shard_region's layout with dest_g =
+// K), and there is no exact-path fallback (it needs whole tables)
+static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy, uint32_t K = 1)
 {
     Layout l;
     l.G = G;
     l.pool_cap = pool_cap;
+    l.K = K;
     size_t off = 0;
     auto take = [&](size_t bytes) {
         size_t o = off;
@@ -166,19 +171,21 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     };
     // tabA/tabB: the exact path's LSD ping-pong buffers, or the bucketed path's levels with
     // slack: level 1 in tabA, level 2 in tabB, level 3 (P = 3) in tabA again
-    const size_t exact_b = (size_t)G * g.N * 8;
-    const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half : 256 * g.cap1) * 8;
-    const size_t lvl2_b = g.P == 2   ? (size_t)G * 131072 * g.half * 8
-                          : g.P == 3 ? (size_t)G * 65536 * g.cap2 * 8
+    const uint64_t nb = (256 + K - 1) / K; // level-1 digits per pass
+    const size_t exact_b = K > 1 ? 0 : (size_t)G * g.N * 8;
+    const size_t lvl1_b = (size_t)G * (g.P == 1 ? 512 * g.half : nb * g.cap1) * 8;
+    const size_t lvl2_b = g.P == 2   ? (size_t)G * nb * 512 * g.half * 8
+                          : g.P == 3 ? (size_t)G * nb * 256 * g.cap2 * 8
                                      : 0;
-    const size_t lvl3_b = g.P == 3 ? (size_t)G * 2 * g.n_buckets * g.half * 8 : 0;
+    const size_t lvl3_b = g.P == 3 ? (size_t)G * 2 * (g.n_buckets / 256 * nb) * g.half * 8 : 0;
     l.tabA = take(std::max({exact_b, lvl1_b, lvl3_b}));
     l.tabB_bytes = std::max(exact_b, lvl2_b);
     l.tabB = take(l.tabB_bytes);
     l.fill1 = take((size_t)G * 512 * 4);
-    l.fill2 = take(g.P == 2 ? (size_t)G * 131072 * 4 : g.P == 3 ? (size_t)G * 65536 * 4 : 4);
-    l.fill3 = take(g.P == 3 ? (size_t)G * 2 * g.n_buckets * 4 : 4);
-    l.status_bytes = std::max(sort_status_bytes(g.N, G), sort_status_bytes(pool_cap, 1));
+    l.fill2 = take(g.P == 2 ? (size_t)G * nb * 512 * 4 : g.P == 3 ? (size_t)G * nb * 256 * 4 : 4);
+    l.fill3 = take(g.P == 3 ? (size_t)G * 2 * (g.n_buckets / 256 * nb) * 4 : 4);
+    l.status_bytes = std::max(K > 1 ? (size_t)0 : sort_status_bytes(g.N, G),
+                              sort_status_bytes(pool_cap, 1));
     l.status = take(l.status_bytes);
     l.hist = take((size_t)8 * std::max<uint32_t>(G, 1) * 256 * 4);
     l.ctrs = take(CTR_BYTES);
@@ -398,10 +405,12 @@ static uint64_t stored_keep(const Geometry &g)
 // Build + partition the key tables of lengths [l_lo, l_hi] (level 1 fused with a2, then the
 // refine levels; the final buckets end in tabB for P = 2, tabA for P = 1 and P = 3).
 static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint32_t l_lo,
-                                           uint32_t l_hi, PhaseTimer &tm, lasagna_stats *st)
+                                           uint32_t l_hi, PhaseTimer &tm, lasagna_stats *st,
+                                           uint32_t sub = 0)
 {
     const Geometry &g = r.g;
     const uint32_t G = l_hi - l_lo + 1;
+    const uint32_t K = r.lay.K, nb = (256 + K - 1) / K; // sub-pass `sub` of K: digit range
     unsigned int *ovf = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
     LSG_CUDA(cudaMemsetAsync(r.fill1, 0, (size_t)G * 512 * 4, r.s));
     ScatterArgs sa;
@@ -421,9 +430,12 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
     sa.overflow = ovf;
     sa.ascii = r.ascii; // fused a1 (first group only)
     sa.claimed = r.prune ? r.claimed : nullptr;
-    sa.pruned = r.ctr64 + CTR_PRUNED;
+    sa.pruned = sub == 0 ? r.ctr64 + CTR_PRUNED : nullptr; // counted once per length
     sa.packed_out = r.packed_out;
     sa.first_bad = r.first_bad;
+    sa.dest_g = K;
+    sa.nb_pad = nb;
+    sa.keep_owner = K > 1 ? (int32_t)sub : -1;
     const char *host = r.ascii_host;
     r.ascii = nullptr;
     r.ascii_host = nullptr;
@@ -450,7 +462,7 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
         ra.split = g.P == 2;
         ra.overflow = ovf;
         if ((rc = tm.start(PH_SORT)) != LASAGNA_OK) return rc;
-        if ((rc = launch_refine(ra, (uint64_t)G * 256, r.s)) != LASAGNA_OK) return rc;
+        if ((rc = launch_refine(ra, (uint64_t)G * nb, r.s)) != LASAGNA_OK) return rc;
         if (g.P == 3) {
             // level 3: dlast more bits, split into build and probe halves
             ra.in = r.tab[1];
@@ -462,7 +474,7 @@ static lasagna_status build_group_bucketed(Run &r, const uint64_t *packed, uint3
             ra.fill_out = r.fill3;
             ra.cap_out = g.half;
             ra.split = true;
-            if ((rc = launch_refine(ra, (uint64_t)G * 65536, r.s)) != LASAGNA_OK) return rc;
+            if ((rc = launch_refine(ra, (uint64_t)G * nb * 256, r.s)) != LASAGNA_OK) return rc;
         }
         if ((rc = tm.stop()) != LASAGNA_OK) return rc;
         if (st) st->sort_launches += g.P - 1;
@@ -516,11 +528,14 @@ static bool join_filter() { return env_flag("LASAGNA_JOIN_FILTER", '1'); }
 // Join (search + verify) of length l into the pool; if m_out, synchronise and report the
 // pair count.
 static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, uint32_t l_lo,
-                                    int which, uint64_t *m_out)
+                                    int which, uint64_t *m_out, bool reset_pool = true)
 {
     const Geometry &g = r.g;
     const uint32_t s = l - l_lo;
-    LSG_CUDA(cudaMemsetAsync(r.ctr64 + CTR_POOL, 0, sizeof(unsigned long long), r.s));
+    // buckets per length: all of them, or those of one hash-range sub-pass
+    const uint64_t nbk = r.lay.K > 1 ? g.n_buckets / 256 * ((256 + r.lay.K - 1) / r.lay.K) : g.n_buckets;
+    if (reset_pool)
+        LSG_CUDA(cudaMemsetAsync(r.ctr64 + CTR_POOL, 0, sizeof(unsigned long long), r.s));
     JoinArgs ja;
     ja.packed = packed;
     ja.keys = r.tab[which] + (uint64_t)s * g.N;
@@ -542,10 +557,10 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.j = ja;
         bj.overflow = reinterpret_cast<unsigned int *>(r.ctr64 + CTR_OVERFLOW);
         // final level: [G][n_buckets][2][half] (tabB for P = 2, tabA for P = 1 and 3)
-        bj.buckets = (g.P == 2 ? r.tab[1] : r.tab[0]) + (uint64_t)s * 2 * g.n_buckets * g.half;
-        bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * g.n_buckets;
+        bj.buckets = (g.P == 2 ? r.tab[1] : r.tab[0]) + (uint64_t)s * 2 * nbk * g.half;
+        bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * nbk;
         bj.half_cap = g.half;
-        bj.n_buckets = g.n_buckets;
+        bj.n_buckets = nbk;
         // block windows (partition.cu); LASAGNA_JOIN=warp (A/B only): one warp per bucket
         // (warpjoin.cu) when a half fits a warp's slice — measured slower at cfg3 (31.9 vs
         // 17.1 ms per step)
@@ -562,6 +577,18 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         *m_out = m;
     }
     return LASAGNA_OK;
+}
+
+// hash-range sub-passes needed when no whole length fits (G == 0): the smallest power of two
+// K whose one-length layout fits `bytes` (bucketed path, two or three levels); 1 otherwise
+static bool use_bucketed(const Geometry &g);
+static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool greedy, uint32_t K);
+static uint32_t subpasses_for(const Geometry &g, size_t bytes, uint64_t cap, uint32_t G)
+{
+    if (G > 0 || !use_bucketed(g) || g.P < 2) return 1;
+    for (uint32_t K = 2; K <= 256; K *= 2)
+        if (layout(g, 1, cap, true, K).total <= bytes) return K;
+    return 1;
 }
 
 static uint32_t choose_G(const Geometry &g, uint32_t want, size_t bytes, uint64_t cap, bool greedy)
@@ -677,14 +704,16 @@ lasagna_status lasagna_plan(uint64_t n, uint32_t L, uint32_t l_min, size_t budge
     Geometry g = geometry(n, L, l_min);
     uint64_t cap = default_pool_cap(g);
     uint32_t G = choose_G(g, 0, budget_bytes, cap, true);
+    const uint32_t K = subpasses_for(g, budget_bytes, cap, G);
+    if (K > 1) G = 1;
     if (G == 0) {
         *lengths_per_pass = 0;
-        *workspace_bytes = layout(g, 1, cap, true).total;
-        set_error("budget %zu below the one-length workspace %zu", budget_bytes, *workspace_bytes);
+        *workspace_bytes = layout(g, 1, cap, true, use_bucketed(g) && g.P >= 2 ? 256 : 1).total;
+        set_error("budget %zu below the smallest workspace %zu", budget_bytes, *workspace_bytes);
         return LASAGNA_ENOSPC;
     }
     *lengths_per_pass = G;
-    *workspace_bytes = layout(g, G, cap, true).total;
+    *workspace_bytes = layout(g, G, cap, true, K).total;
     return LASAGNA_OK;
 }
 
@@ -724,21 +753,27 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         return LASAGNA_EINVAL;
     }
     uint32_t G = choose_G(g, G_req, *workspace_bytes, cap, true);
+    // f4: when even one length's tables exceed the workspace, each length is
+    // built and joined in K hash-range sub-passes (level-1 digit ranges) — the B200 form of the
+    // paper's external merge (Alg. 1): a range's tables are complete in HBM, so
+    // nothing is merged; the fingerprints are recomputed per sub-pass instead of spilled
+    uint32_t K = subpasses_for(g, *workspace_bytes, cap, G);
+    if (K > 1) G = 1;
     if (G == 0) {
-        *workspace_bytes = layout(g, 1, cap, true).total;
+        *workspace_bytes = layout(g, 1, cap, true, use_bucketed(g) && g.P >= 2 ? 256 : 1).total;
         set_error("workspace too small");
         return LASAGNA_ENOSPC;
     }
     // spare bytes beyond the chosen layout enlarge the pair pool
     {
-        size_t spare = *workspace_bytes - layout(g, G, cap, true).total;
+        size_t spare = *workspace_bytes - layout(g, G, cap, true, K).total;
         cap += spare / 16; // pool + pool2: 16 B per pair (the status words shrink it below)
-        while (cap > default_pool_cap(g) && layout(g, G, cap, true).total > *workspace_bytes) cap -= cap / 256 + 1;
+        while (cap > default_pool_cap(g) && layout(g, G, cap, true, K).total > *workspace_bytes) cap -= cap / 256 + 1;
     }
     cudaStream_t s = (cudaStream_t)stream;
     Run r;
     r.g = g;
-    r.lay = layout(g, G, cap, true);
+    r.lay = layout(g, G, cap, true, K);
     r.s = s;
     r.bind(workspace);
     uint32_t *claimed = r.at<uint32_t>(r.lay.claimed);
@@ -773,6 +808,10 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
 
   for (int attempt = 0; attempt < 2; ++attempt) {
     r.bucketed = attempt == 0 && use_bucketed(g);
+    if (r.lay.K > 1 && !r.bucketed) {
+        set_error("hash-range sub-passes need the bucketed path");
+        return LASAGNA_EINVAL;
+    }
     gb.epoch = 1;
     lasagna_stats st;
     memset(&st, 0, sizeof st);
@@ -801,6 +840,27 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         // a claimed end can never gain an edge).  LASAGNA_NO_PRUNE=1 keeps them (then
         // n_pairs is the full |P|).
         r.prune = l_hi != (int64_t)L - 1 && !env_flag("LASAGNA_NO_PRUNE", '1');
+        if (r.lay.K > 1) {
+            // one length in K hash-range sub-passes: each builds the tables of one digit range
+            // and joins them into the length's pool; the greedy runs once all are in
+            const uint32_t l = (uint32_t)l_hi;
+            for (uint32_t sub = 0; sub < r.lay.K; ++sub) {
+                if ((rc = build_group_bucketed(r, packed, l, l, tm, &st, sub)) != LASAGNA_OK)
+                    return rc;
+                ++st.passes;
+                if ((rc = tm.start(PH_SEARCH)) != LASAGNA_OK) return rc;
+                if ((rc = search_length(r, packed, l, l, 0, nullptr, sub == 0)) != LASAGNA_OK)
+                    return rc;
+                if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+                ++st.search_launches;
+            }
+            if ((rc = tm.start(PH_GREEDY)) != LASAGNA_OK) return rc;
+            if ((rc = old_greedy() ? greedy_length(gb, (uint8_t)l, succ, olen, s)
+                                   : greedy_length_peers(peers, (uint8_t)l, s)) != LASAGNA_OK)
+                return rc;
+            if ((rc = tm.stop()) != LASAGNA_OK) return rc;
+            continue;
+        }
         if ((rc = build_group(r, packed, l_lo, (uint32_t)l_hi, &which, tm, &st)) != LASAGNA_OK)
             return rc;
         ++st.passes;
@@ -831,12 +891,19 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
             return LASAGNA_EINVAL;
         }
     }
-    if (r.bucketed && h[CTR_OVERFLOW]) continue; // a slack region overflowed: exact path
+    if (r.bucketed && h[CTR_OVERFLOW]) {
+        if (r.lay.K > 1) { // the exact path needs whole tables: not in a sub-pass workspace
+            set_error("a slack region overflowed in a hash-range sub-pass: give the call a "
+                      "workspace for one whole length (%zu bytes)", layout(g, 1, cap, true, 1).total);
+            return LASAGNA_ENOSPC;
+        }
+        continue; // a slack region overflowed: exact path
+    }
     const unsigned long long *book = old_greedy() ? h + CTR_BOOK : h + CTR_PEER + PC_BOOK;
     const unsigned long long work = old_greedy() ? h[CTR_WORK] : h[CTR_PEER + PC_WORK];
     if (book[2] > cap) {
         const uint64_t need = book[2] + book[2] / 4;
-        *workspace_bytes = layout(g, G, need, true).total;
+        *workspace_bytes = layout(g, G, need, true, r.lay.K).total;
         set_error("a length produced %llu pairs > pool %llu", book[2], (unsigned long long)cap);
         return LASAGNA_ENOSPC;
     }
@@ -849,6 +916,7 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
         st.greedy_pair_rounds = work;
         st.pruned_entries = h[CTR_PRUNED];
         st.partition_levels = r.bucketed ? g.P : 0;
+        st.hash_subpasses = r.lay.K;
         if ((rc = tm.finish(&st)) != LASAGNA_OK) return rc;
         st.kernel_launches = launch_count() - launches0;
         *stats = st;

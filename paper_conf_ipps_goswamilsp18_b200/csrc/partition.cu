@@ -258,7 +258,10 @@ scatter_table_kernel(ScatterArgs a)
     for (uint32_t t = threadIdx.x; t < NBIN; t += SC_THREADS) cnt[t] = 0;
     if (!SPLIT)
         for (uint32_t d = threadIdx.x; d < 256; d += SC_THREADS)
-            rbase[d] = (uint32_t)shard_region(0, a.l_hi - a.l_lo + 1u, d, a.dest_g, a.nb_pad);
+            rbase[d] = (uint32_t)(shard_region(0, a.l_hi - a.l_lo + 1u, d, a.dest_g, a.nb_pad) -
+                                  (a.keep_owner < 0 ? 0ull
+                                                    : (uint64_t)a.keep_owner *
+                                                          (a.l_hi - a.l_lo + 1u) * a.nb_pad));
     __syncthreads();
     const uint64_t v0 = 2 * (a.read_offset + i);
     FpStreams st;
@@ -314,8 +317,13 @@ scatter_table_kernel(ScatterArgs a)
                 kk[2 * q] = e0;
                 kk[2 * q + 1] = e1;
                 const uint32_t b0 = q * NBL + d0, b1 = q * NBL + d1;
-                if (live0) rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
-                if (live1) rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
+                bool k0 = live0, k1 = live1;
+                if (!SPLIT && a.keep_owner >= 0) { // block-uniform: this sub-pass's digits only
+                    k0 = k0 && (int32_t)((d0 * a.dest_g) >> 8) == a.keep_owner;
+                    k1 = k1 && (int32_t)((d1 * a.dest_g) >> 8) == a.keep_owner;
+                }
+                if (k0) rk[2 * q] = (b0 << 16) | atomicAdd(&cnt[b0], 1u);
+                if (k1) rk[2 * q + 1] = (b1 << 16) | atomicAdd(&cnt[b1], 1u);
             }
         }
         {

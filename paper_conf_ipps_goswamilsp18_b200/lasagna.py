@@ -37,7 +37,7 @@ class _Stats(ctypes.Structure):
                 ("ms_greedy", ctypes.c_float),
                 ("greedy_pair_rounds", ctypes.c_uint64), ("pruned_entries", ctypes.c_uint64),
                 ("partition_levels", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32)]
+                ("hash_subpasses", ctypes.c_uint32)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -240,6 +240,7 @@ class GreedyGraph:
         self.device = torch.device(device)
         if self.device.type == "cuda" and self.device.index is None:
             self.device = torch.device("cuda", torch.cuda.current_device())
+        planned = None
         if lengths_per_pass == 0:
             if budget_bytes is None:
                 free, _ = torch.cuda.mem_get_info(self.device)
@@ -247,12 +248,14 @@ class GreedyGraph:
             lp, need = plan(n, L, l_min, max(0, budget_bytes))
             if lp == 0:
                 raise LasagnaError(ENOSPC, f"needs {need} bytes of workspace, budget {budget_bytes}")
-            lengths_per_pass = lp
+            lengths_per_pass, planned = lp, need
         self.lengths_per_pass = lengths_per_pass
         ws = ctypes.c_size_t(0)
         _check(lib().lasagna_greedy_graph(None, n, L, l_min, lengths_per_pass, None,
                                           ctypes.byref(ws), None, None, None, None))
-        self.ws_bytes = int(ws.value)
+        # below one whole length the planner's workspace runs hash-range sub-passes (smaller
+        # than the one-length query)
+        self.ws_bytes = int(ws.value) if planned is None else min(int(ws.value), planned)
         self.ws = _workspace(self.ws_bytes, self.device)
         self.succ = torch.empty(2 * n, dtype=torch.int32, device=self.device)
         self.olen = torch.empty(2 * n, dtype=torch.uint8, device=self.device)

@@ -43,6 +43,22 @@ def main():
     c = lz.compress(packed, n, L, r.succ, r.olen)
     eb, _, _ = oracle.compress(reads, esucc, eolen)
     assert c.bases.cpu().numpy().tobytes() == eb
+    # hash-range sub-passes (f4): a workspace below one whole length
+    import ctypes
+    ws = ctypes.c_size_t(0)
+    lz.lasagna._check(lz.lib().lasagna_greedy_graph(None, n, L, l_min, 1, None, ctypes.byref(ws),
+                                                    None, None, None, None))
+    os.environ["LASAGNA_TEST_LEVELS"] = "2"
+    sub = lz.GreedyGraph(n, L, l_min, "cuda", budget_bytes=int(ws.value * 0.3))
+    r = sub(packed)
+    assert r.stats["hash_subpasses"] > 1, r.stats
+    assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), esucc)
+    del os.environ["LASAGNA_TEST_LEVELS"]
+    # the sharded greedy's cross-rank protocol: three ranks in one launch
+    from tests.test_gpu_sharded import _sharded_greedy
+    ssucc, solen, _ = _sharded_greedy(n, pl.cpu().numpy(), pa.cpu().numpy().view(np.uint32),
+                                      pb.cpu().numpy().view(np.uint32), 3)
+    assert np.array_equal(ssucc, esucc) and np.array_equal(solen, eolen)
     keys = torch.randint(0, 2**62, (100_003,), dtype=torch.int64, device="cuda")
     lz.sort_u64(keys)
     torch.cuda.synchronize()

@@ -239,3 +239,59 @@ def test_pruning_off_gives_full_pair_count(lz, cfg2, monkeypatch):
     assert r.stats["passes"] == 8 and r.stats["pruned_entries"] == 0
     assert r.stats["n_pairs"] == m and r.stats["n_greedy"] == acc
     assert np.array_equal(_u32(r.succ), esucc) and np.array_equal(_u8(r.olen), eolen)
+
+
+def _one_length_workspace(lz, n, L, l_min) -> int:
+    import ctypes
+    ws = ctypes.c_size_t(0)
+    lz.lasagna._check(lz.lib().lasagna_greedy_graph(None, n, L, l_min, 1, None, ctypes.byref(ws),
+                                                    None, None, None, None))
+    return int(ws.value)
+
+
+@gpu
+@pytest.mark.parametrize("frac,levels", [(0.6, ""), (0.12, ""), (0.02, ""), (0.3, "3")])
+def test_hash_range_subpasses_cfg2(lz, cfg2, monkeypatch, frac, levels):
+    """f4: a workspace below one whole length's tables makes every length run
+    in K hash-range sub-passes (the replacement of the paper's external merge, Alg. 1): the
+    graph, |P| (live pairs under pruning) and the pruned-entry count equal the oracle's."""
+    import torch
+    if levels:
+        monkeypatch.setenv("LASAGNA_TEST_LEVELS", levels)
+        monkeypatch.setenv("LASAGNA_TEST_LAST_BITS", "4")
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    one = _one_length_workspace(lz, cfg.n, cfg.L, cfg.l_min)
+    budget = int(one * frac)
+    lp, need = lz.plan(cfg.n, cfg.L, cfg.l_min, budget)
+    assert lp == 1 and need <= budget
+    runner = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda", budget_bytes=budget)
+    assert runner.ws_bytes <= budget
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = runner(packed)
+    K = r.stats["hash_subpasses"]
+    assert K > 1 and K & (K - 1) == 0, r.stats
+    assert r.stats["passes"] == K * (cfg.L - cfg.l_min)
+    assert r.stats["partition_levels"] == (3 if levels else 2)
+    assert np.array_equal(_u32(r.succ), esucc) and np.array_equal(r.olen.cpu().numpy(), eolen)
+    found, pruned = pruning_expectations(cfg.L, cfg.l_min, 1, _P2["P"], eolen)
+    assert (r.stats["n_pairs"], r.stats["pruned_entries"], r.stats["n_greedy"]) == (found, pruned, acc)
+    # the same from device ASCII (a1 fused into the first sub-pass of the first length)
+    r2 = runner.from_ascii(torch.from_numpy(reads).cuda())
+    assert np.array_equal(_u32(r2.succ), esucc) and np.array_equal(r2.olen.cpu().numpy(), eolen)
+
+
+@gpu
+def test_plan_subpasses_monotone(lz):
+    """The planner: one whole length at its exact size, then the fewest sub-passes that fit,
+    K doubling as the budget shrinks; ENOSPC only below 256 sub-passes."""
+    n, L, l_min = 2_000_000, 100, 63
+    one = _one_length_workspace(lz, n, L, l_min)
+    lp, need = lz.plan(n, L, l_min, one)
+    assert lp == 1 and need == one
+    prev = one
+    for frac in (0.7, 0.4, 0.2, 0.1, 0.05):
+        lp, need = lz.plan(n, L, l_min, int(one * frac))
+        assert lp == 1 and need <= int(one * frac) and need < prev
+        prev = need
+    lp, need = lz.plan(n, L, l_min, 1 << 20)
+    assert lp == 0 and need > 1 << 20

@@ -272,3 +272,64 @@ def test_fingerprint_collision_rate_small_modulus():
     assert abs(pairs - exp) <= 5 * exp ** 0.5, (pairs, exp)
     bad = {oracle.F(x, 4, 8192) for x in strs}
     assert len(bad) == 1
+
+
+# ---------------------------------------------------------------- approximate mode
+_CODE = {"A": 0, "C": 1, "T": 2, "G": 3}
+_COMPL = {"A": "T", "C": "G", "G": "C", "T": "A"}
+
+
+def _oriented_str(r: str, o: int) -> str:
+    return r if o == 0 else "".join(_COMPL[c] for c in reversed(r))
+
+
+def _fp_bigint(s: str, sigma: int, q: int) -> int:
+    """F(s) = sum_k c(s_k) sigma^(|s|-1-k) mod q as one Python big integer, reduced once."""
+    return sum(_CODE[c] * sigma ** (len(s) - 1 - k) for k, c in enumerate(s)) % q
+
+
+def _approx_brute(reads: list[str], l_min: int, s1, q1, s2, q2):
+    """The definition over every ordered pair of oriented reads: (l, u, v^1) for u < v^1, other
+    reads, when the suffix_l of seq(u) and the prefix_l of seq(v) have equal fingerprint pairs."""
+    L = len(reads[0])
+    seqs = [_oriented_str(reads[v >> 1], v & 1) for v in range(2 * len(reads))]
+    out = []
+    for l in range(L - 1, l_min - 1, -1):
+        pref = [(_fp_bigint(s[:l], s1, q1), _fp_bigint(s[:l], s2, q2)) for s in seqs]
+        for u, su in enumerate(seqs):
+            f = (_fp_bigint(su[L - l:], s1, q1), _fp_bigint(su[L - l:], s2, q2))
+            for v in range(len(seqs)):
+                if (u >> 1) != (v >> 1) and u < (v ^ 1) and pref[v] == f:
+                    out.append((l, u, v ^ 1))
+    return sorted(out, key=lambda t: (-t[0], t[1], t[2]))
+
+
+@pytest.mark.parametrize("case", range(9))
+def test_approx_overlaps_equal_exact_with_128bit_fingerprints(case):
+    """With the paper's two 64-bit-class fingerprints (radix 5 mod 2^61-1, radix 7 mod
+    2^64-59) the approximate pair list is the exact overlap set (brute force of strings)."""
+    reads, l_min = _tiny_instances()[case]
+    got = list(zip(*(t.tolist() for t in oracle.overlaps_approx(to_array(reads), l_min))))
+    assert got == brute.pairs(reads, l_min)
+
+
+@pytest.mark.parametrize("case,q1,q2", [(0, 11, 13), (3, 7, 5), (6, 31, 29), (8, 3, 2)])
+def test_approx_overlaps_tiny_moduli_match_definition(case, q1, q2):
+    """Deliberately tiny primes: fingerprints collide, the approximate list grows past the
+    exact one, and equals a big-integer brute force of its definition; every exact overlap is
+    in it (equal strings have equal fingerprints)."""
+    reads, l_min = _tiny_instances()[case]
+    got = list(zip(*(t.tolist() for t in oracle.overlaps_approx(to_array(reads), l_min, 7, q2, 5, q1))))
+    assert got == _approx_brute(reads, l_min, 5, q1, 7, q2)
+    exact = set(brute.pairs(reads, l_min))
+    assert exact <= set(got)
+    assert len(got) > len(exact)  # the tiny moduli do produce false pairs
+
+
+def test_approx_overlaps_cfg1_equal_exact():
+    """cfg1 reads (20 k reads, 10x): the 128-bit approximate mode finds no false pair."""
+    cfg = readgen.CONFIGS["cfg1"]
+    reads = readgen.config_reads(cfg)
+    e = oracle.overlaps(reads, cfg.l_min)
+    a = oracle.overlaps_approx(reads, cfg.l_min)
+    assert all(np.array_equal(x, y) for x, y in zip(e, a))
