@@ -110,6 +110,19 @@ LASAGNA_API lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, 
                                 uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
                                 uint64_t *n_pairs, void *stream);
 
+/* Approximate mode: as lasagna_overlaps, but a fingerprint hit is
+ * accepted when the 128-bit fingerprint pair of the suffix and the prefix agree — F (radix 5
+ * mod 2^61 - 1) and F2 (radix 7 mod 2^64 - 59, R22) — instead of the bases.  Equal
+ * strings have equal fingerprints, so every exact pair is in the result; a pair whose strings
+ * differ appears only if both fingerprints collide (none observed; the oracle's
+ * oracle_overlaps_approx is the reference, R23). */
+LASAGNA_API lasagna_status lasagna_overlaps_approx(const uint64_t *packed, uint64_t n, uint32_t L,
+                                                   uint32_t l_min, void *workspace,
+                                                   size_t *workspace_bytes, uint32_t *pair_a,
+                                                   uint32_t *pair_b, uint8_t *pair_l,
+                                                   uint64_t capacity, uint64_t *n_pairs,
+                                                   void *stream);
+
 typedef struct {
     uint64_t n_pairs;          /* |P|: read-end pairs found (overlap edges / 2)             */
     uint64_t n_greedy;         /* pairs accepted by the greedy (directed edges / 2)         */

@@ -89,6 +89,17 @@ __device__ __forceinline__ uint64_t canon_key_d1(uint64_t H, uint64_t Hr, uint64
     *d1 = (uint32_t)(m >> 56);
     return ((m << 8) & keep) | (f << vbits) | v;
 }
+// The same entry from the bucketed path's mod-2^64 key streams (fingerprint.cuh Fp64Streams,
+// reading R26): H and Hr are exact residues already.
+__device__ __forceinline__ uint64_t canon_key64_d1(uint64_t H, uint64_t Hr, uint64_t keep,
+                                                   uint32_t vbits, uint64_t v, uint32_t *d1)
+{
+    const uint64_t c = H < Hr ? H : Hr;
+    const uint64_t f = H < Hr ? 0ull : (H > Hr ? 1ull : 2ull);
+    const uint64_t m = mix(c);
+    *d1 = (uint32_t)(m >> 56);
+    return ((m << 8) & keep) | (f << vbits) | v;
+}
 __device__ __forceinline__ uint32_t key_flag(uint64_t key, uint32_t vbits)
 {
     return (uint32_t)(key >> vbits) & 3u;
@@ -208,6 +219,67 @@ __device__ __forceinline__ bool verify_overlap(const uint64_t *__restrict__ pack
 #pragma unroll
     for (int j = 0; j < W; ++j) eq &= (su[j] == sv[j]);
     return eq;
+}
+
+// ---- approximate mode ("128-bit fingerprints (two 64-bit values
+// generated with different radixes and primes)"): a hit is accepted when the fingerprint PAIR
+// of the suffix and of the prefix agree — F (radix 5 mod 2^61 - 1) and F2 (radix 7
+// mod 2^64 - 59, the largest prime below 2^64; reading R22) — instead of the bases.
+constexpr uint64_t Q2_64 = 0xFFFFFFFFFFFFFFC5ull; // 2^64 - 59
+// P * 7 + c mod Q2_64 for P < Q2_64: 2^64 == 59 (mod Q2_64)
+__device__ __forceinline__ uint64_t horner7_q2(uint64_t P, uint32_t c)
+{
+    const uint64_t lo = P * 7ull;
+    uint64_t hi = __umul64hi(P, 7ull);
+    const uint64_t t = lo + c;
+    hi += t < lo;
+    uint64_t u = t + hi * 59ull;
+    if (u < t) u += 59ull; // wrapped past 2^64
+    return u >= Q2_64 ? u - Q2_64 : u;
+}
+
+template <int W>
+__device__ __forceinline__ void fp_pair(const uint64_t (&s)[W], uint32_t l, uint64_t *f1, uint64_t *f2)
+{
+    uint64_t a = 0, b = 0;
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+        uint64_t x = s[w];
+        const uint32_t kb = 32u * w;
+        for (uint32_t j = 0; j < 32u && kb + j < l; ++j) {
+            const uint32_t c = (uint32_t)(x & 3u);
+            a = horner5(a, c);
+            b = horner7_q2(b, c);
+            x >>= 2;
+        }
+    }
+    *f1 = exact61(a);
+    *f2 = b;
+}
+// Approximate check of the directed overlap (u, v, l): F and F2 of suffix_l(seq(u)) equal F
+// and F2 of prefix_l(seq(v)) (no base comparison).
+template <int W>
+__device__ __forceinline__ bool verify_fp128(const uint64_t *__restrict__ packed, uint32_t stride,
+                                             uint32_t L, uint32_t u, uint32_t v, uint32_t l)
+{
+    uint64_t x[W], su[W], y[W], sv[W];
+    load_read<W>(packed, stride, u >> 1, x);
+    load_read<W>(packed, stride, v >> 1, y);
+    if (u & 1) rc_words<W>(x, L, su);
+    else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) su[j] = x[j];
+    }
+    if (v & 1) rc_words<W>(y, L, sv);
+    else {
+#pragma unroll
+        for (int j = 0; j < W; ++j) sv[j] = y[j];
+    }
+    shr_words<W>(su, 2u * (L - l));
+    uint64_t a1, a2, b1, b2;
+    fp_pair<W>(su, l, &a1, &a2);
+    fp_pair<W>(sv, l, &b1, &b2);
+    return a1 == b1 && a2 == b2;
 }
 
 __host__ __device__ inline uint32_t words_for(uint32_t L) { return (L + 31) / 32; }

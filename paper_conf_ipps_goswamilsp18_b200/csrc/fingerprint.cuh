@@ -44,6 +44,38 @@ struct FpStreams {
     }
 };
 
+// ---- the bucketed path's table keys: the same radix-5 Rabin-Karp polynomial evaluated modulo
+// 2^64 (reading R26).  The keys only have to bring equal strings together — every hit is
+// verified on the bases (R12) — and modulo 2^64 a step is two multiply-adds on the FMA pipe
+// instead of the shifts, folds and exact reductions of mod 2^61 - 1 on the integer ALU pipe,
+// which bounds the scatter kernel (ncu: ALU pipe 67 % of peak, FMA 17 %).
+struct Pow64Table {
+    uint64_t m[256];
+};
+constexpr Pow64Table make_pow64_table()
+{
+    Pow64Table t{};
+    uint64_t p = 1;
+    for (int j = 0; j < 256; ++j) {
+        t.m[j] = p;
+        p *= 5u;
+    }
+    return t;
+}
+static __constant__ Pow64Table c_pow64 = make_pow64_table();
+
+struct Fp64Streams {
+    uint64_t P0, P1, S0, S1; // exact values mod 2^64
+    __device__ __forceinline__ void step(uint32_t ca, uint32_t cb, uint32_t j)
+    {
+        const uint64_t pw = c_pow64.m[j];
+        P0 = P0 * 5u + ca;
+        P1 = P1 * 5u + cb;
+        S1 += (uint64_t)(ca ^ 2u) * pw;
+        S0 += (uint64_t)(cb ^ 2u) * pw;
+    }
+};
+
 // ---- absorbing a read's leading bases without per-base modular steps
 // Lengths below the first one a kernel emits need no intermediate values, only the stream
 // states after them, so whole 16-base half-words are absorbed in 8-base chunks: the chunk's
@@ -175,6 +207,65 @@ __device__ __forceinline__ void fp_absorb(const uint64_t (&x)[W], const uint64_t
         S0 = mulsmall61(S0, POW5_8) + chunk8_bwd(hy);
     }
     st.P0 = fold61(P0), st.P1 = fold61(P1), st.S0 = fold61(S0), st.S1 = fold61(S1);
+}
+
+// fp_absorb modulo 2^64 (the key streams of the bucketed path, R26)
+template <int W>
+__device__ __forceinline__ void fp64_absorb(const uint64_t (&x)[W], const uint64_t (&y)[W],
+                                          uint32_t nb, Fp64Streams &st)
+{
+    const uint32_t nh = nb >> 4, rem = nb & 15u;
+    uint64_t P0 = 0, P1 = 0, S0 = 0, S1 = 0;
+#pragma unroll
+    for (int h = 0; h < 2 * W; ++h) {
+        if ((uint32_t)h >= nh) break;
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1)));
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1)));
+        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd(hx);
+        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd(hx >> 16);
+        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd(hy);
+        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd(hy >> 16);
+    }
+    // the partial half-word nh (bases 16 nh .. 16 nh + rem - 1), rem < 16
+    uint32_t px = 0, py = 0;
+    if (rem) {
+        px = (uint32_t)(wsel<W>(x, nh >> 1) >> (32 * (nh & 1)));
+        py = (uint32_t)(wsel<W>(y, nh >> 1) >> (32 * (nh & 1)));
+        const uint32_t mask = rem == 16 ? 0xFFFFFFFFu : ((1u << (2 * rem)) - 1u);
+        px &= mask;
+        py &= mask;
+        const uint32_t k1 = min(rem, 8u), k2 = rem - k1; // forward: low chunk first
+        const uint32_t m1 = pow5_small(k1);
+        P0 = (P0) * (uint64_t)(m1) + chunk8_fwd((px & 0xFFFFu) << (2 * (8 - k1)));
+        P1 = (P1) * (uint64_t)(m1) + chunk8_fwd((py & 0xFFFFu) << (2 * (8 - k1)));
+        if (k2) {
+            const uint32_t m2 = pow5_small(k2);
+            P0 = (P0) * (uint64_t)(m2) + chunk8_fwd(((px >> 16) << (2 * (8 - k2))) & 0xFFFFu);
+            P1 = (P1) * (uint64_t)(m2) + chunk8_fwd(((py >> 16) << (2 * (8 - k2))) & 0xFFFFu);
+        }
+        // ascending-power streams: the partial (highest) bases first, high chunk first
+        const uint32_t cx = px ^ (0xAAAAAAAAu & mask), cy = py ^ (0xAAAAAAAAu & mask);
+        if (k2) {
+            S1 = chunk8_bwd(cx >> 16);
+            S0 = chunk8_bwd(cy >> 16);
+            S1 = (S1) * (uint64_t)(m1) + chunk8_bwd(cx & 0xFFFFu);
+            S0 = (S0) * (uint64_t)(m1) + chunk8_bwd(cy & 0xFFFFu);
+        } else {
+            S1 = chunk8_bwd(cx & 0xFFFFu);
+            S0 = chunk8_bwd(cy & 0xFFFFu);
+        }
+    }
+#pragma unroll
+    for (int h = 2 * W - 1; h >= 0; --h) {
+        if ((uint32_t)h >= nh) continue;
+        const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
+        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd(hx >> 16);
+        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd(hx);
+        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd(hy >> 16);
+        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd(hy);
+    }
+    st.P0 = P0, st.P1 = P1, st.S0 = S0, st.S1 = S1;
 }
 
 // half-words a kernel whose first emitted length is l_first can absorb (bases < l_first - 1)

@@ -53,7 +53,7 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
         return;
     }
     // staging full: verify inline and emit straight to global memory
-    if (!verify_overlap<W>(a.packed, a.stride, a.L, lo, hi ^ 1u, a.l)) {
+    if (!verify_pair<W>(a, lo, hi ^ 1u)) {
         ++nfalse;
         return;
     }
@@ -74,7 +74,7 @@ __device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long l
     for (uint32_t t = from + threadIdx.x; t < to; t += NT) {
         const unsigned long long rec = buf[t];
         const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
-        if (!verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
+        if (!verify_pair<W>(a, u, b ^ 1u)) {
             buf[t] = ~0ull;
             ++nfalse;
             continue;

@@ -58,7 +58,17 @@ struct JoinArgs {
     // (bitmap) are counted in *found but not stored — they can never be accepted
     const uint32_t *claimed = nullptr;
     unsigned long long *found = nullptr;
+    // approximate mode: hits are accepted by the 128-bit fingerprint
+    // pair (common.cuh verify_fp128) instead of the bases
+    bool approx = false;
 };
+// the check a hit passes: bases (exact) or the fingerprint pair (approximate mode)
+template <int W>
+__device__ __forceinline__ bool verify_pair(const JoinArgs &a, uint32_t u, uint32_t v)
+{
+    return a.approx ? verify_fp128<W>(a.packed, a.stride, a.L, u, v, a.l)
+                    : verify_overlap<W>(a.packed, a.stride, a.L, u, v, a.l);
+}
 lasagna_status launch_join(const JoinArgs &a, cudaStream_t s);
 lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsigned long long *count,
                                     uint64_t m, unsigned long long cap, uint32_t vbits,

@@ -262,6 +262,7 @@ struct Run {
     unsigned long long *pool, *pool2;
     const uint32_t *claimed = nullptr; // greedy mode: the join drops pairs with a claimed end
     bool prune = false; // this group's scatter drops entries whose read end is claimed (f1)
+    bool approx = false; // f4: hits accepted by the 128-bit fingerprint pair
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
     void bind(void *workspace)
     {
@@ -551,6 +552,7 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.false_matches = r.ctr64 + CTR_FALSE;
     ja.claimed = join_filter() ? r.claimed : nullptr;
     ja.found = ja.claimed ? r.ctr64 + CTR_FOUND : nullptr;
+    ja.approx = r.approx;
     lasagna_status rc;
     if (r.bucketed) {
         BucketJoinArgs bj;
@@ -962,12 +964,36 @@ lasagna_status lasagna_greedy_graph_ascii(const char *ascii, uint64_t n, uint32_
                              stream);
 }
 
+static lasagna_status overlaps_impl(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                    void *workspace, size_t *workspace_bytes, uint32_t *pair_a,
+                                    uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
+                                    uint64_t *n_pairs, void *stream, bool approx);
+
 lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
                                 void *workspace, size_t *workspace_bytes, uint32_t *pair_a,
                                 uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
                                 uint64_t *n_pairs, void *stream)
 {
     g_err[0] = 0;
+    return overlaps_impl(packed, n, L, l_min, workspace, workspace_bytes, pair_a, pair_b, pair_l,
+                         capacity, n_pairs, stream, false);
+}
+
+lasagna_status lasagna_overlaps_approx(const uint64_t *packed, uint64_t n, uint32_t L,
+                                       uint32_t l_min, void *workspace, size_t *workspace_bytes,
+                                       uint32_t *pair_a, uint32_t *pair_b, uint8_t *pair_l,
+                                       uint64_t capacity, uint64_t *n_pairs, void *stream)
+{
+    g_err[0] = 0;
+    return overlaps_impl(packed, n, L, l_min, workspace, workspace_bytes, pair_a, pair_b, pair_l,
+                         capacity, n_pairs, stream, true);
+}
+
+static lasagna_status overlaps_impl(const uint64_t *packed, uint64_t n, uint32_t L, uint32_t l_min,
+                                    void *workspace, size_t *workspace_bytes, uint32_t *pair_a,
+                                    uint32_t *pair_b, uint8_t *pair_l, uint64_t capacity,
+                                    uint64_t *n_pairs, void *stream, bool approx)
+{
     lasagna_status rc = check_shape(n, L, l_min);
     if (rc != LASAGNA_OK) return rc;
     if (!workspace_bytes || !n_pairs) {
@@ -1005,6 +1031,7 @@ lasagna_status lasagna_overlaps(const uint64_t *packed, uint64_t n, uint32_t L, 
     r.lay = layout(g, G, cap, false);
     r.s = s;
     r.bind(workspace);
+    r.approx = approx;
   for (int attempt = 0; attempt < 2; ++attempt) {
     r.bucketed = attempt == 0 && use_bucketed(g);
     PhaseTimer tm;

@@ -264,9 +264,9 @@ scatter_table_kernel(ScatterArgs a)
                                                           (a.l_hi - a.l_lo + 1u) * a.nb_pad));
     __syncthreads();
     const uint64_t v0 = 2 * (a.read_offset + i);
-    FpStreams st;
+    Fp64Streams st; // key streams modulo 2^64 (R26)
     // the l_lo - 1 bases before the first emitted length, absorbed in 8-base chunks
-    fp_absorb<W>(x, y, a.l_lo - 1u, st);
+    fp64_absorb<W>(x, y, a.l_lo - 1u, st);
     // Base cursors over x (y is dead from here): tx holds base k of r in its low bits; ty
     // holds base L-1-k of r in its top bits, i.e. base k of r' = RC(r) complemented.  A word
     // boundary reloads a cursor from x with a register select (block-uniform branch).
@@ -308,8 +308,8 @@ scatter_table_kernel(ScatterArgs a)
             rk[2 * q] = rk[2 * q + 1] = ~0u; // no key (pruned or no read)
             if (live0 | live1) {
                 uint32_t d0, d1; // level-1 digits (implied by the region, not stored)
-                const uint64_t e0 = canon_key_d1(st.P0, st.S1, a.keep, a.vbits, v0, &d0);
-                const uint64_t e1 = canon_key_d1(st.P1, st.S0, a.keep, a.vbits, v0 + 1, &d1);
+                const uint64_t e0 = canon_key64_d1(st.P0, st.S1, a.keep, a.vbits, v0, &d0);
+                const uint64_t e1 = canon_key64_d1(st.P1, st.S0, a.keep, a.vbits, v0 + 1, &d1);
                 if constexpr (SPLIT) {
                     d0 = (d0 << 1) | (uint32_t)((e0 >> a.vbits) & 1);
                     d1 = (d1 << 1) | (uint32_t)((e1 >> a.vbits) & 1);

@@ -51,7 +51,7 @@ __device__ __forceinline__ void wj_flush(const JoinArgs &a, WarpSlice &S, unsign
         if (t < n) {
             rec = S.cand[t];
             const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
-            if (verify_overlap<W>(a.packed, a.stride, a.L, u, b ^ 1u, a.l)) {
+            if (verify_pair<W>(a, u, b ^ 1u)) {
                 keep = true;
                 if (a.found) atomicAdd(a.found, 1ull);
                 if (a.claimed && (((a.claimed[u >> 5] >> (u & 31u)) | (a.claimed[b >> 5] >> (b & 31u))) & 1u))
@@ -94,7 +94,7 @@ __device__ __forceinline__ void wj_probe(const JoinArgs &a, WarpSlice &S, const 
                 const uint32_t slot = atomicAdd(&S.ncand, 1u);
                 if (slot < (uint32_t)WJ_CAND) {
                     S.cand[slot] = rec;
-                } else if (!verify_overlap<W>(a.packed, a.stride, a.L, min(x, y), max(x, y) ^ 1u, a.l)) {
+                } else if (!verify_pair<W>(a, min(x, y), max(x, y) ^ 1u)) {
                     ++nfalse; // buffer full (rare): verify inline, emit straight to the pool
                 } else {
                     if (a.found) atomicAdd(a.found, 1ull);

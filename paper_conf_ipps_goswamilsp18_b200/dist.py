@@ -398,140 +398,186 @@ class _Phases:
         return out
 
 
-def greedy_graph_fast(ascii_local: torch.Tensor, n_total: int, L: int, l_min: int, group=None,
-                      lengths_per_pass: int = 0, pair_capacity: int | None = None,
-                      timing: bool = False):
-    """Greedy string graph over the ranks of `group` on the bucketed kernels (include/lasagna.h
-    "Sharded FAST path"): per length group one fused scatter of the local reads, two equal-split
-    all-to-alls, the multi-source refine, then per length the join and the sharded greedy over
-    peer memory.  No host synchronisation between the first scatter and the end of the call.
-    Rank r holds reads fast_shard_range(n_total, g, r).  Returns (succ, olen, stats), identical
-    on every rank."""
-    world = dist.get_world_size(group)
-    rank = dist.get_rank(group)
-    Lb = lz.lib()
-    dev = ascii_local.device if ascii_local.is_cuda else torch.device("cuda", torch.cuda.current_device())
-    geo = shard_geometry(n_total, world, L, l_min)
-    lo, hi, n_pad = fast_shard_range(n_total, world, rank)
-    assert n_pad == geo.n_pad and ascii_local.shape[0] == hi - lo, (n_pad, geo.n_pad, ascii_local.shape)
-    n_local = hi - lo
-    s = lz._stream(dev)
-    C = _Coll(group, dev)
-    W = lz.words_per_read(L)
-    # 1. packed reads: local pack, all-gather (padded slices) -> every rank verifies any hit
-    buf = torch.zeros((n_pad, W), dtype=torch.int64, device=dev)
-    if n_local:
-        buf[:n_local] = lz.load_reads(ascii_local, device=dev)
-    packed_all = torch.empty(world * n_pad * W, dtype=torch.int64, device=dev)
-    C.all_gather_into_tensor(packed_all, buf.reshape(-1))
-    packed_all = packed_all.view(world * n_pad, W)
-    packed_local = packed_all[lo:lo + n_pad]
-    n_len = L - l_min
-    G = n_len if lengths_per_pass <= 0 else min(lengths_per_pass, n_len)
-    G = min(G, 64)
-    cap = pair_capacity if pair_capacity is not None else max(1 << 20, (2 * n_total) // 8)
-    pool = torch.empty(cap, dtype=torch.int64, device=dev)
-    pool2 = torch.empty(cap, dtype=torch.int64, device=dev)
-    pool_count = torch.zeros(1, dtype=torch.int64, device=dev)
-    counters = torch.zeros(4, dtype=torch.int64, device=dev)
-    arena = PeerArena(int(geo.slice), dev, group)
-    ph = _Phases(timing)
-    try:
-        ranks = (lz.GreedyRank * world)()
-        for q in range(world):
-            ranks[q].ctr = arena.ptr(q, "ctr")
-            ranks[q].best = arena.ptr(q, "best")
-            ranks[q].claimed = arena.ptr(q, "claimed")
-            ranks[q].succ = arena.ptr(q, "succ")
-            ranks[q].olen = arena.ptr(q, "olen")
-            ranks[q].tail = arena.ptr(q, "tail")
-        ranks[rank].pool = pool.data_ptr()
-        ranks[rank].pool2 = pool2.data_ptr()
-        ranks[rank].pool_count = pool_count.data_ptr()
-        claimed_mine = arena.ptr(rank, "claimed")
+class ShardedGraph:
+    """Reusable runner of the sharded fast path (include/lasagna.h "Sharded FAST path"): the
+    peer arena (opened by every rank once), the pair pools, the packed-read buffer and the
+    exchange / partition buffers are allocated once and kept across calls.  Per call: one fused
+    scatter of the local reads per length group, two equal-split all-to-alls, the multi-source
+    refine, then per length the join and the sharded greedy over peer memory — no host
+    synchronisation until the end of the call.  Rank r holds reads fast_shard_range(n, g, r)."""
+
+    def __init__(self, n_total: int, L: int, l_min: int, group=None, device=None,
+                 lengths_per_pass: int = 0, pair_capacity: int | None = None):
+        self.n, self.L, self.l_min, self.group = n_total, L, l_min, group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.dev = torch.device(device) if device is not None else \
+            torch.device("cuda", torch.cuda.current_device())
+        self.Lb = lz.lib()
+        self.geo = shard_geometry(n_total, self.world, L, l_min)
+        self.lo, self.hi, n_pad = fast_shard_range(n_total, self.world, self.rank)
+        assert n_pad == self.geo.n_pad, (n_pad, self.geo.n_pad)
+        self.n_local = self.hi - self.lo
+        n_len = L - l_min
+        G = n_len if lengths_per_pass <= 0 else min(lengths_per_pass, n_len)
+        self.G = min(G, 64)
+        self.W = lz.words_per_read(L)
+        self.cap = pair_capacity if pair_capacity is not None else max(1 << 20, (2 * n_total) // 8)
+        dev = self.dev
+        self.coll = _Coll(group, dev)
+        self.packed_all = torch.zeros((self.world * n_pad, self.W), dtype=torch.int64, device=dev)
+        self.pool = torch.empty(self.cap, dtype=torch.int64, device=dev)
+        self.pool2 = torch.empty(self.cap, dtype=torch.int64, device=dev)
+        self.pool_count = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.counters = torch.zeros(4, dtype=torch.int64, device=dev)
+        self.send = torch.empty(self.G * self.geo.send_entries, dtype=torch.int64, device=dev)
+        self.send_fill = torch.empty(self.G * self.geo.fill_words, dtype=torch.int32, device=dev)
+        # one rank: the exchange is the identity (no copy)
+        self.recv = torch.empty_like(self.send) if self.world > 1 else self.send
+        self.recv_fill = torch.empty_like(self.send_fill) if self.world > 1 else self.send_fill
+        nbytes = ctypes.c_size_t(0)
+        lz._check(self.Lb.lasagna_shard_part_bytes(n_total, self.world, L, l_min, self.G,
+                                                   ctypes.byref(nbytes)))
+        self.part = lz._workspace(nbytes.value, dev)
+        self.arena = PeerArena(int(self.geo.slice), dev, group)
+        ranks = (lz.GreedyRank * self.world)()
+        for q in range(self.world):
+            for f in ("ctr", "best", "claimed", "succ", "olen", "tail"):
+                setattr(ranks[q], f, self.arena.ptr(q, f))
+        ranks[self.rank].pool = self.pool.data_ptr()
+        ranks[self.rank].pool2 = self.pool2.data_ptr()
+        ranks[self.rank].pool_count = self.pool_count.data_ptr()
+        self.ranks = ranks
+        self.succ_all = torch.empty(self.world * int(self.geo.slice), dtype=torch.int32, device=dev)
+        self.olen_all = torch.empty(self.world * int(self.geo.slice), dtype=torch.uint8, device=dev)
+
+    def close(self):
+        if self.arena is not None:
+            self.arena.close()
+            self.arena = None
+
+    def __call__(self, ascii_local: torch.Tensor, timing: bool = False):
+        """(succ int32 [2n], olen uint8 [2n], stats) of the whole read set, identical on every
+        rank; ascii_local: this rank's (n_local, L) uint8 reads (device, or host: copied in)."""
+        n_total, L, l_min, world, rank = self.n, self.L, self.l_min, self.world, self.rank
+        geo, Lb, dev, C = self.geo, self.Lb, self.dev, self.coll
+        assert ascii_local.shape[0] == self.n_local, (ascii_local.shape, self.n_local)
+        s = lz._stream(dev)
+        ph = _Phases(timing)
+        n_pad, lo, n_local, cap = int(geo.n_pad), self.lo, self.n_local, self.cap
+        # per call: fresh greedy state in the arena, zeroed counters
+        self.arena.view.zero_()
+        self.arena.tensor("succ", torch.int32).fill_(-1)
+        self.counters.zero_()
+        # 1. packed reads: local pack into my slice, all-gather -> every rank verifies any hit
+        mine = self.packed_all[rank * n_pad:(rank + 1) * n_pad]
+        if n_local:
+            mine[:n_local] = lz.load_reads(ascii_local.to(dev, non_blocking=True), device=dev)
+        if world > 1:
+            C.all_gather_into_tensor(self.packed_all.view(-1), mine.reshape(-1).clone())
+        packed_all = self.packed_all
+        packed_local = mine
+        claimed_mine = self.arena.ptr(rank, "claimed")
+        G = self.G
         first = True
         for l_hi in range(L - 1, l_min - 1, -G):
             l_lo = max(l_min, l_hi - G + 1)
             Gc = l_hi - l_lo + 1
+            send = self.send[:Gc * geo.send_entries]
+            send_fill = self.send_fill[:Gc * geo.fill_words]
             # 2. a1..a3 + level 1 of my reads, regions in shard order (pruned after group 1)
-            send = torch.empty(Gc * geo.send_entries, dtype=torch.int64, device=dev)
-            send_fill = torch.empty(Gc * geo.fill_words, dtype=torch.int32, device=dev)
             t = ph.start("scatter")
             lz._check(Lb.lasagna_shard_scatter(
                 lz._ptr(packed_local), n_local, lo, n_total, world, L, l_min, l_lo, l_hi,
                 None if first else ctypes.c_void_p(claimed_mine), lz._ptr(send),
-                lz._ptr(send_fill), lz._ptr(counters), s))
+                lz._ptr(send_fill), lz._ptr(self.counters), s))
             ph.stop(t)
             ph.launches["scatter"] += 1
             first = False
             # 3. the hash-range shuffle: equal split sizes, nothing to count or synchronise
-            recv = torch.empty_like(send)
-            recv_fill = torch.empty_like(send_fill)
-            t = ph.start("exchange")
-            C.all_to_all_single(recv, send)
-            C.all_to_all_single(recv_fill, send_fill)
-            ph.stop(t)
-            del send, send_fill
-            nbytes = ctypes.c_size_t(0)
-            lz._check(Lb.lasagna_shard_part_bytes(n_total, world, L, l_min, Gc, ctypes.byref(nbytes)))
-            part = lz._workspace(nbytes.value, dev)
+            recv = self.recv[:Gc * geo.send_entries]
+            recv_fill = self.recv_fill[:Gc * geo.fill_words]
+            if world > 1:
+                t = ph.start("exchange")
+                C.all_to_all_single(recv, send)
+                C.all_to_all_single(recv_fill, send_fill)
+                ph.stop(t)
             t = ph.start("refine")
             lz._check(Lb.lasagna_shard_partition(lz._ptr(recv), lz._ptr(recv_fill), n_total, world,
-                                                 L, l_min, l_lo, l_hi, lz._ptr(part),
-                                                 lz._ptr(counters), s))
+                                                 L, l_min, l_lo, l_hi, lz._ptr(self.part),
+                                                 lz._ptr(self.counters), s))
             ph.stop(t)
             ph.launches["refine"] += int(geo.levels) - 1
-            del recv, recv_fill
             # 4. per length: join (my buckets) and the sharded greedy (everyone's pairs)
             for l in range(l_hi, l_lo - 1, -1):
                 t = ph.start("join")
-                lz._check(Lb.lasagna_shard_join(lz._ptr(part), n_total, world, L, l_min, l_lo,
-                                                l_hi, l, lz._ptr(packed_all), lz._ptr(pool), cap,
-                                                lz._ptr(pool_count), lz._ptr(counters), s))
+                lz._check(Lb.lasagna_shard_join(lz._ptr(self.part), n_total, world, L, l_min, l_lo,
+                                                l_hi, l, lz._ptr(packed_all), lz._ptr(self.pool),
+                                                cap, lz._ptr(self.pool_count),
+                                                lz._ptr(self.counters), s))
                 ph.stop(t)
                 t = ph.start("greedy")
-                lz._check(Lb.lasagna_greedy_shard_length(ranks, world, rank, int(geo.slice), cap,
-                                                         l, s))
+                lz._check(Lb.lasagna_greedy_shard_length(self.ranks, world, rank, int(geo.slice),
+                                                         cap, l, s))
                 ph.stop(t)
                 ph.launches["join"] += 1
                 ph.launches["greedy_lengths"] += 1
-            del part
-        # 5. outcome: region overflow or pool overflow anywhere -> every rank reruns
-        ctr = arena.tensor("ctr", torch.int64)
-        flags = torch.stack([counters[0].clamp(max=1), ctr[5]]).to(torch.int64)
+        # 5. outcome: region or pool overflow anywhere -> every rank reruns
+        ctr = self.arena.tensor("ctr", torch.int64)
+        flags = torch.stack([self.counters[0].clamp(max=1), ctr[5]]).to(torch.int64)
         C.all_reduce(flags, op=dist.ReduceOp.MAX)
         ovf, max_pl = (int(x) for x in flags.tolist())
         if ovf:
             raise RegionOverflow("a slack region overflowed")
         if max_pl > cap:
-            need = max_pl * 5 // 4 + 1
+            raise PoolOverflow(max_pl)
+        # the graph: every rank's slices of succ/olen, all-gathered
+        if world > 1:
+            C.all_gather_into_tensor(self.succ_all, self.arena.tensor("succ", torch.int32).clone())
+            C.all_gather_into_tensor(self.olen_all, self.arena.tensor("olen", torch.uint8).clone())
         else:
-            need = 0
-            # the graph: every rank's slices of succ/olen, all-gathered
-            slice_ = int(geo.slice)
-            succ_all = torch.empty(world * slice_, dtype=torch.int32, device=dev)
-            olen_all = torch.empty(world * slice_, dtype=torch.uint8, device=dev)
-            C.all_gather_into_tensor(succ_all, arena.tensor("succ", torch.int32).clone())
-            C.all_gather_into_tensor(olen_all, arena.tensor("olen", torch.uint8).clone())
-            tot = torch.stack([ctr[4], ctr[3], counters[1], counters[3]]).clone()
-            C.all_reduce(tot)
-            mx = ctr[6:7].clone()
-            C.all_reduce(mx, op=dist.ReduceOp.MAX)
-            n_pairs, n_greedy, pruned, false_m = (int(x) for x in tot.tolist())
-            stats = {"n_pairs": n_pairs, "n_greedy": n_greedy, "pruned_entries": pruned,
-                     "fp_false_matches": false_m, "rounds_max": int(mx.item()),
-                     "lengths_per_pass": G, "partition_levels": int(geo.levels), "path": "fast",
-                     "greedy_pair_rounds": int(ctr[7].item()), "n_local": n_local,
-                     "launches": dict(ph.launches)}
-            if timing:
-                torch.cuda.synchronize()
-                stats["ms"] = ph.totals()
-            out = (succ_all[:2 * n_total], olen_all[:2 * n_total], stats)
-    finally:
-        arena.close()
-    if need:
-        return greedy_graph_fast(ascii_local, n_total, L, l_min, group, lengths_per_pass, need)
-    return out
+            self.succ_all.copy_(self.arena.tensor("succ", torch.int32))
+            self.olen_all.copy_(self.arena.tensor("olen", torch.uint8))
+        tot = torch.stack([ctr[4], ctr[3], self.counters[1], self.counters[3]]).clone()
+        C.all_reduce(tot)
+        mx = ctr[6:7].clone()
+        C.all_reduce(mx, op=dist.ReduceOp.MAX)
+        n_pairs, n_greedy, pruned, false_m = (int(x) for x in tot.tolist())
+        stats = {"n_pairs": n_pairs, "n_greedy": n_greedy, "pruned_entries": pruned,
+                 "fp_false_matches": false_m, "rounds_max": int(mx.item()),
+                 "lengths_per_pass": G, "partition_levels": int(geo.levels), "path": "fast",
+                 "greedy_pair_rounds": int(ctr[7].item()), "n_local": n_local,
+                 "launches": dict(ph.launches)}
+        if timing:
+            torch.cuda.synchronize()
+            stats["ms"] = ph.totals()
+        return self.succ_all[:2 * n_total], self.olen_all[:2 * n_total], stats
+
+
+class PoolOverflow(RuntimeError):
+    """A length produced more candidate pairs than the pool holds (rerun with a larger one)."""
+
+    def __init__(self, need: int):
+        super().__init__(f"a length produced {need} pairs")
+        self.need = need
+
+
+def greedy_graph_fast(ascii_local: torch.Tensor, n_total: int, L: int, l_min: int, group=None,
+                      lengths_per_pass: int = 0, pair_capacity: int | None = None,
+                      timing: bool = False):
+    """One call of the sharded fast path (a ShardedGraph built, run and closed); a pool
+    overflow reruns with a pool 1.25x the largest length.  Returns (succ, olen, stats)."""
+    dev = ascii_local.device if ascii_local.is_cuda else None
+    for _ in range(2):
+        g = ShardedGraph(n_total, L, l_min, group, dev, lengths_per_pass, pair_capacity)
+        try:
+            succ, olen, st = g(ascii_local, timing)
+            return succ.clone(), olen.clone(), st
+        except PoolOverflow as e:
+            pair_capacity = e.need * 5 // 4 + 1
+        finally:
+            g.close()
+    raise RuntimeError("sharded fast path: pool overflow after a resize")
 
 
 def lz_words(L: int) -> int:
@@ -606,11 +652,11 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
     be = CudaBackend(dev)
     stream = torch.cuda.current_stream(dev)
 
+    runner = ShardedGraph(n, L, l_min, None, dev, args.lengths_per_pass) if fast else None
+
     def step(src, d2h: bool, timing: bool = False):
         if fast:
-            succ, olen, st = greedy_graph_fast(src.to(dev, non_blocking=True), n, L, l_min,
-                                               lengths_per_pass=args.lengths_per_pass,
-                                               timing=timing)
+            succ, olen, st = runner(src, timing=timing)
         else:
             succ, olen, st = greedy_graph(src, n, L, l_min, be,
                                           lengths_per_pass=args.lengths_per_pass)
@@ -675,5 +721,7 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
         if world == 1 and not getattr(args, "no_cpu_baseline", False):
             out["cpu_baseline"] = cpu_baseline(cfg, host.numpy())
         print(json.dumps(out), flush=True)
+    if runner is not None:
+        runner.close()
     dist.barrier()
     dist.destroy_process_group()

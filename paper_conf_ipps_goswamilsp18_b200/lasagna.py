@@ -88,6 +88,7 @@ def lib() -> ctypes.CDLL:
         "lasagna_load_reads": [vp, u64, u32, vp, vp, vp],
         "lasagna_fingerprints": [vp, u64, u32, u32, vp, vp, vp],
         "lasagna_overlaps": [vp, u64, u32, u32, vp, psz, vp, vp, vp, u64, pu64, vp],
+        "lasagna_overlaps_approx": [vp, u64, u32, u32, vp, psz, vp, vp, vp, u64, pu64, vp],
         "lasagna_greedy_graph": [vp, u64, u32, u32, u32, vp, psz, vp, vp,
                                  ctypes.POINTER(_Stats), vp],
         "lasagna_greedy_graph_ascii": [vp, u64, u32, u32, u32, vp, psz, vp, vp, vp, vp,
@@ -181,24 +182,26 @@ def fingerprints(packed: torch.Tensor, n: int, L: int, l_min: int):
 
 
 # ---------------------------------------------------------------------------- a2..a5
-def overlaps(packed: torch.Tensor, n: int, L: int, l_min: int, capacity: int | None = None):
+def overlaps(packed: torch.Tensor, n: int, L: int, l_min: int, capacity: int | None = None,
+             approx: bool = False):
     """All read-end pairs sorted by (l desc, a, b): (pl uint8, pa int32, pb int32) tensors
-    (pa/pb hold u32 vertex ids)."""
+    (pa/pb hold u32 vertex ids).  approx: the paper's 128-bit fingerprint acceptance
+    (lasagna_overlaps_approx) instead of the exact base comparison."""
     dev = packed.device
+    fn = lib().lasagna_overlaps_approx if approx else lib().lasagna_overlaps
     ws_bytes = ctypes.c_size_t(0)
     npairs = ctypes.c_uint64(0)
     with torch.cuda.device(dev):
-        _check(lib().lasagna_overlaps(_ptr(packed), n, L, l_min, None, ctypes.byref(ws_bytes),
-                                      None, None, None, 0, ctypes.byref(npairs), _stream(dev)))
+        _check(fn(_ptr(packed), n, L, l_min, None, ctypes.byref(ws_bytes), None, None, None, 0,
+                  ctypes.byref(npairs), _stream(dev)))
         for _ in range(4):
             ws = _workspace(ws_bytes.value, dev)
             cap = max(1, int(capacity if capacity is not None else max(1, n)))
             pa = torch.empty(cap, dtype=torch.int32, device=dev)
             pb = torch.empty(cap, dtype=torch.int32, device=dev)
             pl = torch.empty(cap, dtype=torch.uint8, device=dev)
-            st = lib().lasagna_overlaps(_ptr(packed), n, L, l_min, _ptr(ws), ctypes.byref(ws_bytes),
-                                        _ptr(pa), _ptr(pb), _ptr(pl), cap, ctypes.byref(npairs),
-                                        _stream(dev))
+            st = fn(_ptr(packed), n, L, l_min, _ptr(ws), ctypes.byref(ws_bytes), _ptr(pa),
+                    _ptr(pb), _ptr(pl), cap, ctypes.byref(npairs), _stream(dev))
             if st == ENOSPC:
                 if npairs.value > cap:
                     capacity = npairs.value

@@ -19,15 +19,26 @@ def main():
     reads = readgen.reads(20181, 60_000, n, L, 0.01)
     esucc, eolen, m, acc = oracle.greedy_graph(reads, l_min)
     packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    quick = bool(os.environ.get("SANITIZE_QUICK"))  # racecheck: one geometry, fewer calls
+    envs = ({"LASAGNA_TEST_LEVELS": "2"},) if quick else (
+        {}, {"LASAGNA_TEST_LEVELS": "2"}, {"LASAGNA_TEST_LEVELS": "3", "LASAGNA_TEST_LAST_BITS": "2"},
+        {"LASAGNA_PATH": "exact"})
     # bucketed one level (T = 8), forced two and three levels, the exact path
-    for env in ({}, {"LASAGNA_TEST_LEVELS": "2"}, {"LASAGNA_TEST_LEVELS": "3", "LASAGNA_TEST_LAST_BITS": "2"},
-                {"LASAGNA_PATH": "exact"}):
+    for env in envs:
         os.environ.update(env)
         r = lz.greedy_graph(packed, n, L, l_min, lengths_per_pass=5)
         assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), esucc), env
         assert np.array_equal(r.olen.cpu().numpy(), eolen), env
         for k in env:
             del os.environ[k]
+    if quick:
+        from tests.test_gpu_sharded import _sharded_greedy
+        pl, pa, pb = lz.overlaps(packed, n, L, l_min)
+        ssucc, solen, _ = _sharded_greedy(n, pl.cpu().numpy(), pa.cpu().numpy().view(np.uint32),
+                                          pb.cpu().numpy().view(np.uint32), 2)
+        assert np.array_equal(ssucc, esucc) and np.array_equal(solen, eolen)
+        print("sanitize driver ok (quick)")
+        return
     # fused a1 from device and pinned ASCII (two levels)
     os.environ["LASAGNA_TEST_LEVELS"] = "2"
     g = lz.GreedyGraph(n, L, l_min, "cuda", lengths_per_pass=7)
@@ -49,7 +60,8 @@ def main():
     lz.lasagna._check(lz.lib().lasagna_greedy_graph(None, n, L, l_min, 1, None, ctypes.byref(ws),
                                                     None, None, None, None))
     os.environ["LASAGNA_TEST_LEVELS"] = "2"
-    sub = lz.GreedyGraph(n, L, l_min, "cuda", budget_bytes=int(ws.value * 0.3))
+    _, least = lz.plan(n, L, l_min, 1)
+    sub = lz.GreedyGraph(n, L, l_min, "cuda", budget_bytes=least + (int(ws.value) - least) // 4)
     r = sub(packed)
     assert r.stats["hash_subpasses"] > 1, r.stats
     assert np.array_equal(r.succ.cpu().numpy().view(np.uint32), esucc)

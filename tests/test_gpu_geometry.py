@@ -250,7 +250,7 @@ def _one_length_workspace(lz, n, L, l_min) -> int:
 
 
 @gpu
-@pytest.mark.parametrize("frac,levels", [(0.6, ""), (0.12, ""), (0.02, ""), (0.3, "3")])
+@pytest.mark.parametrize("frac,levels", [(0.6, ""), (0.12, ""), (0.0, ""), (0.3, "3")])
 def test_hash_range_subpasses_cfg2(lz, cfg2, monkeypatch, frac, levels):
     """f4: a workspace below one whole length's tables makes every length run
     in K hash-range sub-passes (the replacement of the paper's external merge, Alg. 1): the
@@ -261,7 +261,8 @@ def test_hash_range_subpasses_cfg2(lz, cfg2, monkeypatch, frac, levels):
         monkeypatch.setenv("LASAGNA_TEST_LAST_BITS", "4")
     cfg, reads, esucc, eolen, m, acc = cfg2
     one = _one_length_workspace(lz, cfg.n, cfg.L, cfg.l_min)
-    budget = int(one * frac)
+    _, least = lz.plan(cfg.n, cfg.L, cfg.l_min, 1)  # 256 sub-passes: the fixed parts remain
+    budget = least + int((one - least) * frac)
     lp, need = lz.plan(cfg.n, cfg.L, cfg.l_min, budget)
     assert lp == 1 and need <= budget
     runner = lz.GreedyGraph(cfg.n, cfg.L, cfg.l_min, "cuda", budget_bytes=budget)
@@ -288,10 +289,12 @@ def test_plan_subpasses_monotone(lz):
     one = _one_length_workspace(lz, n, L, l_min)
     lp, need = lz.plan(n, L, l_min, one)
     assert lp == 1 and need == one
+    lp, least = lz.plan(n, L, l_min, 1 << 20)
+    assert lp == 0 and least > 1 << 20 and least < one
     prev = one
     for frac in (0.7, 0.4, 0.2, 0.1, 0.05):
-        lp, need = lz.plan(n, L, l_min, int(one * frac))
-        assert lp == 1 and need <= int(one * frac) and need < prev
+        b = least + int((one - least) * frac)
+        lp, need = lz.plan(n, L, l_min, b)
+        assert lp == 1 and least <= need <= b and need <= prev
         prev = need
-    lp, need = lz.plan(n, L, l_min, 1 << 20)
-    assert lp == 0 and need > 1 << 20
+    assert prev < one
