@@ -16,6 +16,9 @@
 //
 // One launch may also run SEVERAL ranks (GreedyPeers::nranks_here > 1: blocks grouped by rank)
 // so that the cross-rank protocol is tested on one GPU with plain device pointers.
+#include <cstdio>
+#include <utility>
+
 #include "kernels.cuh"
 
 namespace lsg {
@@ -438,22 +441,34 @@ lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t
         return LASAGNA_EINVAL;
     }
     GreedyPeers q = p;
-    if (q.bpr == 0) {
+    // blocks per SM of the first round (the whole pool) and of the later rounds (survivors);
+    // LASAGNA_GREEDY_BPS=a,b overrides (A/B only)
+    static const std::pair<uint32_t, uint32_t> bps = [] {
+        uint32_t a0 = 16, a1 = 16;
+        if (const char *e = getenv("LASAGNA_GREEDY_BPS")) sscanf(e, "%u,%u", &a0, &a1);
+        return std::make_pair(std::max(1u, a0), std::max(1u, a1));
+    }();
+    auto per_rank = [&](uint32_t per_sm) {
         const uint64_t want = std::max<uint64_t>(
-            1, std::min<uint64_t>(ceil_div(q.cap, GR_THREADS * GR_K), (uint64_t)num_sms() * 16));
-        q.bpr = (uint32_t)std::max<uint64_t>(1, want / q.nranks_here);
-    }
-    const dim3 grid(q.bpr * q.nranks_here);
+            1, std::min<uint64_t>(ceil_div(q.cap, GR_THREADS * GR_K), (uint64_t)num_sms() * per_sm));
+        return (uint32_t)std::max<uint64_t>(1, want / q.nranks_here);
+    };
+    const uint32_t bpr0 = q.bpr ? q.bpr : per_rank(bps.first);
+    const uint32_t bpr1 = q.bpr ? q.bpr : per_rank(bps.second);
     auto run = [&](auto multi) -> lasagna_status {
         constexpr bool M = decltype(multi)::value;
         for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
+            q.bpr = r == 0 ? bpr0 : bpr1;
+            const dim3 grid(q.bpr * q.nranks_here);
             greedy_propose_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r);
             LSG_LAUNCHED("greedy_propose_kernel");
             if (M) {
                 greedy_xbar_kernel<<<q.nranks_here, 1, 0, s>>>(q);
                 LSG_LAUNCHED("greedy_xbar_kernel");
             }
-            greedy_accept_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r + 1, l);
+            q.bpr = bpr1;
+            const dim3 grid2(q.bpr * q.nranks_here);
+            greedy_accept_kernel<M><<<grid2, GR_THREADS, 0, s>>>(q, 2 * r + 1, l);
             LSG_LAUNCHED("greedy_accept_kernel");
             if (M) {
                 greedy_xbar_kernel<<<q.nranks_here, 1, 0, s>>>(q);

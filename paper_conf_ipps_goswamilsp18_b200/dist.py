@@ -471,8 +471,8 @@ class ShardedGraph:
         self.counters.zero_()
         # 1. packed reads: local pack into my slice, all-gather -> every rank verifies any hit
         mine = self.packed_all[rank * n_pad:(rank + 1) * n_pad]
-        if n_local:
-            mine[:n_local] = lz.load_reads(ascii_local.to(dev, non_blocking=True), device=dev)
+        if n_local:  # device ASCII, or page-locked host ASCII read in place by the pack kernel
+            mine[:n_local] = lz.load_reads(ascii_local, device=dev)
         if world > 1:
             C.all_gather_into_tensor(self.packed_all.view(-1), mine.reshape(-1).clone())
         packed_all = self.packed_all
@@ -654,6 +654,9 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
 
     runner = ShardedGraph(n, L, l_min, None, dev, args.lengths_per_pass) if fast else None
 
+    h_succ = torch.empty(2 * n, dtype=torch.int32).pin_memory()
+    h_olen = torch.empty(2 * n, dtype=torch.uint8).pin_memory()
+
     def step(src, d2h: bool, timing: bool = False):
         if fast:
             succ, olen, st = runner(src, timing=timing)
@@ -661,7 +664,8 @@ def bench_main(args, cfg, metric, peak, ClockSampler, bus_id, cpu_baseline) -> N
             succ, olen, st = greedy_graph(src, n, L, l_min, be,
                                           lengths_per_pass=args.lengths_per_pass)
         if d2h:
-            succ.cpu(), olen.cpu()
+            h_succ.copy_(succ, non_blocking=True)
+            h_olen.copy_(olen, non_blocking=True)
         return st
 
     for _ in range(args.warmup):
