@@ -177,7 +177,7 @@ def cpu_baseline(cfg, host_reads: np.ndarray, target_s: float = 12.0) -> dict:
 
 # ------------------------------------------------------------------ algorithmic bytes
 def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict, ms_step: float,
-             sm_mhz: float | None = None, ascii_fused: bool = True) -> dict:
+             sm_mhz: float | None = None, ascii_fused: bool = True, cfg_name: str = "cfg3") -> dict:
     """Dominant phase and its achieved ALGORITHMIC GB/s (bytes per unit in DESIGN.md x units
     per launch / CUDA-event time per launch), plus the whole step's algorithmic GB/s.  Stats
     are summed over `steps` steps."""
@@ -218,7 +218,7 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict, ms
     traffic = None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-            traffic = json.load(f).get(name)
+            traffic = json.load(f).get(cfg_name, {}).get(name)  # captured on this config only
     except Exception:
         pass
     phases = {k: {"ms_per_step": v[0] / steps, "launches_per_step": v[1] / steps,
@@ -236,7 +236,7 @@ def roofline(stats: dict, n: int, L: int, l_min: int, steps: int, peak: dict, ms
     issue = None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_inst.json")) as f:
-            inst = json.load(f).get(name)
+            inst = json.load(f).get(cfg_name, {}).get(name)
         if inst and avg_s > 0:
             import torch
             sms = torch.cuda.get_device_properties(0).multi_processor_count
@@ -459,7 +459,7 @@ def main_streaming(args, cfg) -> None:
     checks["packed_equals_ascii_path"] = same_as_packed
     peak = _peaks()
     roof = roofline(st, n, L, l_min, args.steps, peak, ms_step, clocks.get("sm_mhz"),
-                    ascii_fused=False)
+                    ascii_fused=False, cfg_name=cfg.name)
     lpp_used = st["lengths_per_pass"]
     if not args.no_verify_lpp1 and lpp_used > 1:
         # a8 equality: the same graph with one length per pass (37 device passes at cfg5)
@@ -640,7 +640,8 @@ def main() -> None:
         assert np.array_equal(outs[j][0].numpy(), ref_succ), f"lane {j} differs"
 
     peak = _peaks()
-    roof = roofline(st, n, L, l_min, args.steps, peak, ms_step, clocks.get("sm_mhz"))
+    roof = roofline(st, n, L, l_min, args.steps, peak, ms_step, clocks.get("sm_mhz"),
+                    cfg_name=cfg.name)
     out = {
         "metric": METRIC, "value": value, "unit": "reads/s", "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,

@@ -12,7 +12,11 @@
 // read-end pair (a << 32) | b, a < b.
 #pragma once
 
+#include <cooperative_groups.h>
+
 #include "kernels.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace lsg {
 
@@ -47,7 +51,12 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
     const uint32_t x = w ^ 1u, y = v ^ 1u;
     const uint32_t lo = min(x, y), hi = max(x, y);
     const unsigned long long rec = ((unsigned long long)lo << 32) | hi;
-    const uint32_t slot = atomicAdd(sg.bcount, 1u);
+    // one shared atomic per converged group of lanes (candidates arrive from chain walks in
+    // which several lanes of a warp often match in the same step)
+    const cg::coalesced_group grp = cg::coalesced_threads();
+    uint32_t base = 0;
+    if (grp.thread_rank() == 0) base = atomicAdd(sg.bcount, grp.size());
+    const uint32_t slot = grp.shfl(base, 0) + grp.thread_rank();
     if (slot < sg.bufcap) {
         sg.buf[slot] = rec;
         return;

@@ -568,13 +568,16 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
 // CTA overwrote beforehand (in global memory) with a sentinel of the wrong tag — ~0 (tag 1)
 // in a prefix half, ~0 ^ (1 << vbits) (tag 0) in a suffix half — so the insert and probe
 // loops skip it by its tag bit alone.  Two barriers per window.
-constexpr int BJ_THREADS = 1024; // threads per CTA (one CTA per SM)
-constexpr int BJ_HALF = 4096;   // staged entries per half per window
-constexpr int BJ_BUF = 2 * BJ_THREADS; // staged candidate pairs
+// CTA geometry (BjCfg): threads, staged entries per half per window, chain heads (u32
+// epoch-tagged), filter words (u32) per buffer.  Default 1024 / 4096 / 4096 / 2048 (one CTA
+// per SM, a 64 Ki-bit filter); smaller CTAs run several per SM (a block barrier then stalls
+// one of them, not the SM).
+template <int NT, int HALF, int SLOTS, int BLOOMW>
+struct BjCfg {
+    static constexpr int THREADS = NT, HALF_ = HALF, SLOTS_ = SLOTS, BLOOM = BLOOMW;
+};
 constexpr int BJ_MAXB = 64;     // buckets per window
 constexpr int BJ_FILLS = 256;   // buckets whose fills are staged at once
-constexpr int BJ_SLOTS = 4096;  // chain heads (u32 epoch-tagged)
-constexpr int BJ_BLOOM = 2048;  // u32 words: a 64 Ki-bit filter of the build keys, per buffer
 constexpr int BJ_QCAP = 64;     // per-warp queue of probes that passed the filter
 
 struct WinDesc {
@@ -585,7 +588,7 @@ struct WinDesc {
 // one bucket with a half larger than a staging buffer (massively repeated fingerprints),
 // joined in global memory: every probe entry (the probe half, plus flag-2 entries of the build
 // half) scans the build half
-template <int W>
+template <int W, int BJ_THREADS>
 __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const uint64_t *P,
                                                      uint32_t nP, const uint64_t *S, uint32_t nS,
                                                      Stager &em, unsigned long long &nfalse)
@@ -602,10 +605,14 @@ __device__ __forceinline__ void oversized_join_split(const JoinArgs &a, const ui
     }
 }
 
-template <int W>
-__global__ void __launch_bounds__(BJ_THREADS, BJ_THREADS >= 1024 ? 1 : 2)
+template <int W, class C>
+__global__ void __launch_bounds__(C::THREADS, 1024 / C::THREADS)
 bucket_join_kernel(BucketJoinArgs b)
 {
+    constexpr int BJ_THREADS = C::THREADS, BJ_HALF = C::HALF_, BJ_SLOTS = C::SLOTS_;
+    constexpr int BJ_BLOOM = C::BLOOM, BJ_BUF = 2 * BJ_THREADS;
+    static_assert((BJ_BLOOM & (BJ_BLOOM - 1)) == 0 && (BJ_SLOTS & (BJ_SLOTS - 1)) == 0, "powers of two");
+    constexpr uint32_t FMASK = BJ_BLOOM * 32u - 1u; // filter bit index mask
     extern __shared__ __align__(128) unsigned char jsm[];
     uint64_t *pst = reinterpret_cast<uint64_t *>(jsm);                    // [2][BJ_HALF]
     uint64_t *sst = pst + 2 * BJ_HALF;                                    // [2][BJ_HALF]
@@ -736,7 +743,7 @@ bucket_join_kernel(BucketJoinArgs b)
             if (d.nb == 0) {
                 const uint64_t bk = c0 + d.first;
                 const uint64_t *gb = b.buckets + bk * 2 * b.half_cap;
-                oversized_join_split<W>(a, gb, sfill[2 * d.first], gb + b.half_cap,
+                oversized_join_split<W, BJ_THREADS>(a, gb, sfill[2 * d.first], gb + b.half_cap,
                                         sfill[2 * d.first + 1], em, nfalse);
             } else {
                 mbar_wait(&mbar[w], (phases >> w) & 1u);
@@ -757,7 +764,7 @@ bucket_join_kernel(BucketJoinArgs b)
                     if (e & tagbit) continue; // sentinel
                     if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
                     const uint32_t hk = (uint32_t)(e >> kshift);
-                    atomicOr(&bl[(hk & 0xFFFFu) >> 5], 1u << (hk & 31u));
+                    atomicOr(&bl[(hk & FMASK) >> 5], 1u << (hk & 31u));
                     const uint32_t old = atomicExch(&slot[hk & (BJ_SLOTS - 1)], tag | k2);
                     next[k2] = (old >> 16) == epoch ? (unsigned short)(old & 0xFFFFu) : 0xFFFFu;
                 }
@@ -793,7 +800,7 @@ bucket_join_kernel(BucketJoinArgs b)
                     }
                 };
                 auto passes = [&](uint64_t e) {
-                    const uint32_t hk = (uint32_t)(e >> kshift) & 0xFFFFu;
+                    const uint32_t hk = (uint32_t)(e >> kshift) & FMASK;
                     return ((bl[hk >> 5] >> (hk & 31u)) & 1u) != 0;
                 };
 #pragma unroll 2
@@ -826,26 +833,42 @@ bucket_join_kernel(BucketJoinArgs b)
     if ((threadIdx.x & 31) == 0 && nfalse) atomicAdd(a.false_matches, nfalse);
 }
 
+template <int W, class C>
+static lasagna_status launch_bucket_join_cfg(const BucketJoinArgs &args, cudaStream_t s)
+{
+    constexpr int NT = C::THREADS, HALF = C::HALF_;
+    const size_t smem = (size_t)4 * HALF * 8 + (size_t)2 * NT * 8 + (size_t)C::SLOTS_ * 4 +
+                        (size_t)2 * C::BLOOM * 4 + (size_t)(NT / 32) * BJ_QCAP * 2 +
+                        (size_t)HALF * 2 + (size_t)2 * BJ_FILLS * 4;
+    LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W, C>,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bucket_join_kernel<W, C>, NT,
+                                                           smem));
+    per_sm = std::max(per_sm, 1);
+    const uint64_t blocks =
+        std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)num_sms() * per_sm, args.n_buckets));
+    bucket_join_kernel<W, C><<<(unsigned)blocks, NT, smem, s>>>(args);
+    LSG_LAUNCHED("bucket_join_kernel");
+    return LASAGNA_OK;
+}
+
 lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
 {
     if (args.n_buckets == 0) return LASAGNA_OK;
     if (args.half_cap & 1) return LASAGNA_EINVAL; // sentinels need an even half capacity
+    // CTA geometry: LASAGNA_BJ=1 (A/B): 512 threads, 2048-entry halves, two CTAs per SM;
+    // LASAGNA_BJ=2: 256 threads, 1024-entry halves, four per SM.  A geometry is only used when
+    // a whole bucket half fits its staging buffer twice over.
+    int v = 0;
+    if (const char *e = getenv("LASAGNA_BJ")) v = atoi(e);
+    if (v == 2 && 2 * args.half_cap > 1024) v = 1;
+    if (v == 1 && 2 * args.half_cap > 2048) v = 0;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        const size_t smem = (size_t)4 * BJ_HALF * 8 + (size_t)BJ_BUF * 8 + (size_t)BJ_SLOTS * 4 +
-                            (size_t)2 * BJ_BLOOM * 4 + (size_t)(BJ_THREADS / 32) * BJ_QCAP * 2 +
-                            (size_t)BJ_HALF * 2 + (size_t)2 * BJ_FILLS * 4;
-        LSG_CUDA(cudaFuncSetAttribute(bucket_join_kernel<W>,
-                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        int per_sm = 0;
-        LSG_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bucket_join_kernel<W>,
-                                                               BJ_THREADS, smem));
-        per_sm = std::max(per_sm, 1);
-        const uint64_t blocks =
-            std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)num_sms() * per_sm, args.n_buckets));
-        bucket_join_kernel<W><<<(unsigned)blocks, BJ_THREADS, smem, s>>>(args);
-        LSG_LAUNCHED("bucket_join_kernel");
-        return LASAGNA_OK;
+        if (v == 2) return launch_bucket_join_cfg<W, BjCfg<256, 1024, 1024, 512>>(args, s);
+        if (v == 1) return launch_bucket_join_cfg<W, BjCfg<512, 2048, 2048, 1024>>(args, s);
+        return launch_bucket_join_cfg<W, BjCfg<1024, 4096, 4096, 2048>>(args, s);
     });
 }
 

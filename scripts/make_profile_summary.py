@@ -56,8 +56,13 @@ def launch_table(path: str) -> str:
 
 
 def raw(path: str) -> dict:
-    txt = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    """One launch's raw page: an .ncu-rep, or its `--page raw --csv` export (.csv)."""
+    if path.endswith(".csv"):
+        txt = open(path).read()
+        txt = txt[txt.index('"ID"'):] if '"ID"' in txt else txt
+    else:
+        txt = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
+                             text=True).stdout
     rows = list(csv.reader(txt.splitlines()))
     hdr, units, vals = rows[0], rows[1], rows[2]
     d = {"Kernel Name": vals[hdr.index("Kernel Name")]}
@@ -74,21 +79,25 @@ def to_bytes(v: str, unit: str) -> float:
 
 
 def main() -> None:
-    tag, launches, reps = sys.argv[1], sys.argv[2], sys.argv[3:]
+    # python scripts/make_profile_summary.py TAG CFG launches.csv|- prof...
+    tag, cfg, launches, reps = sys.argv[1], sys.argv[2], sys.argv[3], sys.argv[4:]
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
-    with open(os.path.join(prof, f"{tag}_launches.md"), "w") as f:
-        f.write(f"# {tag}: kernel launch list of one bench step\n\n")
+    if launches != "-":
+      with open(os.path.join(prof, f"{tag}_launches.md"), "w") as f:
+        f.write(f"# {tag}: kernel launch list of one bench step ({cfg})\n\n")
         f.write("`ncu --metrics gpu__time_duration.sum --clock-control none` over "
                 "`bench.py --steps 1 --warmup 1` (every step the bench runs: warm-up, timed, "
                 "the serial and pipelined e2e legs). Cold-cache, "
                 "serialised: compare shares, not absolute times.\n\n")
         f.write(launch_table(launches) + "\n")
     traffic_path = os.path.join(prof, "ncu_traffic.json")
-    traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+    traffic_all = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+    traffic = traffic_all.setdefault(cfg, {})  # per config: bytes depend on the workload
     inst_path = os.path.join(prof, "ncu_inst.json")
-    inst = json.load(open(inst_path)) if os.path.exists(inst_path) else {}
-    lines = [f"# {tag}: one `ncu --set full --clock-control none` launch per kernel (cfg3)\n"]
+    inst_all = json.load(open(inst_path)) if os.path.exists(inst_path) else {}
+    inst = inst_all.setdefault(cfg, {})
+    lines = [f"# {tag}: one `ncu --set full --clock-control none` launch per kernel ({cfg})\n"]
     for rp in reps:
         d = raw(rp)
         name = d["Kernel Name"].split("(")[0].replace("void ", "").split("<")[0]
@@ -107,9 +116,9 @@ def main() -> None:
     with open(os.path.join(prof, f"{tag}_ncu.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     with open(traffic_path, "w") as f:
-        json.dump(traffic, f, indent=1)
+        json.dump(traffic_all, f, indent=1)
     with open(inst_path, "w") as f:
-        json.dump(inst, f, indent=1)
+        json.dump(inst_all, f, indent=1)
     print("wrote", tag)
 
 
