@@ -134,7 +134,7 @@ typedef struct {
     uint32_t key_sort_bits;    /* key bits T the tables are radix-sorted by (bucket bits)   */
     uint32_t sort_launches;    /* onesweep passes launched (each sorts a whole group)       */
     uint32_t search_launches;  /* search (join) launches, one per length                    */
-    uint32_t bucketed;         /* 1: radix-partition path (partition.cu), 0: exact LSD path */
+    uint32_t bucketed;         /* 1: radix-partition path (partition_*.cu), 0: exact LSD path */
     /* device time per phase, CUDA events on `stream` (ms).  ms_table covers a1 (when the
      * staging is fused into the first pass), a2 and the level-1 partition: one kernel */
     float ms_table, ms_sort, ms_search, ms_greedy;

@@ -73,7 +73,7 @@ __device__ __forceinline__ uint64_t canon_key(uint64_t H, uint64_t Hr, uint64_t 
     const uint64_t f = h < hr ? 0ull : (h > hr ? 1ull : 2ull);
     return (mix(c) & keep) | (f << vbits) | v;
 }
-// The bucketed path's form of the same entry (partition.cu): the top 8 bits of mix(min) pick
+// The bucketed path's form of the same entry (partition_scatter.cu): the top 8 bits of mix(min) pick
 // the level-1 region and are implied by the region an entry sits in, so the stored key drops
 // them and keeps the next 62 - vbits bits instead — 8 more fingerprint bits in every
 // comparison (R12: at vbits = 32, 30 stored + 8 implied = 38 bits instead of 30):
@@ -91,14 +91,22 @@ __device__ __forceinline__ uint64_t canon_key_d1(uint64_t H, uint64_t Hr, uint64
 }
 // The same entry from the bucketed path's mod-2^64 key streams (fingerprint.cuh Fp64Streams,
 // reading R26): H and Hr are exact residues already.
+// fl1 = 1 << vbits, fl2 = 2 << vbits (the flag field); v < 2^vbits <= 2^32.
 __device__ __forceinline__ uint64_t canon_key64_d1(uint64_t H, uint64_t Hr, uint64_t keep,
-                                                   uint32_t vbits, uint64_t v, uint32_t *d1)
+                                                   uint64_t fl1, uint64_t fl2, uint32_t v,
+                                                   uint32_t *d1)
 {
-    const uint64_t c = H < Hr ? H : Hr;
-    const uint64_t f = H < Hr ? 0ull : (H > Hr ? 1ull : 2ull);
+    const bool lt = H < Hr;
+    const uint64_t c = lt ? H : Hr;
+    const uint64_t fb = lt ? 0ull : (H == Hr ? fl2 : fl1);
     const uint64_t m = mix(c);
-    *d1 = (uint32_t)(m >> 56);
-    return ((m << 8) & keep) | (f << vbits) | v;
+    const uint32_t mlo = (uint32_t)m, mhi = (uint32_t)(m >> 32);
+    *d1 = mhi >> 24;
+    // (m << 8) & keep | flag | v on 32-bit halves (a funnel shift for the high half: the
+    // compiler otherwise folds the shift into a second 64-bit multiply)
+    const uint32_t klo = ((mlo << 8) & (uint32_t)keep) | (uint32_t)fb | v;
+    const uint32_t khi = (__funnelshift_l(mlo, mhi, 8) & (uint32_t)(keep >> 32)) | (uint32_t)(fb >> 32);
+    return ((uint64_t)khi << 32) | klo;
 }
 __device__ __forceinline__ uint32_t key_flag(uint64_t key, uint32_t vbits)
 {
@@ -355,6 +363,11 @@ uint64_t launch_count();
 template <typename F>
 lasagna_status dispatch_W(uint32_t L, F &&f)
 {
+#ifdef LSG_DEV_ONLY_W // SASS inspection builds only: one read width
+    if (words_for(L) == LSG_DEV_ONLY_W) return f(std::integral_constant<int, LSG_DEV_ONLY_W>{});
+    set_error("L=%u: dev build for W=%d only", L, LSG_DEV_ONLY_W);
+    return LASAGNA_EINVAL;
+#endif
     switch (words_for(L)) {
     case 1: return f(std::integral_constant<int, 1>{});
     case 2: return f(std::integral_constant<int, 2>{});

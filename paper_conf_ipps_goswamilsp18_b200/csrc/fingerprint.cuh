@@ -1,5 +1,5 @@
 // fingerprint.cuh — the rolling Rabin-Karp streams of a2 (Fig. 5/6), shared by
-// the table kernels (fingerprint.cu, partition.cu).
+// the table kernels (fingerprint.cu, partition_scatter.cu).
 #pragma once
 
 #include "kernels.cuh"

@@ -1,5 +1,5 @@
 // joinwin.cuh — the shared-memory join of one window of whole buckets (a5), used by the
-// contiguous-table join (search.cu) and the bucketed join (partition.cu).
+// contiguous-table join (search.cu) and the bucketed join (partition_join.cu).
 //
 // A window holds the entries of complete T-bit buckets, so every fingerprint match of a
 // probe entry is a build entry of the same window ("a fingerprint present in W_S
@@ -12,11 +12,7 @@
 // read-end pair (a << 32) | b, a < b.
 #pragma once
 
-#include <cooperative_groups.h>
-
 #include "kernels.cuh"
-
-namespace cg = cooperative_groups;
 
 namespace lsg {
 
@@ -51,12 +47,7 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
     const uint32_t x = w ^ 1u, y = v ^ 1u;
     const uint32_t lo = min(x, y), hi = max(x, y);
     const unsigned long long rec = ((unsigned long long)lo << 32) | hi;
-    // one shared atomic per converged group of lanes (candidates arrive from chain walks in
-    // which several lanes of a warp often match in the same step)
-    const cg::coalesced_group grp = cg::coalesced_threads();
-    uint32_t base = 0;
-    if (grp.thread_rank() == 0) base = atomicAdd(sg.bcount, grp.size());
-    const uint32_t slot = grp.shfl(base, 0) + grp.thread_rank();
+    const uint32_t slot = atomicAdd(sg.bcount, 1u);
     if (slot < sg.bufcap) {
         sg.buf[slot] = rec;
         return;

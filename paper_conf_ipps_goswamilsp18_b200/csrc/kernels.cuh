@@ -76,7 +76,7 @@ lasagna_status launch_pairs_to_keys(const unsigned long long *pool, const unsign
 lasagna_status launch_keys_to_output(const uint64_t *keys, uint64_t m, uint32_t vbits, uint8_t l,
                                      uint32_t *pa, uint32_t *pb, uint8_t *pl, cudaStream_t s);
 
-// ---- bucketed a3/a4/a5 (partition.cu)
+// ---- bucketed a3/a4/a5 (partition_*.cu)
 struct ScatterArgs {
     const uint64_t *packed;
     uint64_t n, read_offset;

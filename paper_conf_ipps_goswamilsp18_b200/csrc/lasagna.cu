@@ -59,7 +59,7 @@ static bool env_flag(const char *name, char first)
 struct Geometry {
     uint64_t n, V, N;
     uint32_t L, l_min, n_len, vbits, T;
-    // bucketed path (partition.cu): P MSD levels (8, 8, dlast bits), capacities with slack
+    // bucketed path (partition_*.cu): P MSD levels (8, 8, dlast bits), capacities with slack
     uint32_t P, dlast;
     uint64_t cap1, cap2;    // unsplit region capacities of levels 1 and 2 (when not final)
     uint64_t half;          // half-bucket capacity of the final level
@@ -201,7 +201,7 @@ static Layout layout(const Geometry &g, uint32_t G, uint64_t pool_cap, bool gree
     return l;
 }
 
-// The bucketed path (partition.cu) serves every geometry (P <= 3); LASAGNA_PATH=exact forces
+// The bucketed path (partition_*.cu) serves every geometry (P <= 3); LASAGNA_PATH=exact forces
 // the exact LSD-sort path (also the fallback when a slack region overflows).
 static bool use_bucketed(const Geometry &g)
 {
@@ -252,7 +252,7 @@ struct Run {
     SortCtx sctx;
     uint64_t *tab[2];
     uint32_t *hist;
-    bool bucketed;              // partition.cu path (else exact LSD sort + contiguous join)
+    bool bucketed;              // partition_*.cu path (else exact LSD sort + contiguous join)
     const unsigned char *ascii = nullptr; // a1 still to do: the first group's scatter packs it
     const char *ascii_host = nullptr;     // ... from this page-locked host copy (chunked DMA)
     uint64_t *packed_out = nullptr;
@@ -563,7 +563,7 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
         bj.fills = (g.P == 1 ? r.fill1 : g.P == 2 ? r.fill2 : r.fill3) + (uint64_t)s * 2 * nbk;
         bj.half_cap = g.half;
         bj.n_buckets = nbk;
-        // block windows (partition.cu); LASAGNA_JOIN=warp (A/B only): one warp per bucket
+        // block windows (partition_*.cu); LASAGNA_JOIN=warp (A/B only): one warp per bucket
         // (warpjoin.cu) when a half fits a warp's slice — measured slower at cfg3 (31.9 vs
         // 17.1 ms per step)
         rc = (env_flag("LASAGNA_JOIN", 'w') && warp_join_fits(bj)) ? launch_warp_join(bj, r.s)

@@ -2,7 +2,7 @@
 // (Algorithm 2: "a fingerprint present in W_S cannot be present in any window
 // except W_P" — a bucket is such a window pair: its build half plays W_P, its probe half W_S).
 //
-// The block-wide window join (partition.cu bucket_join_kernel) pays two block barriers, a
+// The block-wide window join (partition_join.cu bucket_join_kernel) pays two block barriers, a
 // window plan and a filter clear per ~7 K entries: ~105 instructions per entry at cfg3.  A
 // bucket holds ~1 K entries (cfg3: ~531 per half), small enough for one warp:
 //   1. the warp copies its bucket's build half (flags 0/2) into its own shared-memory slice
