@@ -3,12 +3,30 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <cstdio>
 #include <stdint.h>
 
 #include <algorithm>
 #include <type_traits>
 
 #include "lasagna.h"
+
+// Device-side bounds checks of the checked build (build.build(checked=True) compiles with
+// -DLSG_CHECKS into liblasagna_checked.so; LASAGNA_CHECKED=1 loads it).  compute-sanitizer is
+// not available on the GPU pool, so the GPU tests run once against this build: a failed check
+// prints its site and traps (the call then returns LASAGNA_ECUDA).  Free in the product build.
+#ifdef LSG_CHECKS
+#define LSG_DCHECK(cond)                                                                       \
+    do {                                                                                       \
+        if (!(cond)) {                                                                         \
+            printf("LSG_DCHECK failed %s:%d: %s (block %d thread %d)\n", __FILE__, __LINE__,  \
+                   #cond, (int)blockIdx.x, (int)threadIdx.x);                                  \
+            __trap();                                                                          \
+        }                                                                                      \
+    } while (0)
+#else
+#define LSG_DCHECK(cond) do { } while (0)
+#endif
 
 namespace lsg {
 

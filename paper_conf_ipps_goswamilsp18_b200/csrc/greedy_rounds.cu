@@ -63,6 +63,7 @@ struct Owner {
     }
     __device__ __forceinline__ bool claimed(uint32_t x) const
     {
+        LSG_DCHECK(p->slice == 0 || x < p->slice * p->g);
         const uint64_t i = local(x);
         const uint32_t *w = p->r[rank(x)].claimed + (i >> 5);
         const uint32_t v = MULTI ? *(volatile const uint32_t *)w : *w;
@@ -75,6 +76,7 @@ struct Owner {
     }
     __device__ __forceinline__ unsigned long long *best(uint32_t x) const
     {
+        LSG_DCHECK(p->slice == 0 || x < p->slice * p->g);
         return p->r[rank(x)].best + local(x);
     }
     __device__ __forceinline__ void propose(uint32_t a, uint32_t b, uint32_t epoch) const

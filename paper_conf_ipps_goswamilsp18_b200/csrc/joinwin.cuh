@@ -42,6 +42,7 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
                                           uint64_t vmask, Stager &sg, unsigned long long &nfalse)
 {
     const uint32_t w = (uint32_t)(e & vmask), v = (uint32_t)(p & vmask);
+    LSG_DCHECK(a.V == 0 || (w < a.V && v < a.V));
     if ((w >> 1) == (v >> 1)) return; // R9: no same-read edge (also the entry itself)
     if (w > v && key_flag(e, a.vbits) == 2 && key_flag(p, a.vbits) == 2) return;
     const uint32_t x = w ^ 1u, y = v ^ 1u;
@@ -74,6 +75,7 @@ __device__ __forceinline__ void verify_staged(const JoinArgs &a, unsigned long l
     for (uint32_t t = from + threadIdx.x; t < to; t += NT) {
         const unsigned long long rec = buf[t];
         const uint32_t u = (uint32_t)(rec >> 32), b = (uint32_t)rec;
+        LSG_DCHECK(a.V == 0 || (u < a.V && b < a.V));
         if (!verify_pair<W>(a, u, b ^ 1u)) {
             buf[t] = ~0ull;
             ++nfalse;

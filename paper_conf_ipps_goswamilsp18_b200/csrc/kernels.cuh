@@ -61,6 +61,7 @@ struct JoinArgs {
     // approximate mode: hits are accepted by the 128-bit fingerprint
     // pair (common.cuh verify_fp128) instead of the bases
     bool approx = false;
+    uint64_t V = 0; // vertex ids in the pairs are < V (checked build; 0: not checked)
 };
 // the check a hit passes: bases (exact) or the fingerprint pair (approximate mode)
 template <int W>

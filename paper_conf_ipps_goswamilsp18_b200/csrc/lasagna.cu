@@ -541,6 +541,7 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.packed = packed;
     ja.keys = r.tab[which] + (uint64_t)s * g.N;
     ja.N = g.N;
+    ja.V = g.V;
     ja.L = g.L;
     ja.stride = stride_for(g.L);
     ja.l = l;
@@ -1363,6 +1364,7 @@ lasagna_status lasagna_join(const uint64_t *keys, uint64_t count, const uint64_t
     ja.packed = packed_all;
     ja.keys = keys;
     ja.N = count;
+    ja.V = g.V;
     ja.L = L;
     ja.stride = stride_for(L);
     ja.l = l;
@@ -1635,6 +1637,7 @@ lasagna_status lasagna_shard_join(const void *part, uint64_t n_total, uint32_t w
     bj.j.packed = packed_all;
     bj.j.keys = nullptr;
     bj.j.N = 0;
+    bj.j.V = g.V;
     bj.j.L = L;
     bj.j.stride = stride_for(L);
     bj.j.l = l;

@@ -149,6 +149,7 @@ bucket_join_kernel(BucketJoinArgs b)
             }
             __syncwarp();
             if ((uint32_t)lane < nb) {
+                LSG_DCHECK(c0 + j < b.n_buckets);
                 const uint64_t *gb = b.buckets + (c0 + j) * 2 * b.half_cap;
                 if (pp)
                     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::"

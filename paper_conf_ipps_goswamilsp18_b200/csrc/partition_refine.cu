@@ -119,6 +119,7 @@ refine_kernel(RefineArgs a)
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
             const long long go = gofs[binof(k)];
+            LSG_DCHECK(go < 0 || (uint64_t)(go + u) < (uint64_t)gridDim.x * nb * a.cap_out);
             if (go >= 0) a.out[go + u] = k;
         }
         __syncthreads();

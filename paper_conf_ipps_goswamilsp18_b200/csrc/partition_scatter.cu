@@ -68,6 +68,13 @@ scatter_table_kernel(ScatterArgs a)
     __syncthreads();
     const uint32_t v0 = (uint32_t)(2 * (a.read_offset + i)); // V < 2^32
     const uint64_t fl1 = 1ull << a.vbits, fl2 = 2ull << a.vbits;
+#ifdef LSG_CHECKS
+    // regions this call may fill: [G][512] split, else the shard layout (a sub-pass: one range)
+    const uint64_t nreg = SPLIT ? (uint64_t)(a.l_hi - a.l_lo + 1u) * 512u
+                                : (uint64_t)(a.l_hi - a.l_lo + 1u) * a.nb_pad *
+                                      (a.keep_owner >= 0 ? 1u : a.dest_g);
+    LSG_DCHECK(v0 / 2u < a.read_offset + a.n || !valid);
+#endif
     Fp64Streams st; // key streams modulo 2^64 (R26)
     // the l_lo - 1 bases before the first emitted length, absorbed in 8-base chunks
     fp64_absorb<W>(x, y, a.l_lo - 1u, st);
@@ -143,6 +150,7 @@ scatter_table_kernel(ScatterArgs a)
                 const uint32_t q = bin / NBL;
                 rg[b] = SPLIT ? (uint64_t)(lfirst - a.l_lo + q) * NBL + bin % NBL
                               : (uint64_t)rbase[bin % NBL] + (uint64_t)(lfirst - a.l_lo + q) * a.nb_pad;
+                LSG_DCHECK(!(c[b] && q < kc) || rg[b] < nreg);
                 bs[b] = (c[b] && q < kc) ? atomicAdd(&a.fill[rg[b]], c[b]) : 0u;
                 sum += c[b];
             }
@@ -175,6 +183,7 @@ scatter_table_kernel(ScatterArgs a)
             const uint32_t total = lstart[NBIN];
             for (uint32_t u = threadIdx.x; u < total; u += NT) {
                 const long long go = gofs[sbin[u]];
+                LSG_DCHECK(go < 0 || (uint64_t)(go + u) < nreg * a.cap);
                 if (go >= 0) a.out[go + u] = stage[u];
             }
             // the next round's first barrier orders these reads before stage/lstart reuse

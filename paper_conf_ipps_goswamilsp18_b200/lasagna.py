@@ -66,10 +66,11 @@ def lib() -> ctypes.CDLL:
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.SO
+    checked = os.environ.get("LASAGNA_CHECKED", "") == "1"  # bounds-checked build (tests)
+    path = _build.SO_CHECKED if checked else _build.SO
     try:
-        if _build.stale():
-            _build.build()
+        if _build.stale(checked):
+            _build.build(checked=checked)
     except RuntimeError:
         if not os.path.exists(path):
             raise
