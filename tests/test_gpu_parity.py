@@ -667,11 +667,12 @@ def test_product_path_fails_loudly_without_the_library(monkeypatch, tmp_path):
     raises instead of computing anything; the package never imports the oracle."""
     from paper_conf_ipps_goswamilsp18_b200 import lasagna as lz
 
-    def no_nvcc():
+    def no_nvcc(*_a, **_k):
         raise RuntimeError("nvcc not found")
 
     monkeypatch.setattr(lz, "_lib", None)
     monkeypatch.setattr(lz._build, "SO", str(tmp_path / "liblasagna.so"))
+    monkeypatch.setattr(lz._build, "SO_CHECKED", str(tmp_path / "liblasagna_checked.so"))
     monkeypatch.setattr(lz._build, "stale", no_nvcc)
     with pytest.raises((lz.LasagnaError, RuntimeError)):
         lz.lib()
