@@ -364,6 +364,32 @@ lasagna_status cuda_status(cudaError_t e, const char *what);
 void count_launch();
 uint64_t launch_count();
 
+// Programmatic dependent launch (PDL) of back-to-back dependent kernels (the greedy's rounds):
+// the next grid is scheduled while this one drains and waits in pdl_wait() until this grid's
+// memory is visible, hiding the launch gap.  A kernel launched by launch_pdl MUST call
+// pdl_wait() before touching anything its predecessor wrote; without PDL both are no-ops.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger()
+{
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t s, Args... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 #define LSG_CUDA(call)                                                                         \
     do {                                                                                       \
         cudaError_t e_ = (call);                                                               \

@@ -164,6 +164,8 @@ template <bool MULTI>
 __global__ void __launch_bounds__(GR_THREADS)
 greedy_propose_kernel(GreedyPeers p, uint32_t j)
 {
+    pdl_wait(); // launched with PDL after the previous round / the join
+    pdl_trigger();
     __shared__ uint32_t wsum[GR_THREADS / 32];
     __shared__ unsigned long long sbase;
     const uint32_t me = p.rank0 + blockIdx.x / p.bpr;
@@ -214,6 +216,8 @@ template <bool MULTI>
 __global__ void __launch_bounds__(GR_THREADS)
 greedy_accept_kernel(GreedyPeers p, uint32_t j, uint8_t l)
 {
+    pdl_wait(); // launched with PDL after the previous round / the join
+    pdl_trigger();
     __shared__ uint32_t wsum[GR_THREADS / 32];
     __shared__ unsigned long long sbase;
     const uint32_t me = p.rank0 + blockIdx.x / p.bpr;
@@ -312,6 +316,8 @@ template <bool MULTI>
 __global__ void __launch_bounds__(TL_THREADS)
 greedy_tail_kernel(GreedyPeers p, uint8_t l)
 {
+    pdl_wait(); // launched with PDL after the previous round / the join
+    pdl_trigger();
     __shared__ unsigned long long s[TL_SEQ_MAX];
     __shared__ unsigned long long offs[MAX_PEERS + 1];
     __shared__ uint32_t s_live, s_acc;
@@ -457,12 +463,18 @@ lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t
     };
     const uint32_t bpr0 = q.bpr ? q.bpr : per_rank(bps.first);
     const uint32_t bpr1 = q.bpr ? q.bpr : per_rank(bps.second);
+    // PDL between the single-GPU rounds (LASAGNA_PDL=0: plain launches, A/B only)
+    static const bool use_pdl = [] {
+        const char *e = getenv("LASAGNA_PDL");
+        return !(e && e[0] == '0');
+    }();
     auto run = [&](auto multi) -> lasagna_status {
         constexpr bool M = decltype(multi)::value;
         for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
             q.bpr = r == 0 ? bpr0 : bpr1;
             const dim3 grid(q.bpr * q.nranks_here);
-            greedy_propose_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r);
+            if (M || !use_pdl) greedy_propose_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r);
+            else LSG_CUDA(launch_pdl(greedy_propose_kernel<M>, grid, dim3(GR_THREADS), 0, s, q, 2 * r));
             LSG_LAUNCHED("greedy_propose_kernel");
             if (M) {
                 greedy_xbar_kernel<<<q.nranks_here, 1, 0, s>>>(q);
@@ -470,14 +482,18 @@ lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t
             }
             q.bpr = bpr1;
             const dim3 grid2(q.bpr * q.nranks_here);
-            greedy_accept_kernel<M><<<grid2, GR_THREADS, 0, s>>>(q, 2 * r + 1, l);
+            if (M || !use_pdl) greedy_accept_kernel<M><<<grid2, GR_THREADS, 0, s>>>(q, 2 * r + 1, l);
+            else LSG_CUDA(launch_pdl(greedy_accept_kernel<M>, grid2, dim3(GR_THREADS), 0, s, q,
+                                     2 * r + 1, l));
             LSG_LAUNCHED("greedy_accept_kernel");
             if (M) {
                 greedy_xbar_kernel<<<q.nranks_here, 1, 0, s>>>(q);
                 LSG_LAUNCHED("greedy_xbar_kernel");
             }
         }
-        greedy_tail_kernel<M><<<q.nranks_here, TL_THREADS, 0, s>>>(q, l);
+        if (M || !use_pdl) greedy_tail_kernel<M><<<q.nranks_here, TL_THREADS, 0, s>>>(q, l);
+        else LSG_CUDA(launch_pdl(greedy_tail_kernel<M>, dim3(q.nranks_here), dim3(TL_THREADS), 0, s,
+                                 q, l));
         LSG_LAUNCHED("greedy_tail_kernel");
         return LASAGNA_OK;
     };

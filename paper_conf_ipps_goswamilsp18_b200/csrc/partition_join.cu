@@ -97,7 +97,9 @@ bucket_join_kernel(BucketJoinArgs b)
         for (uint32_t t = threadIdx.x; t < 2 * nc; t += BJ_THREADS) {
             const uint32_t f = b.fills[2 * c0 + t];
             if (f > b.half_cap) *b.overflow = 1u;
-            const uint32_t fc = (uint32_t)min64(f, b.half_cap);
+            // an overflowed half lost keys and holds slots this call never wrote: the call is
+            // redone on the exact path, so join nothing from it (no stale vertex ids)
+            const uint32_t fc = f > b.half_cap ? 0u : f;
             sfill[t] = fc;
             if (fc & 1) // half_cap is even: the slot after an odd fill is inside the half
                 b.buckets[(c0 + t / 2) * 2 * b.half_cap + (t & 1) * b.half_cap + fc] =

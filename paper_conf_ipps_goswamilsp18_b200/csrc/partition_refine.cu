@@ -8,7 +8,7 @@ namespace lsg {
 // other half of a double buffer while tile t is ranked (shared atomics: order inside a
 // sub-region is irrelevant), staged by digit and written out in digit runs.
 template <bool SPLIT, int RF_KPT>
-__global__ void __launch_bounds__(RF_THREADS, 1)
+__global__ void __launch_bounds__(RF_THREADS, RF_KPT == 16 ? 1 : 2)
 refine_kernel(RefineArgs a)
 {
     constexpr int RF_TILE = RF_THREADS * RF_KPT;
@@ -36,7 +36,9 @@ refine_kernel(RefineArgs a)
         for (uint32_t k = 0; k < a.n_src; ++k) {
             const uint32_t f = a.fill_in[k * a.src_stride + r];
             if (f > a.cap_in) *a.overflow = 1u;
-            scount[k] = min64(f, a.cap_in);
+            // an overflowed region dropped whole bin runs (unwritten slots below cap): move
+            // nothing from it (the overflow flag makes the caller redo the call)
+            scount[k] = f > a.cap_in ? 0u : f;
             stile[k] = acc;
             acc += (uint32_t)ceil_div(scount[k], RF_TILE);
         }

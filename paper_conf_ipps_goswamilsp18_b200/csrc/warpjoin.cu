@@ -160,8 +160,7 @@ warp_join_kernel(BucketJoinArgs b)
         fS = b.fills[2 * k + 1];
         if (fP > b.half_cap || fS > b.half_cap) {
             if (lane == 0) *b.overflow = 1u; // the call is redone on the exact path
-            fP = (uint32_t)min64(fP, b.half_cap);
-            fS = (uint32_t)min64(fS, b.half_cap);
+            fP = fS = 0; // unwritten slots: join nothing from an overflowed bucket
         }
     };
     uint32_t fP = 0, fS = 0;
