@@ -160,9 +160,11 @@ __device__ __forceinline__ unsigned long long *ring_slot(const PeerRank &R, uint
     return k == 0 ? R.in_count : R.ctr + PC_RING + k;
 }
 
-template <bool MULTI>
+// VW > 0 (first round with deferred verification): candidates are checked on the bases
+// (read width VW words) before they propose; a rejected hit is dropped and counted
+template <bool MULTI, int VW = 0>
 __global__ void __launch_bounds__(GR_THREADS)
-greedy_propose_kernel(GreedyPeers p, uint32_t j)
+greedy_propose_kernel(GreedyPeers p, uint32_t j, uint8_t l)
 {
     pdl_wait(); // launched with PDL after the previous round / the join
     pdl_trigger();
@@ -179,13 +181,14 @@ greedy_propose_kernel(GreedyPeers p, uint32_t j)
     if (bl == 0 && threadIdx.x == 0) {
         *ring_slot(R, (j + 2) % 3) = 0;
         atomicAdd(&R.ctr[PC_WORK], m);
-        if (j == 0) { // first round of a length: |P_l| bookkeeping
-            atomicAdd(&R.ctr[PC_BOOK + 1], c);
+        if (j == 0) { // first round of a length: |P_l| bookkeeping (VW > 0: counted below)
+            if (VW == 0) atomicAdd(&R.ctr[PC_BOOK + 1], c);
             atomicMax(&R.ctr[PC_BOOK + 2], c);
         }
     }
     const unsigned long long *X = R.pool;
     unsigned long long *outc = ring_slot(R, (j + 1) % 3);
+    uint32_t ntrue = 0, nbad = 0; // VW > 0
     const uint64_t stride = (uint64_t)p.bpr * GR_THREADS * GR_K;
     for (uint64_t i0 = (uint64_t)bl * GR_THREADS * GR_K + threadIdx.x; i0 - threadIdx.x < m;
          i0 += stride) { // block-uniform trip count
@@ -195,6 +198,19 @@ greedy_propose_kernel(GreedyPeers p, uint32_t j)
         for (int k = 0; k < GR_K; ++k) {
             const uint64_t i = i0 + (uint64_t)k * GR_THREADS;
             r[k] = i < m ? X[i] : ~0ull;
+        }
+        if constexpr (VW > 0) {
+            // the bases decide (as the join's verify_staged would): a pair (u, b) of read ends
+            // is the directed overlap (u, b ^ 1, l)
+#pragma unroll
+            for (int k = 0; k < GR_K; ++k)
+                if (r[k] != ~0ull) {
+                    if (verify_overlap<VW>(p.vpacked, p.vstride, p.vL, (uint32_t)(r[k] >> 32),
+                                           (uint32_t)r[k] ^ 1u, l))
+                        ++ntrue;
+                    else
+                        ++nbad, r[k] = ~0ull;
+                }
         }
 #pragma unroll
         for (int k = 0; k < GR_K; ++k)
@@ -208,6 +224,16 @@ greedy_propose_kernel(GreedyPeers p, uint32_t j)
             keepm |= 1u << k;
         }
         block_append(r, keepm, R.pool2, outc, wsum, &sbase);
+    }
+    if constexpr (VW > 0) {
+        for (int o = 16; o; o >>= 1) {
+            ntrue += __shfl_xor_sync(0xffffffffu, ntrue, o);
+            nbad += __shfl_xor_sync(0xffffffffu, nbad, o);
+        }
+        if ((threadIdx.x & 31) == 0) {
+            if (ntrue) atomicAdd(&R.ctr[PC_BOOK + 1], (unsigned long long)ntrue);
+            if (nbad) atomicAdd(p.vfalse, (unsigned long long)nbad);
+        }
     }
     if (MULTI) __threadfence_system(); // proposals to peers' best[] before the barrier kernel
 }
@@ -473,8 +499,21 @@ lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t
         for (uint32_t r = 0; r < FAST_ROUNDS; ++r) {
             q.bpr = r == 0 ? bpr0 : bpr1;
             const dim3 grid(q.bpr * q.nranks_here);
-            if (M || !use_pdl) greedy_propose_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r);
-            else LSG_CUDA(launch_pdl(greedy_propose_kernel<M>, grid, dim3(GR_THREADS), 0, s, q, 2 * r));
+            if (!M && r == 0 && q.vpacked) {
+                // first round with deferred verification: the kernel for the read width
+                lasagna_status rc = dispatch_W(q.vL, [&](auto wc) -> lasagna_status {
+                    constexpr int VW = decltype(wc)::value;
+                    if (!use_pdl) greedy_propose_kernel<false, VW><<<grid, GR_THREADS, 0, s>>>(q, 0, l);
+                    else LSG_CUDA(launch_pdl(greedy_propose_kernel<false, VW>, grid, dim3(GR_THREADS),
+                                             0, s, q, 0u, l));
+                    return LASAGNA_OK;
+                });
+                if (rc != LASAGNA_OK) return rc;
+            } else if (M || !use_pdl) {
+                greedy_propose_kernel<M><<<grid, GR_THREADS, 0, s>>>(q, 2 * r, l);
+            } else {
+                LSG_CUDA(launch_pdl(greedy_propose_kernel<M>, grid, dim3(GR_THREADS), 0, s, q, 2 * r, l));
+            }
             LSG_LAUNCHED("greedy_propose_kernel");
             if (M) {
                 greedy_xbar_kernel<<<q.nranks_here, 1, 0, s>>>(q);

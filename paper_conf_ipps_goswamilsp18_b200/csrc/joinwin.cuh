@@ -53,8 +53,8 @@ __device__ __forceinline__ void candidate(const JoinArgs &a, uint64_t e, uint64_
         sg.buf[slot] = rec;
         return;
     }
-    // staging full: verify inline and emit straight to global memory
-    if (!verify_pair<W>(a, lo, hi ^ 1u)) {
+    // staging full: verify inline (unless the greedy verifies) and emit straight to global memory
+    if (!a.defer_verify && !verify_pair<W>(a, lo, hi ^ 1u)) {
         ++nfalse;
         return;
     }
@@ -192,8 +192,10 @@ __device__ __forceinline__ void window_epilogue(const JoinArgs &a, unsigned long
 {
     const uint32_t to = min(*bcount, 2u * NT);
     if (to >= (uint32_t)NT) {
-        verify_staged<W, NT>(a, buf, 0, to, nfalse);
-        __syncthreads();
+        if (!a.defer_verify) {
+            verify_staged<W, NT>(a, buf, 0, to, nfalse);
+            __syncthreads();
+        }
         flush_staged<NT>(buf, to, a.pairs, a.cap, a.count);
         __syncthreads();
         if (threadIdx.x == 0) *bcount = 0;
@@ -209,8 +211,10 @@ __device__ __forceinline__ void final_flush(const JoinArgs &a, unsigned long lon
 {
     __syncthreads();
     const uint32_t to = min(*bcount, 2u * NT);
-    verify_staged<W, NT>(a, buf, 0, to, nfalse);
-    __syncthreads();
+    if (!a.defer_verify) {
+        verify_staged<W, NT>(a, buf, 0, to, nfalse);
+        __syncthreads();
+    }
     flush_staged<NT>(buf, to, a.pairs, a.cap, a.count);
 }
 

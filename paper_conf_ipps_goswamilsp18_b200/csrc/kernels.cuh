@@ -62,6 +62,9 @@ struct JoinArgs {
     // pair (common.cuh verify_fp128) instead of the bases
     bool approx = false;
     uint64_t V = 0; // vertex ids in the pairs are < V (checked build; 0: not checked)
+    // greedy mode, single GPU: store the fingerprint hits unverified; the greedy's first round
+    // verifies them on the bases (greedy_rounds.cu), in parallel with its random proposals
+    bool defer_verify = false;
 };
 // the check a hit passes: bases (exact) or the fingerprint pair (approximate mode)
 template <int W>
@@ -193,6 +196,12 @@ struct GreedyPeers {
     uint32_t rank0 = 0;       // first rank this launch runs (multi-GPU: my rank)
     uint32_t nranks_here = 1; // ranks this launch runs (> 1: one-GPU test of the protocol)
     uint32_t bpr = 0;         // blocks per rank (0: sized from cap)
+    // deferred verification (single GPU, JoinArgs::defer_verify): the first round checks every
+    // candidate on the bases (R12) before proposing; true pairs are counted in
+    // ctr[PC_BOOK + 1] (|P_l|), rejected hits in *vfalse.  vpacked = nullptr: verified by the join
+    const uint64_t *vpacked = nullptr;
+    uint32_t vL = 0, vstride = 0;
+    unsigned long long *vfalse = nullptr;
 };
 constexpr uint32_t GR_TAIL_CAP = 4096;
 lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t s);

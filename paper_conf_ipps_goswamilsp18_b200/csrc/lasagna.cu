@@ -263,6 +263,7 @@ struct Run {
     const uint32_t *claimed = nullptr; // greedy mode: the join drops pairs with a claimed end
     bool prune = false; // this group's scatter drops entries whose read end is claimed (f1)
     bool approx = false; // f4: hits accepted by the 128-bit fingerprint pair
+    bool defer_verify = false; // greedy mode: the greedy's first round verifies the join's hits
     template <typename T> T *at(size_t off) { return reinterpret_cast<T *>(ws + off); }
     void bind(void *workspace)
     {
@@ -554,6 +555,7 @@ static lasagna_status search_length(Run &r, const uint64_t *packed, uint32_t l, 
     ja.claimed = join_filter() ? r.claimed : nullptr;
     ja.found = ja.claimed ? r.ctr64 + CTR_FOUND : nullptr;
     ja.approx = r.approx;
+    ja.defer_verify = r.defer_verify;
     lasagna_status rc;
     if (r.bucketed) {
         BucketJoinArgs bj;
@@ -807,7 +809,18 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     gb.claimed = claimed;
     gb.cap = cap;
     gb.epoch = 1;
-    const GreedyPeers peers = single_peers(gb, r.ctr64 + CTR_PEER, succ, olen, g.V);
+    GreedyPeers peers = single_peers(gb, r.ctr64 + CTR_PEER, succ, olen, g.V);
+    // the join stores its fingerprint hits unverified and the greedy's first round checks them
+    // on the bases, overlapping the random base reads with its random proposals (LASAGNA_
+    // VERIFY=join: verified inside the join, A/B only; the round-1 greedy and the join-side
+    // claimed filter need verified pairs)
+    r.defer_verify = !old_greedy() && !join_filter() && !env_flag("LASAGNA_VERIFY", 'j');
+    if (r.defer_verify) {
+        peers.vpacked = packed;
+        peers.vL = L;
+        peers.vstride = stride_for(L);
+        peers.vfalse = r.ctr64 + CTR_FALSE;
+    }
 
   for (int attempt = 0; attempt < 2; ++attempt) {
     r.bucketed = attempt == 0 && use_bucketed(g);
