@@ -810,11 +810,12 @@ static lasagna_status greedy_graph_impl(const uint64_t *packed, const char *asci
     gb.cap = cap;
     gb.epoch = 1;
     GreedyPeers peers = single_peers(gb, r.ctr64 + CTR_PEER, succ, olen, g.V);
-    // the join stores its fingerprint hits unverified and the greedy's first round checks them
-    // on the bases, overlapping the random base reads with its random proposals (LASAGNA_
-    // VERIFY=join: verified inside the join, A/B only; the round-1 greedy and the join-side
-    // claimed filter need verified pairs)
-    r.defer_verify = !old_greedy() && !join_filter() && !env_flag("LASAGNA_VERIFY", 'j');
+    // LASAGNA_VERIFY=greedy (R27): the join stores its fingerprint hits unverified and the
+    // greedy's first round checks them on the bases.  Measured the same at cfg3 (join 12.13 +
+    // greedy 11.70 vs 17.34 + 6.37 ms: the ~5 ms of random base reads cost the same in either
+    // kernel), so the default verifies inside the join, like the overlaps and multi-GPU paths.
+    // (The round-1 greedy and the join-side claimed filter need verified pairs.)
+    r.defer_verify = !old_greedy() && !join_filter() && env_flag("LASAGNA_VERIFY", 'g');
     if (r.defer_verify) {
         peers.vpacked = packed;
         peers.vL = L;

@@ -38,7 +38,8 @@ constexpr int RF_THREADS = 512;
 
 
 // exclusive scan of v over the first NB threads (NB a multiple of 32, <= 512); every thread of
-// the block must call it.  wsum: 16 shared words.
+// the block must call it.  wsum: 16 shared words.  The caller must pass a block barrier before
+// the next call (both callers do: their offsets are published with one right after).
 template <int NB>
 __device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t *wsum)
 {
@@ -54,7 +55,6 @@ __device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t *wsum)
     uint32_t add = 0;
     if (threadIdx.x < NB)
         for (int w = 0; w < warp; ++w) add += wsum[w];
-    __syncthreads();
     return x - v + add;
 }
 

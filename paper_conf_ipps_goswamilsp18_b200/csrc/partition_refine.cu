@@ -99,6 +99,7 @@ refine_kernel(RefineArgs a)
         if (threadIdx.x < nb) {
             lstart[threadIdx.x] = ex;
             const uint32_t run = running[threadIdx.x];
+            running[threadIdx.x] = run + c; // this thread's bin only: no barrier needed
             if ((uint64_t)run + c > a.cap_out) {
                 gofs[threadIdx.x] = -1;
                 *a.overflow = 1u;
@@ -124,9 +125,9 @@ refine_kernel(RefineArgs a)
             LSG_DCHECK(go < 0 || (uint64_t)(go + u) < (uint64_t)gridDim.x * nb * a.cap_out);
             if (go >= 0) a.out[go + u] = k;
         }
-        __syncthreads();
-        if (threadIdx.x < nb) running[threadIdx.x] += c;
-        __syncthreads();
+        // no barrier here: the next tile's first barrier (after its ranking, which touches only
+        // cnt and the other input buffer) orders these reads of rstage/gofs before they are
+        // rewritten, and this tile's buffer was last read before the staging barrier above
     }
     if (threadIdx.x < nb) {
         a.fill_out[r * nb + threadIdx.x] = running[threadIdx.x];

@@ -126,6 +126,26 @@ def test_exact_path_multipass(lz, cfg2, monkeypatch):
 
 
 @gpu
+@pytest.mark.parametrize("path,lpp,levels", [("", 0, ""), ("", 5, ""), ("", 5, "3"), ("exact", 5, "")])
+def test_verification_in_the_greedy(lz, cfg2, monkeypatch, path, lpp, levels):
+    """R27: with LASAGNA_VERIFY=greedy the join stores its fingerprint hits unverified and the
+    greedy's first round of each length checks them on the bases; the graph, |P| (counted
+    there) and the accepted pairs must equal the oracle on the two- and three-level and exact
+    paths, one and several length groups."""
+    import torch
+    cfg, reads, esucc, eolen, m, acc = cfg2
+    monkeypatch.setenv("LASAGNA_VERIFY", "greedy")
+    if path:
+        monkeypatch.setenv("LASAGNA_PATH", path)
+    if levels:
+        monkeypatch.setenv("LASAGNA_TEST_LEVELS", levels)
+    packed = lz.load_reads(torch.from_numpy(reads).cuda())
+    r = lz.greedy_graph(packed, cfg.n, cfg.L, cfg.l_min, lengths_per_pass=lpp)
+    assert r.stats["bucketed"] == (0 if path else 1)
+    _same(r, esucc, eolen, m, acc)
+
+
+@gpu
 @pytest.mark.parametrize("lpp,src", [(0, "packed"), (5, "packed"), (5, "pinned"), (3, "device")])
 def test_three_level_geometry(lz, cfg2, monkeypatch, lpp, src):
     """The cfg4/cfg5 geometry (three partition levels of 8, 8 and 4 bits: T = 20, 2^20 split
