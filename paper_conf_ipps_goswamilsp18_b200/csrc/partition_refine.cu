@@ -18,7 +18,7 @@ refine_kernel(RefineArgs a)
     uint64_t *rstage = rsm + 2 * RF_TILE; // [RF_TILE]
     __shared__ __align__(8) unsigned long long mbar[2];
     __shared__ uint32_t cnt[NBMAX], lstart[NBMAX], running[NBMAX], wsum[16];
-    __shared__ long long gofs[NBMAX];
+    __shared__ uint64_t *gdst[NBMAX]; // per bin: a.out + offset - first stage slot; nullptr = overflow
     const uint32_t nb = (1u << a.dbits) << (SPLIT ? 1 : 0);
     const uint32_t dmask = (1u << a.dbits) - 1u;
     auto binof = [&](uint64_t k) -> uint32_t {
@@ -101,11 +101,10 @@ refine_kernel(RefineArgs a)
             const uint32_t run = running[threadIdx.x];
             running[threadIdx.x] = run + c; // this thread's bin only: no barrier needed
             if ((uint64_t)run + c > a.cap_out) {
-                gofs[threadIdx.x] = -1;
+                gdst[threadIdx.x] = nullptr;
                 *a.overflow = 1u;
             } else {
-                gofs[threadIdx.x] =
-                    (long long)((r * nb + threadIdx.x) * a.cap_out + run) - (long long)ex;
+                gdst[threadIdx.x] = a.out + ((r * nb + threadIdx.x) * a.cap_out + run) - ex;
             }
         }
         __syncthreads();
@@ -121,12 +120,12 @@ refine_kernel(RefineArgs a)
 #pragma unroll 4
         for (uint32_t u = threadIdx.x; u < m; u += RF_THREADS) {
             const uint64_t k = rstage[u];
-            const long long go = gofs[binof(k)];
-            LSG_DCHECK(go < 0 || (uint64_t)(go + u) < (uint64_t)gridDim.x * nb * a.cap_out);
-            if (go >= 0) a.out[go + u] = k;
+            uint64_t *d = gdst[binof(k)];
+            LSG_DCHECK(!d || (uint64_t)(d + u - a.out) < (uint64_t)gridDim.x * nb * a.cap_out);
+            if (d) __stcg(d + u, k);
         }
         // no barrier here: the next tile's first barrier (after its ranking, which touches only
-        // cnt and the other input buffer) orders these reads of rstage/gofs before they are
+        // cnt and the other input buffer) orders these reads of rstage/gdst before they are
         // rewritten, and this tile's buffer was last read before the staging barrier above
     }
     if (threadIdx.x < nb) {
