@@ -26,9 +26,7 @@ scatter_table_kernel(ScatterArgs a)
     unsigned short *sbin = reinterpret_cast<unsigned short *>(stage + NT * KPT);
     __shared__ uint32_t cnt[NBIN], lstart[NBIN + 1], wsum[16];
     __shared__ uint32_t rbase[SPLIT ? 1 : 256]; // region of (segment 0, digit d); + s * nb_pad
-    // per bin: the destination of stage slot 0 (a.out + region offset - the bin's first stage
-    // slot, so slot u goes to gdst[bin] + u); nullptr = overflowed
-    __shared__ uint64_t *gdst[NBIN];
+    __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
 
     const uint64_t i = (uint64_t)blockIdx.x * NT + threadIdx.x;
     const bool valid = i < a.n;
@@ -162,10 +160,10 @@ scatter_table_kernel(ScatterArgs a)
                 const uint32_t bin = threadIdx.x * BPT + b;
                 lstart[bin] = run;
                 if ((uint64_t)bs[b] + c[b] > a.cap) {
-                    gdst[bin] = nullptr;
+                    gofs[bin] = -1;
                     *a.overflow = 1u;
                 } else {
-                    gdst[bin] = a.out + (rg[b] * a.cap + bs[b]) - run;
+                    gofs[bin] = (long long)(rg[b] * a.cap + bs[b]) - (long long)run;
                 }
                 run += c[b];
             }
@@ -184,9 +182,9 @@ scatter_table_kernel(ScatterArgs a)
             __syncthreads();
             const uint32_t total = lstart[NBIN];
             for (uint32_t u = threadIdx.x; u < total; u += NT) {
-                uint64_t *d = gdst[sbin[u]];
-                LSG_DCHECK(!d || (uint64_t)(d + u - a.out) < nreg * a.cap);
-                if (d) __stcg(d + u, stage[u]); // st.global (the pointer came from shared memory)
+                const long long go = gofs[sbin[u]];
+                LSG_DCHECK(go < 0 || (uint64_t)(go + u) < nreg * a.cap);
+                if (go >= 0) a.out[go + u] = stage[u];
             }
             // the next round's first barrier orders these reads before stage/lstart reuse
         }
