@@ -487,8 +487,14 @@ def main_streaming(args, cfg) -> None:
                    "ascii_gb": n * L / 1e9,
                    "table_set_gb": 8.0 * 2 * n * (L - l_min) / 1e9,
                    "l2": "inputs larger than L2 and than HBM"},
-        "overlap_edges_per_s": st["n_pairs"] / (ms_step / 1e3),
+        # overlap edges/s needs the UNPRUNED |P|; with several length groups the
+        # claimed-end pruning (f1) drops entries, so the count below is pairs found after it
+        "overlap_edges_per_s": (st["n_pairs"] / (ms_step / 1e3)
+                                if not st.get("pruned_entries") else None),
         "read_end_pairs": st["n_pairs"], "greedy_pairs": st["n_greedy"],
+        "pairs_note": ("read_end_pairs = pairs found after claimed-end pruning (f1: %d entries "
+                       "pruned); the full |P| needs LASAGNA_NO_PRUNE=1" % st["pruned_entries"])
+                      if st.get("pruned_entries") else "read_end_pairs = |P| (no pruning)",
         "fp_false_matches": st["fp_false_matches"], "greedy_rounds_max": st["rounds_max"],
         "e2e": {"value": n / (e2e_ms / 1e3), "unit": "reads/s", "ms_per_step": e2e_ms,
                 "h2d_bytes_per_step": n * L, "d2h_bytes_per_step": 2 * n * 5,

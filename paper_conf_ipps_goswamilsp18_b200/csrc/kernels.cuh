@@ -148,6 +148,7 @@ struct BucketJoinArgs {
     const uint32_t *fills;    // [n_buckets][2]
     uint64_t half_cap, n_buckets;
     uint32_t *overflow;
+    bool planner_builds = false; // A/B: the planning warp takes a build share too
 };
 lasagna_status launch_bucket_join(const BucketJoinArgs &a, cudaStream_t s); // block windows
 lasagna_status launch_warp_join(const BucketJoinArgs &a, cudaStream_t s);   // warp per bucket

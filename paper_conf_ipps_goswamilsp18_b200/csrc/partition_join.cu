@@ -206,8 +206,13 @@ bucket_join_kernel(BucketJoinArgs b)
                 const uint32_t tag = epoch << 16;
                 const uint32_t nP = d.nP, nS = d.nS;
                 // ---- build: chained hash of the build entries + the 64 Ki-bit filter
+                // the planner warp (which planned the next window just before) sits the build
+                // out unless LASAGNA_BJ_PLANNER_BUILDS: its share would make every other warp wait
+                // at the barrier below
+                const uint32_t nbuild = b.planner_builds ? BJ_THREADS : BJ_THREADS - 32;
+                const uint32_t kb0 = (b.planner_builds || !planner) ? threadIdx.x : nP;
 #pragma unroll 2
-                for (uint32_t k2 = threadIdx.x; k2 < nP; k2 += BJ_THREADS) {
+                for (uint32_t k2 = kb0; k2 < nP; k2 += nbuild) {
                     const uint64_t e = P[k2];
                     if (e & tagbit) continue; // sentinel
                     if (e & flag2bit) s_has2[w] = 1u; // a flag-2 entry also probes (rare)
@@ -307,9 +312,15 @@ lasagna_status launch_bucket_join(const BucketJoinArgs &args, cudaStream_t s)
     if (args.half_cap & 1) return LASAGNA_EINVAL; // sentinels need an even half capacity
     // CTA geometry: one 1024-thread CTA per SM (512 x 2 and 256 x 4 per SM with proportionally
     // smaller windows measured the same at cfg3: DESIGN.md 6.1)
+    static const bool planner_builds = [] {
+        const char *e = getenv("LASAGNA_BJ_PLANNER_BUILDS");
+        return e && e[0] == '1';
+    }();
+    BucketJoinArgs a = args;
+    a.planner_builds = planner_builds;
     return dispatch_W(args.j.L, [&](auto wc) -> lasagna_status {
         constexpr int W = decltype(wc)::value;
-        return launch_bucket_join_cfg<W, BjCfg<1024, 4096, 4096, 2048>>(args, s);
+        return launch_bucket_join_cfg<W, BjCfg<1024, 4096, 4096, 2048>>(a, s);
     });
 }
 
