@@ -209,10 +209,40 @@ __device__ __forceinline__ void fp_absorb(const uint64_t (&x)[W], const uint64_t
     st.P0 = fold61(P0), st.P1 = fold61(P1), st.S0 = fold61(S0), st.S1 = fold61(S1);
 }
 
+// Table-driven chunk values: the four 2-bit codes of a byte (code i at bits 2i..2i+1) as a
+// base-5 number, code 0 most significant (forward Horner) or least significant (ascending
+// powers).  A kernel fills the 256-entry tables into shared memory once (Base5Tabs); an
+// 8-base chunk is then two byte extracts, two lookups and one multiply-add instead of eight
+// shift/mask/multiply-add steps.
+__host__ __device__ constexpr uint32_t base5_fwd(uint32_t b)
+{
+    return (b & 3u) * 125u + ((b >> 2) & 3u) * 25u + ((b >> 4) & 3u) * 5u + ((b >> 6) & 3u);
+}
+__host__ __device__ constexpr uint32_t base5_bwd(uint32_t b)
+{
+    return (b & 3u) + ((b >> 2) & 3u) * 5u + ((b >> 4) & 3u) * 25u + ((b >> 6) & 3u) * 125u;
+}
+struct Base5Tabs {
+    const unsigned short *fwd, *bwd; // shared memory, 256 entries each
+};
+__device__ __forceinline__ uint32_t byte_k(uint32_t h, uint32_t k) // byte k of h, zero-extended
+{
+    return __byte_perm(h, 0u, 0x4440u + k);
+}
+// chunk8_fwd / chunk8_bwd of the 8 bases in bytes k, k+1 of h (k = 0: low half, 2: high half)
+__device__ __forceinline__ uint32_t chunk8_fwd_t(const Base5Tabs &t, uint32_t h, uint32_t k)
+{
+    return (uint32_t)t.fwd[byte_k(h, k)] * 625u + t.fwd[byte_k(h, k + 1u)];
+}
+__device__ __forceinline__ uint32_t chunk8_bwd_t(const Base5Tabs &t, uint32_t h, uint32_t k)
+{
+    return (uint32_t)t.bwd[byte_k(h, k + 1u)] * 625u + t.bwd[byte_k(h, k)];
+}
+
 // fp_absorb modulo 2^64 (the key streams of the bucketed path, R26)
 template <int W>
 __device__ __forceinline__ void fp64_absorb(const uint64_t (&x)[W], const uint64_t (&y)[W],
-                                          uint32_t nb, Fp64Streams &st)
+                                          uint32_t nb, Fp64Streams &st, const Base5Tabs &tb)
 {
     const uint32_t nh = nb >> 4, rem = nb & 15u;
     uint64_t P0 = 0, P1 = 0, S0 = 0, S1 = 0;
@@ -221,10 +251,10 @@ __device__ __forceinline__ void fp64_absorb(const uint64_t (&x)[W], const uint64
         if ((uint32_t)h >= nh) break;
         const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1)));
         const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1)));
-        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd(hx);
-        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd(hx >> 16);
-        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd(hy);
-        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd(hy >> 16);
+        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd_t(tb, hx, 0);
+        P0 = (P0) * (uint64_t)(POW5_8) + chunk8_fwd_t(tb, hx, 2);
+        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd_t(tb, hy, 0);
+        P1 = (P1) * (uint64_t)(POW5_8) + chunk8_fwd_t(tb, hy, 2);
     }
     // the partial half-word nh (bases 16 nh .. 16 nh + rem - 1), rem < 16
     uint32_t px = 0, py = 0;
@@ -260,10 +290,10 @@ __device__ __forceinline__ void fp64_absorb(const uint64_t (&x)[W], const uint64
         if ((uint32_t)h >= nh) continue;
         const uint32_t hx = (uint32_t)(x[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
         const uint32_t hy = (uint32_t)(y[h >> 1] >> (32 * (h & 1))) ^ 0xAAAAAAAAu;
-        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd(hx >> 16);
-        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd(hx);
-        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd(hy >> 16);
-        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd(hy);
+        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd_t(tb, hx, 2);
+        S1 = (S1) * (uint64_t)(POW5_8) + chunk8_bwd_t(tb, hx, 0);
+        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd_t(tb, hy, 2);
+        S0 = (S0) * (uint64_t)(POW5_8) + chunk8_bwd_t(tb, hy, 0);
     }
     st.P0 = P0, st.P1 = P1, st.S0 = S0, st.S1 = S1;
 }

@@ -28,6 +28,12 @@ scatter_table_kernel(ScatterArgs a)
     __shared__ uint32_t rbase[SPLIT ? 1 : 256]; // region of (segment 0, digit d); + s * nb_pad
     __shared__ long long gofs[NBIN]; // per bin: element offset of stage slot 0's destination, -1 = overflow
 
+    __shared__ unsigned short s_b5f[256], s_b5b[256]; // base-5 byte tables (fingerprint.cuh)
+    for (uint32_t t = threadIdx.x; t < 256; t += NT) {
+        s_b5f[t] = (unsigned short)base5_fwd(t);
+        s_b5b[t] = (unsigned short)base5_bwd(t);
+    }
+    // (visible to the prologue: the barriers below precede fp64_absorb)
     const uint64_t i = (uint64_t)blockIdx.x * NT + threadIdx.x;
     const bool valid = i < a.n;
     uint64_t x[W], y[W];
@@ -77,7 +83,7 @@ scatter_table_kernel(ScatterArgs a)
 #endif
     Fp64Streams st; // key streams modulo 2^64 (R26)
     // the l_lo - 1 bases before the first emitted length, absorbed in 8-base chunks
-    fp64_absorb<W>(x, y, a.l_lo - 1u, st);
+    fp64_absorb<W>(x, y, a.l_lo - 1u, st, Base5Tabs{s_b5f, s_b5b});
     // Base cursors over x (y is dead from here): tx holds base k of r in its low bits; ty
     // holds base L-1-k of r in its top bits, i.e. base k of r' = RC(r) complemented.  A word
     // boundary reloads a cursor from x with a register select (block-uniform branch).
