@@ -187,7 +187,6 @@ scatter_table_kernel(ScatterArgs a)
             }
             __syncthreads();
             const uint32_t total = lstart[NBIN];
-#pragma unroll 4
             for (uint32_t u = threadIdx.x; u < total; u += NT) {
                 const long long go = gofs[sbin[u]];
                 LSG_DCHECK(go < 0 || (uint64_t)(go + u) < nreg * a.cap);
