@@ -623,7 +623,10 @@ def main() -> None:
 
     del dev_ascii, runner
     torch.cuda.empty_cache()
-    pipe = lz.GraphPipeline(n, L, l_min, dev, args.lengths_per_pass)
+    # batches streamed from page-locked host memory inside each call (BENCH_PIPE_COPY=1: the
+    # whole batch copied to a device buffer first, A/B)
+    pipe = lz.GraphPipeline(n, L, l_min, dev, args.lengths_per_pass,
+                            stream_input=os.environ.get("BENCH_PIPE_COPY") != "1")
     outs = [(torch.zeros(2 * n, dtype=torch.int32).pin_memory(),
              torch.empty(2 * n, dtype=torch.uint8).pin_memory()) for _ in range(2)]
 
@@ -665,6 +668,7 @@ def main() -> None:
         "e2e": {"value": n / (e2e_ms / 1e3), "unit": "reads/s", "ms_per_step": e2e_ms,
                 "h2d_bytes_per_step": n * L, "d2h_bytes_per_step": 2 * n * 5,
                 "batches_in_flight": 2, "serial_ms_per_step": e2e_serial_ms,
+                "pipeline_input": "streamed" if pipe.stream_input else "device copy",
                 "serial_value": n / (e2e_serial_ms / 1e3)},
         "roofline": roof,
         "clocks": clocks,

@@ -334,12 +334,19 @@ class GraphPipeline:
     Plumbing only: every step of the path runs in liblasagna.so (lasagna_greedy_graph_ascii on
     the device copy of the batch)."""
 
-    def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0):
+    def __init__(self, n: int, L: int, l_min: int, device="cuda", lengths_per_pass: int = 0,
+                 stream_input: bool = False):
+        """stream_input: each runner reads its batch straight from page-locked host memory
+        (lasagna_greedy_graph_ascii's chunked DMA, the scatter of chunk c running while chunk
+        c+1 lands), so a batch's fingerprint/partition pass overlaps its own copy and no device
+        input buffers are held; otherwise the batch is first copied whole to a device buffer."""
         dev = torch.device(device)
         if dev.index is None:  # the worker threads select the device by index
             dev = torch.device(dev.type, torch.cuda.current_device())
         self.n, self.L, self.device = n, L, dev
-        self.bufs = [torch.empty((n, L), dtype=torch.uint8, device=self.device) for _ in range(2)]
+        self.stream_input = stream_input
+        self.bufs = [] if stream_input else [
+            torch.empty((n, L), dtype=torch.uint8, device=self.device) for _ in range(2)]
         # the two runners share what is free after the input buffers: half each, less what a
         # runner holds besides its workspace
         free, _ = torch.cuda.mem_get_info(self.device)
@@ -367,10 +374,13 @@ class GraphPipeline:
                         if item is None:
                             return
                         ev, k = item
-                        # wait on the host, not in-stream: a stream parked on an event wait can
-                        # hold a hardware queue that the other lane's kernels share
-                        ev.synchronize()
-                        r = self.runners[j].from_ascii(self.bufs[j], stats=False)
+                        if self.stream_input:  # chunked DMA from the host batch inside the call
+                            r = self.runners[j].from_ascii(batches[k], stats=False)
+                        else:
+                            # wait on the host, not in-stream: a stream parked on an event wait
+                            # can hold a hardware queue that the other lane's kernels share
+                            ev.synchronize()
+                            r = self.runners[j].from_ascii(self.bufs[j], stats=False)
                         outs[k][0].copy_(r.succ, non_blocking=True)
                         outs[k][1].copy_(r.olen, non_blocking=True)
                         self.lanes[j].synchronize()
@@ -388,6 +398,9 @@ class GraphPipeline:
                 free[j].acquire()  # runner j's previous batch has returned
                 if errors:
                     break
+                if self.stream_input:
+                    q[j].put((None, k))
+                    continue
                 self.copy.wait_stream(self.lanes[j])
                 with torch.cuda.stream(self.copy):
                     self.bufs[j].copy_(b, non_blocking=True)

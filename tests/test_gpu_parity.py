@@ -474,14 +474,17 @@ def test_region_overflow_falls_back_to_exact_path(tmp_path):
 
 
 @gpu
-def test_graph_pipeline_batches():
-    """GraphPipeline (two batches in flight, host -> device copy of batch k+1 overlapping batch
-    k): five different read batches, each result equal to the oracle's for that batch."""
+@pytest.mark.parametrize("n,stream_input", [(60_000, False), (60_000, True), (400_000, True)])
+def test_graph_pipeline_batches(n, stream_input):
+    """GraphPipeline (two batches in flight; batch k+1's host -> device copy overlapping batch
+    k, either whole into a device buffer or streamed in chunks inside the call): five different
+    read batches, each result equal to the oracle's for that batch (400 K reads: the two-level
+    path, whose scatter consumes the DMA chunks as they land)."""
     import torch
     import paper_conf_ipps_goswamilsp18_b200 as lz
-    n, L, l_min = 60_000, 100, 63
-    batches = [readgen.reads(100 + k, 300_000, n, L, 0.01) for k in range(5)]
-    pipe = lz.GraphPipeline(n, L, l_min, "cuda")
+    L, l_min = 100, 63
+    batches = [readgen.reads(100 + k, 5 * n, n, L, 0.01) for k in range(5)]
+    pipe = lz.GraphPipeline(n, L, l_min, "cuda", stream_input=stream_input)
     hb = [torch.from_numpy(b).pin_memory() for b in batches]
     outs = [(torch.empty(2 * n, dtype=torch.int32).pin_memory(),
              torch.empty(2 * n, dtype=torch.uint8).pin_memory()) for _ in batches]
