@@ -139,15 +139,11 @@ lasagna_status launch_refine(const RefineArgs &args, uint64_t n_regions, cudaStr
     if (n_regions == 0) return LASAGNA_OK;
     if (args.dbits < 1 || args.dbits > 8) return LASAGNA_EINVAL;
     if (args.n_src < 1 || args.n_src > MAX_REFINE_SRC) return LASAGNA_EINVAL;
-    // tile of 16 keys per thread (one 512-thread CTA per SM, measured faster than 8 keys at
-    // two CTAs per SM: 22 vs 30 ms at cfg3); LASAGNA_RF_KPT=8 selects the smaller tile
-    static const int kpt = [] {
-        const char *e = getenv("LASAGNA_RF_KPT");
-        return (e && atoi(e) == 8) ? 8 : 16;
-    }();
+    // tile of 16 keys per thread, one 512-thread CTA per SM (8-key tiles at two CTAs per SM
+    // measured 15.0 vs 11.0 ms at cfg3: DESIGN.md 6.1, r02g)
+    constexpr int kpt = 16;
     const size_t smem = (size_t)3 * RF_THREADS * kpt * 8;
-    auto kern = kpt == 16 ? (args.split ? refine_kernel<true, 16> : refine_kernel<false, 16>)
-                          : (args.split ? refine_kernel<true, 8> : refine_kernel<false, 8>);
+    auto kern = args.split ? refine_kernel<true, kpt> : refine_kernel<false, kpt>;
     LSG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     kern<<<(unsigned)n_regions, RF_THREADS, smem, s>>>(args);
     LSG_LAUNCHED("refine_kernel");

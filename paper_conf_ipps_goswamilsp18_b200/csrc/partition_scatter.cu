@@ -216,20 +216,8 @@ lasagna_status launch_scatter_table(const ScatterArgs &args, cudaStream_t s)
         if (args.split)
             return args.ascii ? run(scatter_table_kernel<W, true, true, 1>, 1, SC_THREADS)
                               : run(scatter_table_kernel<W, false, true, 1>, 1, SC_THREADS);
-        if constexpr (W == 4) {
-            // CTA geometry A/B (LASAGNA_SC): 1 = 256 reads x 3 CTAs per SM (80 registers),
-            // 2 = 512 reads x 1 (128 registers)
-            static const int v = [] {
-                const char *e = getenv("LASAGNA_SC");
-                return e ? atoi(e) : 0;
-            }();
-            if (v == 1)
-                return args.ascii ? run(scatter_table_kernel<W, true, false, 4, 256, 3>, 4, 256)
-                                  : run(scatter_table_kernel<W, false, false, 4, 256, 3>, 4, 256);
-            if (v == 2)
-                return args.ascii ? run(scatter_table_kernel<W, true, false, 4, 512, 1>, 4, 512)
-                                  : run(scatter_table_kernel<W, false, false, 4, 512, 1>, 4, 512);
-        }
+        // CTA geometry: 512 reads x 2 CTAs per SM at the 64-register cap; 256 x 3 (80 registers)
+        // and 512 x 1 (128 registers) measured 20-25 % slower (r02e)
         return args.ascii ? run(scatter_table_kernel<W, true, false, 4>, 4, SC_THREADS)
                           : run(scatter_table_kernel<W, false, false, 4>, 4, SC_THREADS);
     });
