@@ -478,7 +478,7 @@ lasagna_status greedy_length_peers(const GreedyPeers &p, uint8_t l, cudaStream_t
     // blocks per SM of the first round (the whole pool) and of the later rounds (survivors);
     // LASAGNA_GREEDY_BPS=a,b overrides (A/B only)
     static const std::pair<uint32_t, uint32_t> bps = [] {
-        uint32_t a0 = 16, a1 = 16;
+        uint32_t a0 = 8, a1 = 4; // first round: 8 blocks per SM, later rounds 4 (r02t A/B)
         if (const char *e = getenv("LASAGNA_GREEDY_BPS")) sscanf(e, "%u,%u", &a0, &a1);
         return std::make_pair(std::max(1u, a0), std::max(1u, a1));
     }();
